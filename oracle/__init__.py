@@ -1,0 +1,189 @@
+"""Oracle loader -- TEST INFRASTRUCTURE ONLY.
+
+ctypes binding of ``oracle/oracle.c``, the plain single-threaded CPU reference of the
+tracking hot path (see oracle.h for the contract and citations).  Only ``tests/``,
+``__graft_entry__.smoke()`` and ``bench.py`` (cpu_baseline leg, ``--impl reference``) may
+import this module.  It imports nothing from the CUDA package and the CUDA package
+imports nothing from here.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+import threading
+from typing import Optional
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "oracle.c")
+_HDR = os.path.join(_HERE, "oracle.h")
+_LIB = os.path.join(_HERE, "liboracle.so")
+CFLAGS = ["-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared",
+          "-Wall", "-Wextra"]
+
+END_MASK, END_CURV, END_MAXLEN = 0, 1, 2
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so with gcc (no FMA contraction, no fast-math)."""
+    stale = (not os.path.exists(_LIB) or
+             os.path.getmtime(_LIB) < max(os.path.getmtime(_SRC), os.path.getmtime(_HDR)))
+    if force or stale:
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+class _Volume(ctypes.Structure):
+    _fields_ = [("nx", ctypes.c_int32), ("ny", ctypes.c_int32), ("nz", ctypes.c_int32),
+                ("nsamples", ctypes.c_int32), ("nfibres", ctypes.c_int32),
+                ("is_half", ctypes.c_int32), ("dyads", ctypes.c_void_p),
+                ("f", ctypes.c_void_p), ("mask", ctypes.c_void_p)]
+
+
+class _Params(ctypes.Structure):
+    _fields_ = [("step", ctypes.c_float), ("curv_thr", ctypes.c_float),
+                ("fib_thr", ctypes.c_float), ("max_steps", ctypes.c_int32),
+                ("rng_seed", ctypes.c_uint64), ("particles_per_seed", ctypes.c_int64)]
+
+
+_lib = None
+_lock = threading.Lock()
+
+
+def lib():
+    global _lib
+    with _lock:
+        if _lib is None:
+            L = ctypes.CDLL(build())
+            vp = ctypes.c_void_p
+            L.oracle_philox4x32_10.argtypes = [vp, vp, vp]
+            L.oracle_half_to_float.argtypes = [ctypes.c_uint16]
+            L.oracle_half_to_float.restype = ctypes.c_float
+            L.oracle_half_to_float_array.argtypes = [vp, vp, ctypes.c_int64]
+            L.oracle_axis_index.argtypes = [ctypes.c_float, ctypes.c_int32]
+            L.oracle_axis_index.restype = ctypes.c_int64
+            L.oracle_sample_index.argtypes = [ctypes.c_uint32, ctypes.c_uint32]
+            L.oracle_sample_index.restype = ctypes.c_uint32
+            L.oracle_track.argtypes = [ctypes.POINTER(_Volume), ctypes.POINTER(_Params), vp, vp,
+                                       ctypes.c_int64, ctypes.c_int64, ctypes.c_int64,
+                                       vp, vp, vp, vp, vp, ctypes.c_int32]
+            L.oracle_track.restype = ctypes.c_int
+            _lib = L
+    return _lib
+
+
+def _ptr(a: Optional[np.ndarray]):
+    return None if a is None else a.ctypes.data
+
+
+# ----------------------------------------------------------------------------- primitives
+
+def philox(ctr, key) -> np.ndarray:
+    c = np.ascontiguousarray(ctr, np.uint32)
+    k = np.ascontiguousarray(key, np.uint32)
+    out = np.zeros(4, np.uint32)
+    lib().oracle_philox4x32_10(c.ctypes.data, k.ctypes.data, out.ctypes.data)
+    return out
+
+
+def half_to_float(bits: np.ndarray) -> np.ndarray:
+    b = np.ascontiguousarray(bits, np.uint16)
+    out = np.empty(b.shape, np.float32)
+    lib().oracle_half_to_float_array(b.ctypes.data, out.ctypes.data, b.size)
+    return out
+
+
+def axis_index(q: float, n_axis: int) -> int:
+    return int(lib().oracle_axis_index(ctypes.c_float(q), n_axis))
+
+
+def sample_index(w: int, nsamples: int) -> int:
+    return int(lib().oracle_sample_index(w, nsamples))
+
+
+# ----------------------------------------------------------------------------- tracking
+
+def _structs(volume, step, curv_thr, fib_thr, max_steps, rng_seed, P):
+    v = volume
+    vs = _Volume(v.nx, v.ny, v.nz, v.nsamples, v.nfibres, 1 if v.dyads.dtype == np.float16 else 0,
+                 v.dyads.ctypes.data, v.f.ctypes.data, v.mask.ctypes.data)
+    ps = _Params(step, curv_thr, fib_thr, max_steps, rng_seed, P)
+    return vs, ps
+
+
+def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = True,
+          want_particles: bool = True, path_stride: int = 0, threads: int = 1) -> dict:
+    """Run the oracle on workload ``w`` (a phantom.Workload or duck-typed equivalent).
+
+    Returns dict(map=uint64[Z][Y][X] or None, nsteps=int32[n], reason=uint8[n],
+    end=float32[n][3], paths=float32[n][path_stride][3] or None), particles ordered
+    (seed index, j).  ``threads`` > 1 runs independent single-threaded oracle calls on
+    disjoint seed shards (seed i -> worker i mod threads) and sums their maps.
+    """
+    v = w.volume
+    P = int(w.particles_per_seed)
+    j_end = P if j_end is None else int(j_end)
+    npp = j_end - j_begin
+    seeds = np.ascontiguousarray(w.seeds, np.float32)
+    ids = np.ascontiguousarray(w.ids(), np.uint64)
+    ns = seeds.shape[0]
+    n = ns * npp
+    vs, ps = _structs(v, w.step, w.curv_thr, w.fib_thr, w.max_steps, w.rng_seed, P)
+    nsteps = np.zeros(n, np.int32) if want_particles else None
+    reason = np.zeros(n, np.uint8) if want_particles else None
+    end = np.zeros((n, 3), np.float32) if want_particles else None
+    paths = np.zeros((n, path_stride, 3), np.float32) if path_stride > 0 else None
+    L = lib()
+    threads = max(1, min(int(threads), ns)) if ns else 1
+
+    def run(shard: np.ndarray, mp: Optional[np.ndarray]):
+        sd = np.ascontiguousarray(seeds[shard])
+        si = np.ascontiguousarray(ids[shard])
+        m = len(shard) * npp
+        ln = np.zeros(m, np.int32) if want_particles else None
+        lr = np.zeros(m, np.uint8) if want_particles else None
+        le = np.zeros((m, 3), np.float32) if want_particles else None
+        lp = np.zeros((m, path_stride, 3), np.float32) if paths is not None else None
+        rc = L.oracle_track(ctypes.byref(vs), ctypes.byref(ps), sd.ctypes.data, si.ctypes.data,
+                            len(shard), j_begin, j_end, _ptr(mp), _ptr(ln), _ptr(lr), _ptr(le),
+                            _ptr(lp), path_stride)
+        if rc != 0:
+            raise ValueError(f"oracle_track rejected its arguments (rc={rc})")
+        return ln, lr, le, lp
+
+    maps = [np.zeros((v.nz, v.ny, v.nx), np.uint64) if want_map else None for _ in range(threads)]
+    shards = [np.arange(t, ns, threads) for t in range(threads)]
+    results = [None] * threads
+    if threads == 1:
+        results[0] = run(shards[0], maps[0])
+    else:
+        def worker(t):
+            results[t] = run(shards[t], maps[t])
+        th = [threading.Thread(target=worker, args=(t,)) for t in range(threads)]
+        for t in th:
+            t.start()
+        for t in th:
+            t.join()
+        if any(r is None for r in results):
+            raise RuntimeError("oracle worker failed")
+    for t, shard in enumerate(shards):
+        ln, lr, le, lp = results[t]
+        if len(shard) == 0:
+            continue
+        rows = (shard[:, None] * npp + np.arange(npp)[None, :]).ravel()
+        if want_particles:
+            nsteps[rows] = ln
+            reason[rows] = lr
+            end[rows] = le
+        if paths is not None:
+            paths[rows] = lp
+    mp = None
+    if want_map:
+        mp = maps[0]
+        for m in maps[1:]:
+            mp += m
+    return dict(map=mp, nsteps=nsteps, reason=reason, end=end, paths=paths)

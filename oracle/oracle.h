@@ -1,0 +1,75 @@
+/*
+ * oracle.h -- TEST INFRASTRUCTURE ONLY.
+ *
+ * Plain, slow, single-threaded CPU reference of the probabilistic-streamlining hot path
+ * of Xu et al., "Probabilistic Brain Fiber Tractography on GPUs" (IPDPSW 2012).
+ * Only tests/, __graft_entry__.smoke() and bench.py (cpu_baseline leg and
+ * --impl reference) may load it.  It shares no code, header or constant with the CUDA
+ * path (paper_conf_ipps_xuzwrwxgxy12_b200/csrc, include/pt.h) and includes neither.
+ *
+ * Citations: P:Lnnn = line nnn of the paper text; Rnn = a reading of the
+ * paper recorded in DESIGN.md "Readings".
+ */
+#ifndef ORACLE_H
+#define ORACLE_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Input volume in the canonical layout (Fig. 1: per-voxel sample volumes
+ * of the fibre directions and fractions; directions given as Cartesian vectors, R20).
+ *   dyads [F][S][Z][Y][X][3]  (x fastest, xyz innermost)
+ *   f     [F][S][Z][Y][X]
+ *   mask  [Z][Y][X]           (!= 0 inside)
+ * is_half = 0: float32 values; 1: IEEE binary16 bit patterns (uint16). */
+typedef struct {
+    int32_t nx, ny, nz, nsamples, nfibres;
+    int32_t is_half;
+    const void* dyads;
+    const void* f;
+    const uint8_t* mask;
+} oracle_volume;
+
+/* step: step length in voxels (R3); curv_thr: continue iff |dot| > curv_thr (R4,
+ * P:L117); fib_thr: fibre eligibility f_j > fib_thr (R7); max_steps (R14);
+ * rng_seed: Philox key (R16); particles_per_seed P: pid = seed_id * P + j. */
+typedef struct {
+    float step, curv_thr, fib_thr;
+    int32_t max_steps;
+    uint64_t rng_seed;
+    int64_t particles_per_seed;
+} oracle_params;
+
+enum { ORACLE_END_MASK = 0, ORACLE_END_CURV = 1, ORACLE_END_MAXLEN = 2 };
+
+/* Philox4x32-10 (R16): one block, ctr[4], key[2] -> out[4]. */
+void oracle_philox4x32_10(const uint32_t ctr[4], const uint32_t key[2], uint32_t out[4]);
+/* binary16 -> float32, exact (R15). */
+float oracle_half_to_float(uint16_t h);
+void oracle_half_to_float_array(const uint16_t* h, float* out, int64_t n);
+/* voxel index along one axis for a centred coordinate q (R10). */
+int64_t oracle_axis_index(float q, int32_t n_axis);
+/* sample index for a 32-bit word (R16): floor(w * S / 2^32). */
+uint32_t oracle_sample_index(uint32_t w, uint32_t nsamples);
+
+/* Track particles j in [j_begin, j_end) of every seed (Alg. 1 P:L159-187 inner loop with
+ * the semantics of P:L98-121; contract "C-ALG" in DESIGN.md).
+ *   seeds_xyz [nseeds][3] corner coordinates; seed_ids [nseeds] (NULL => 0..nseeds-1)
+ *   map       [Z][Y][X] uint64, accumulated (+=) ; may be NULL
+ *   nsteps, reason, end_xyz: per particle, index (seed_index*(j_end-j_begin) + j-j_begin);
+ *                            each may be NULL
+ *   paths     [particle][path_stride][3] corner-coordinate positions, point 0 = start,
+ *             point k = after the k-th committed step, unused points = NaN; may be NULL
+ * Returns 0 on success, <0 on invalid arguments (nothing written). */
+int oracle_track(const oracle_volume* vol, const oracle_params* prm,
+                 const float* seeds_xyz, const uint64_t* seed_ids, int64_t nseeds,
+                 int64_t j_begin, int64_t j_end,
+                 uint64_t* map, int32_t* nsteps, uint8_t* reason, float* end_xyz,
+                 float* paths, int32_t path_stride);
+
+#ifdef __cplusplus
+}
+#endif
+#endif
