@@ -1,0 +1,406 @@
+"""bench.py -- streamline steps/s of the B200 tracking hot path (BASELINE.json metric).
+
+Default workload: BASELINE.json configs[2], the whole-brain-shaped phantom (128x128x70,
+50 samples x 2 fibres, all WM seeds x 5000 particles, step 0.5, curvature 0.2, max 2000
+steps), synthetic (phantom.whole_brain).  A "step" of this bench is one pass of the whole
+hot path over that workload: pt_track (repacked records already resident, the persistent
+tracking kernel, the map-sum overflow check) and, for N > 1, the NCCL reduce of the maps.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config c3]
+
+For N > 1 run under torchrun (one rank per GPU, seeds sharded i mod N, global seed ids).
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+METRIC = "streamline steps/sec (and seeds/sec) at 1/2/4/8 B200; % of gather roofline"
+CONFIG_TEXT = {
+    "c3": "configs[2]: 128x128x70 whole-brain-shaped synthetic volume, 50 samples x 2 fibres, "
+          "all WM seeds x 5000 particles, step 0.5 vox, curvature 0.2, max 2000 steps, fp32 records",
+    "c4": "configs[3]: c3 with fp16 packed sample vectors (generator-rounded halves)",
+    "c2": "configs[1]: 64x64x32 two-bundle 90deg crossing, 50 samples x 2 fibres, 1k seeds x 5000",
+    "c2_dispersed": "configs[1] shape, dispersed (sigma 0.15, f jitter 0.03)",
+    "c1": "configs[0]: 32x32x16 straight tube, 64 seeds x 1000",
+}
+
+
+def _env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+# ----------------------------------------------------------------------------- clocks
+
+class ClockSampler:
+    """nvidia-smi sampling DURING the timed region (B200_PROFILING.md clocks line)."""
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+        self.thread = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except (OSError, ValueError):
+            self.proc = None
+            return
+        self.thread = threading.Thread(target=self._read, daemon=True)
+        self.thread.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        if self.thread:
+            self.thread.join(timeout=2)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        sm.sort()
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": max(mx), "samples": len(sm),
+                "reasons": sorted(reasons)}
+
+
+# ----------------------------------------------------------------------------- helpers
+
+def _peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except (OSError, ValueError):
+        return None
+
+
+def _ncu_traffic(cfg):
+    """dram bytes per launch of the tracking kernel from the committed ncu --set full
+    summary (profiles/), or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_track_summary.json")
+    try:
+        d = json.load(open(p))
+        e = d.get("per_config", {}).get(cfg) or {}
+        return e.get("dram_bytes_per_launch")
+    except (OSError, ValueError):
+        return None
+
+
+def _workload(cfg):
+    import phantom
+    return phantom.config(cfg)
+
+
+def _shard(w, rank, world):
+    import numpy as np
+    if world == 1:
+        return w
+    sel = np.arange(rank, w.nseeds, world)
+    return w.replace(seeds=w.seeds[sel].copy(), seed_ids=w.ids()[sel].copy())
+
+
+def _cpu_sample(w, target_s: float, threads: int):
+    """Oracle on a bounded sample of workload w: every k-th seed x particles j < J, sized
+    from a calibration run so the whole sample takes ~target_s of wall time on `threads`
+    host threads.  Returns (steps/s, description, steps, seconds, sample workload, J)."""
+    import oracle
+    import phantom
+    cal = phantom.wm_seeds(w, every=max(1, w.nseeds // 64))
+    t = time.perf_counter()
+    r = oracle.track(cal, 0, 20, want_map=False)
+    dt = time.perf_counter() - t
+    rate1 = max(1.0, r["nsteps"].sum() / max(dt, 1e-6))          # steps/s on one core
+    mean_len = max(1.0, float(r["nsteps"].mean()))
+    particles = target_s * rate1 * threads / mean_len
+    J = int(min(w.particles_per_seed, max(8, particles / max(1, threads * 32))))
+    nseeds = int(max(threads, min(w.nseeds, particles / J)))
+    every = max(1, w.nseeds // nseeds)
+    sub = phantom.wm_seeds(w, every=every)
+    return sub, J, every
+
+
+def _run_oracle_sample(sub, J, threads):
+    import oracle
+    t = time.perf_counter()
+    r = oracle.track(sub, 0, J, want_map=True, threads=threads)
+    dt = time.perf_counter() - t
+    return int(r["nsteps"].sum()), dt
+
+
+# ----------------------------------------------------------------------------- reference arm
+
+def run_reference(args):
+    rank = _env_int("RANK", 0)
+    if rank != 0:
+        return 0
+    import oracle
+    oracle.build()
+    w = _workload(args.config)
+    threads = len(os.sched_getaffinity(0))
+    sub, J, every = _cpu_sample(w, args.cpu_seconds, threads)
+    for _ in range(args.warmup):
+        _run_oracle_sample(sub, J, threads)
+    steps = 0
+    secs = 0.0
+    for _ in range(args.steps):
+        s, dt = _run_oracle_sample(sub, J, threads)
+        steps += s
+        secs += dt
+    v = steps / secs
+    desc = (f"{args.config}: every {every}th WM seed ({sub.nseeds} seeds) x particles j<{J} of "
+            f"{w.particles_per_seed}; oracle single-threaded per worker, {threads} worker threads")
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "steps/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / args.steps,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic", "config": {"workload": CONFIG_TEXT.get(args.config, args.config),
+                                        "sample": desc},
+        "cpu_baseline": {"value": v, "unit": "steps/s", "cores": threads, "kind": "oracle",
+                         "sample": desc},
+        "e2e": {"value": v, "unit": "steps/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ----------------------------------------------------------------------------- our arm
+
+def run_ours(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_xuzwrwxgxy12_b200 as pt
+
+    world = _env_int("WORLD_SIZE", 1)
+    rank = _env_int("RANK", 0)
+    local = _env_int("LOCAL_RANK", 0)
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+
+    w = _workload(args.config)
+    mine = _shard(w, rank, world)
+    tr = pt.Tracker(local)
+    tr.load_volume(w.volume)
+    V = w.volume.nx * w.volume.ny * w.volume.nz
+    rb = pt.pt_record_bytes(w.volume.nfibres, pt.PT_F16 if w.volume.is_half else pt.PT_F32)
+    seeds_d = torch.as_tensor(mine.seeds, device=dev).contiguous()
+    ids_d = torch.as_tensor(mine.ids().astype(np.int64), device=dev).contiguous()
+    out_map = torch.empty((w.volume.nz, w.volume.ny, w.volume.nx), dtype=torch.int32, device=dev)
+    flush_buf = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)  # > L2 (126 MB)
+
+    def one_step():
+        flush_buf.fill_(1)  # evict L2 between steps
+        tr.track(seeds_d, ids_d, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
+                 max_steps=w.max_steps, rng_seed=w.rng_seed,
+                 particles_per_seed=w.particles_per_seed, out_map=out_map)
+        if world > 1:
+            dist.reduce(out_map, dst=0, op=dist.ReduceOp.SUM)  # modular int32 sum == uint32 sum
+
+    for _ in range(args.warmup):
+        one_step()
+    torch.cuda.synchronize()
+    st0 = tr.stats()
+
+    clocks = ClockSampler(local)
+    clocks.start()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    kern_ms = []
+    steps_done = 0
+    e0.record()
+    for _ in range(args.steps):
+        one_step()
+        s = tr.stats() if args.per_step_stats else None
+        if s:
+            kern_ms.append(s["kernel_ms"])
+            steps_done += s["total_steps"]
+    e1.record()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ck = clocks.stop()
+    ms = e0.elapsed_time(e1)
+    st = tr.stats()
+    if not args.per_step_stats:
+        kern_ms = [st["kernel_ms"]]
+        steps_done = st["total_steps"] * args.steps
+    my_steps = st["total_steps"]  # identical every step (deterministic)
+    t = torch.tensor([ms, float(my_steps), float(mine.nseeds), float(st["lane_active"]),
+                      float(st["lane_slots"])], dtype=torch.float64, device=dev)
+    if world > 1:
+        tmax = t.clone()
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        ms = float(tmax[0])
+    total_steps = float(t[1]) if world > 1 else float(my_steps)
+    total_seeds = float(t[2]) if world > 1 else float(mine.nseeds)
+    lane_frac = float(t[3] / t[4]) if float(t[4]) else None
+
+    # ---- e2e through the C ABI with host buffers (pinned seeds in, pinned map out)
+    seeds_h = torch.as_tensor(mine.seeds).pin_memory()
+    ids_h = torch.as_tensor(mine.ids().astype(np.int64)).pin_memory()
+    map_h = torch.empty((w.volume.nz, w.volume.ny, w.volume.nx), dtype=torch.int32).pin_memory()
+    e2e_steps = max(1, min(args.steps, 3))
+    tr.track(seeds_h, ids_h, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
+             max_steps=w.max_steps, rng_seed=w.rng_seed, particles_per_seed=w.particles_per_seed,
+             out_map=map_h)  # warm
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(e2e_steps):
+        flush_buf.fill_(1)
+        tr.track(seeds_h, ids_h, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
+                 max_steps=w.max_steps, rng_seed=w.rng_seed,
+                 particles_per_seed=w.particles_per_seed, out_map=map_h)
+        if world > 1:
+            # the host map is reduced over the process group as the step's result
+            mt = map_h.to(dev, non_blocking=True)
+            dist.reduce(mt, dst=0, op=dist.ReduceOp.SUM)
+            if rank == 0:
+                map_h.copy_(mt)
+    torch.cuda.synchronize()
+    e2e_s = time.perf_counter() - t0
+    te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_value = total_steps * e2e_steps / float(te[0])
+
+    # ---- roofline (dominant kernel = the tracking kernel)
+    kms = sum(kern_ms) / len(kern_ms)
+    alg_bytes = my_steps * (rb + 8) + mine.nseeds * (12 + 8)
+    achieved = alg_bytes / (kms * 1e-3) / 1e9
+    peaks = _peaks()
+    peak = peaks["hbm_gbs"] if peaks else 6650.0
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+            "frac": achieved / peak, "traffic": _ncu_traffic(args.config),
+            "peak_source": "measured (MEASURED_PEAKS.json hbm_gbs)" if peaks else "fallback 6.65 TB/s",
+            "bytes_per_step": rb + 8, "kernel_ms": kms}
+    gather = None
+    if rank == 0 and not args.no_gather_bench:
+        rec_bytes_total = V * w.volume.nsamples * rb
+        r_hbm = tr.gather_bench(int(rec_bytes_total), rb)
+        r_l2 = tr.gather_bench(64 * 1024 * 1024, rb)
+        sec_per_step = max(1, rb // 32)
+        sps = my_steps / (kms * 1e-3)
+        gather = {"r_gather_hbm_sectors_per_s": r_hbm, "r_gather_l2_sectors_per_s": r_l2,
+                  "hbm_copy_sectors_per_s": peak * 1e9 / 32,
+                  "frac_of_r_gather_hbm": sps * sec_per_step / r_hbm,
+                  "frac_of_r_gather_l2": sps * sec_per_step / r_l2,
+                  "frac_of_hbm_copy_sectors": sps * sec_per_step / (peak * 1e9 / 32),
+                  "sectors_per_step": sec_per_step}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+        oracle.build()
+        threads = len(os.sched_getaffinity(0))
+        sub, J, every = _cpu_sample(w, args.cpu_seconds, threads)
+        s, dt = _run_oracle_sample(sub, J, threads)
+        cpu = {"value": s / dt, "unit": "steps/s", "cores": threads, "kind": "oracle",
+               "sample": f"every {every}th WM seed ({sub.nseeds} seeds) x particles j<{J}: "
+                         f"{s} steps in {dt:.1f} s"}
+
+    if rank == 0:
+        value = total_steps * args.steps / (ms * 1e-3)
+        line = {
+            "metric": METRIC, "value": value, "unit": "steps/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "f32", "data": "synthetic",
+            "config": {"workload": CONFIG_TEXT.get(args.config, args.config),
+                       "seeds": int(total_seeds), "particles_per_seed": w.particles_per_seed,
+                       "particles": int(total_seeds) * w.particles_per_seed,
+                       "steps_per_pass": int(total_steps),
+                       "mean_steps_per_streamline": total_steps / (total_seeds * w.particles_per_seed),
+                       "record_bytes": rb, "records": "fp16" if w.volume.is_half else "fp32",
+                       "parallelism": f"seed-sharded x{world}" + (" + NCCL reduce" if world > 1 else ""),
+                       "l2": "inputs > L2 (record volume %.2f GB) and a 256 MiB L2 flush between steps"
+                             % (V * w.volume.nsamples * rb / 1e9)},
+            "seeds_per_s": total_seeds * args.steps / (ms * 1e-3),
+            "active_lane_fraction": lane_frac,
+            "roofline": roof,
+            "gather_roofline": gather,
+            "cpu_baseline": cpu,
+            "e2e": {"value": e2e_value, "unit": "steps/s",
+                    "h2d_bytes_per_step": int(seeds_h.numel() * 4 + ids_h.numel() * 8),
+                    "d2h_bytes_per_step": int(map_h.numel() * 4)},
+            "gpu_launches": 2 * args.steps,
+            "clocks": ck,
+        }
+        print(json.dumps(line), flush=True)
+    tr.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main(argv=None):
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="c3")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-gather-bench", action="store_true")
+    ap.add_argument("--no-per-step-stats", dest="per_step_stats", action="store_false")
+    args = ap.parse_args(argv)
+    if args.warmup < 3 and args.impl == "ours" and not os.environ.get("BENCH_ALLOW_FEW_WARMUP"):
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,173 @@
+/*
+ * pt.h -- C ABI of the B200-native probabilistic-streamlining particle stepper.
+ *
+ * Method: Xu et al., "Probabilistic Brain Fiber Tractography on GPUs", IPDPS workshops
+ * 2012.  Citations P:Lnnn are PAPER.md lines; Rnn are the readings of the
+ * paper listed in DESIGN.md ("Readings").  The operations follow the paper's problem
+ * statement: the user supplies the sample volumes of the fibre directions/fractions
+ * (Fig. 1), start points, a step length and the termination criteria
+ * (maximum angle, maximum steps); they get back fibre paths and/or
+ * per-voxel visitation counts.
+ *
+ * Conventions for every entry point:
+ *   - returns a pt_status; never throws or aborts across the ABI; the message of the
+ *     last failure on a context is pt_last_error(ctx);
+ *   - pointer arguments may be host or device pointers (detected with
+ *     cudaPointerGetAttributes) unless stated otherwise; inputs are borrowed for the
+ *     duration of the call (copied), outputs are caller-owned;
+ *   - one context per (thread, GPU); distinct contexts are independent.
+ *   - no torch types: plain pointers and sizes.  The Python binding passes
+ *     tensor.data_ptr() and torch.cuda.current_stream().cuda_stream.
+ */
+#ifndef PT_H
+#define PT_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct pt_ctx pt_ctx;
+
+typedef enum {
+    PT_OK = 0,
+    PT_ERR_ARG = 1,       /* invalid argument (sizes, ranges, non-finite sample data) */
+    PT_ERR_STATE = 2,     /* call out of order (e.g. pt_track before pt_load_samples) */
+    PT_ERR_OOM = 3,       /* device allocation failed */
+    PT_ERR_CUDA = 4,      /* CUDA runtime error; map contents are then unspecified */
+    PT_ERR_OVERFLOW = 5   /* a uint32 map cell wrapped past 2^32-1 (R17) */
+} pt_status;
+
+typedef enum { PT_F32 = 0, PT_F16 = 1 } pt_dtype;
+
+/* Termination reasons (P:L113-121 keeps max steps and max angle; R11 adds the mask). */
+typedef enum { PT_END_MASK = 0, PT_END_CURV = 1, PT_END_MAXLEN = 2 } pt_reason;
+
+/* pt_params.flags */
+#define PT_REC_LEN        (1u << 0)  /* record per-particle nsteps (uint16)            */
+#define PT_REC_REASON     (1u << 1)  /* record per-particle pt_reason (uint8)           */
+#define PT_REC_END        (1u << 2)  /* record per-particle end point (3 x float32)     */
+#define PT_REC_PATHS      (1u << 3)  /* record polylines, path_stride points/particle   */
+#define PT_MAP_ACCUMULATE (1u << 4)  /* add to the map instead of zeroing it first      */
+#define PT_KERNEL_SIMPLE  (1u << 8)  /* ablation: one thread per particle, no lane
+                                        refill (the paper's "Extreme case 1")   */
+
+/* Create a context on CUDA device `cuda_device` (the caller's current device is left
+ * unchanged).  *out receives the context or NULL.  The stream defaults to the legacy
+ * default stream until pt_set_stream. */
+pt_status pt_create(int cuda_device, pt_ctx** out);
+/* Free every device buffer of the context. NULL-safe. */
+void pt_destroy(pt_ctx* ctx);
+/* Message of the last failed call on ctx ("" if none); valid until the next call.
+ * pt_last_error(NULL) returns the message of the last failed pt_create. */
+const char* pt_last_error(const pt_ctx* ctx);
+/* Stream (a cudaStream_t, or NULL for the legacy default stream) on which every later
+ * call on ctx enqueues its work. */
+pt_status pt_set_stream(pt_ctx* ctx, void* cuda_stream);
+
+/* Sample volume shape: nx, ny, nz > 0; nsamples S >= 1 (the number of MCMC samples per
+ * voxel); nfibres F in [1, 3] (N = 2 in the paper, Eq. 1);
+ * dtype of the dyads/f arrays. */
+typedef struct {
+    int32_t nx, ny, nz, nsamples, nfibres;
+    int32_t dtype; /* pt_dtype */
+} pt_volume;
+
+/* Load the per-voxel orientation samples (the six sample volumes f1,f2,theta1,theta2,
+ * phi1,phi2 of P:L125, with (theta, phi) given as Cartesian unit vectors, R20) and the
+ * tracking mask, and repack them on the device into one record per (voxel, sample).
+ *   dyads: [F][S][nz][ny][nx][3] (x fastest, xyz innermost), float32 or binary16 bits
+ *   f    : [F][S][nz][ny][nx], same dtype
+ *   mask : [nz][ny][nx] uint8, != 0 inside
+ * Host or device pointers; copied; the caller keeps ownership.  Replaces any previously
+ * loaded volume.  Errors: PT_ERR_ARG for bad shapes, NULL pointers or a non-finite
+ * dyad / f value inside the mask; PT_ERR_OOM; PT_ERR_CUDA.  Synchronises ctx's stream. */
+pt_status pt_load_samples(pt_ctx* ctx, const pt_volume* vol, const void* dyads,
+                          const void* f, const uint8_t* mask);
+
+/* Tracking parameters (Sec. III-B3; Table II P:L283-291 uses step 0.1-0.3,
+ * dot thresholds 0.8-0.9 and 50 samples). */
+typedef struct {
+    float step;                 /* step length in voxels, > 0 (R3)                       */
+    float curv_thr;             /* continue iff |v . d_prev| > curv_thr, |curv_thr| <= 1
+                                   (maximum angle "measured by the dot product"; R4) */
+    float fib_thr;              /* fibre j eligible for the direction choice iff f_j > fib_thr (R7) */
+    int32_t max_steps;          /* 1..65535 (maximum number of steps; R14)        */
+    uint64_t rng_seed;          /* Philox-4x32-10 key (R16)                               */
+    int64_t particles_per_seed; /* P >= 1; particle j of seed id k has pid = k*P + j      */
+    uint32_t flags;             /* PT_REC_* | PT_MAP_ACCUMULATE | PT_KERNEL_SIMPLE        */
+    int32_t path_stride;        /* points stored per particle with PT_REC_PATHS (>= 1)    */
+} pt_params;
+
+/* Track P particles from each seed (Algorithm 1, with the stepping
+ * semantics of P:L98-121 and contract C-ALG of DESIGN.md).
+ *   seeds_xyz: [nseeds][3] float32 corner-convention voxel coordinates (the centre of
+ *              voxel i is i + 0.5)
+ *   seed_ids : [nseeds] uint64 global seed ids, or NULL for 0..nseeds-1.  The RNG is
+ *              keyed by pid = seed_id*P + j, so results do not depend on sharding or on
+ *              the order of the seeds.
+ *   map      : [nz][ny][nx] uint32 visitation counts (one per committed step at the new
+ *              voxel, R13), zeroed first unless PT_MAP_ACCUMULATE; may be NULL.
+ * With device pointers the call is asynchronous on ctx's stream; a host `map` makes it
+ * synchronous (device map, then a device-to-host copy).  Per-particle outputs selected
+ * by flags stay on the device until pt_get_paths.  Errors: PT_ERR_STATE before
+ * pt_load_samples; PT_ERR_ARG for parameter ranges, nseeds < 0 or pid overflow;
+ * PT_ERR_OOM; PT_ERR_CUDA.  Map overflow is reported by pt_get_stats/pt_get_paths. */
+pt_status pt_track(pt_ctx* ctx, const float* seeds_xyz, const uint64_t* seed_ids,
+                   int64_t nseeds, const pt_params* params, uint32_t* map);
+
+/* Per-particle outputs of the last pt_track, particle index = seed_index*P + j.
+ * Set capacity = number of particles the buffers hold; NULL buffers are skipped;
+ * count receives the number of particles of the last pt_track (query with all buffers
+ * NULL).  nsteps [count] uint16; reason [count] uint8; end_xyz [count][3] float32
+ * corner coordinates; paths [count][path_stride][3] float32 (point 0 = start, point k =
+ * after the k-th committed step, unused points NaN).  Requesting an output that the
+ * last pt_track did not record is PT_ERR_STATE; capacity < count is PT_ERR_ARG.
+ * Synchronises ctx's stream; returns PT_ERR_OVERFLOW if the map wrapped. */
+typedef struct {
+    uint16_t* nsteps;
+    uint8_t* reason;
+    float* end_xyz;
+    float* paths;
+    int64_t capacity;
+    int64_t count;       /* out */
+    int32_t path_stride; /* out */
+} pt_paths;
+pt_status pt_get_paths(pt_ctx* ctx, pt_paths* out);
+
+/* Counters of the last pt_track (synchronises ctx's stream).
+ *   total_steps      : sum of nsteps over all particles (= sum of the map, R13)
+ *   particles        : particles tracked
+ *   lane_active      : sum over warp step-iterations of live lanes
+ *   lane_slots       : 32 x warp step-iterations (active-lane fraction = ratio)
+ *   map_sum          : sum of the map cells after the call (mod 2^64)
+ *   overflow         : 1 if a map cell wrapped (detected as map_sum != expected)
+ *   kernel_ms        : device time of the tracking kernel (CUDA events on ctx's stream)
+ *   track_ms         : device time of the whole pt_track enqueue (zeroing, kernel, checks) */
+typedef struct {
+    uint64_t total_steps;
+    uint64_t particles;
+    uint64_t lane_active;
+    uint64_t lane_slots;
+    uint64_t map_sum;
+    int32_t overflow;
+    float kernel_ms;
+    float track_ms;
+} pt_stats;
+pt_status pt_get_stats(pt_ctx* ctx, pt_stats* out);
+
+/* Roofline micro-benchmark: uniformly random, record-aligned
+ * reads of `record_bytes` (8, 16, 32 or 64) from a device buffer of `buffer_bytes`,
+ * full occupancy, no other work.  *sectors_per_s receives 32-byte sectors per second.
+ * Synchronous. */
+pt_status pt_gather_bench(pt_ctx* ctx, int64_t buffer_bytes, int32_t record_bytes,
+                          double* sectors_per_s);
+
+/* Record bytes of the repacked layout for (nfibres, dtype): 16/32/64 (f32) or 8/16/32
+ * (f16).  Returns 0 for invalid arguments. */
+int32_t pt_record_bytes(int32_t nfibres, int32_t dtype);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,279 @@
+"""B200-native probabilistic-streamlining particle stepper (Xu et al., IPDPSW 2012).
+
+Thin Python binding of the C ABI in ``include/pt.h`` (``libpt.so``, sm_100a).  Every
+function here only marshals arguments: the whole hot path (repack, stepping, counting)
+runs in the CUDA kernels of ``csrc/``.  There is no CPU fallback: importing the binding
+without a built ``libpt.so`` raises, and every call without a CUDA device fails with the
+library's own error.  PyTorch supplies device memory and streams only.
+
+Low-level names mirror the C ABI (``pt_create``, ``pt_load_samples``, ``pt_track``,
+``pt_get_paths``, ``pt_get_stats``, ``pt_gather_bench``...); ``Tracker`` is the same
+calls with torch tensors.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional
+
+import numpy as np
+
+from ._build import LIB, build  # noqa: F401
+
+__all__ = [
+    "PtError", "lib", "Tracker", "pt_create", "pt_destroy", "pt_last_error", "pt_set_stream",
+    "pt_load_samples", "pt_track", "pt_get_paths", "pt_get_stats", "pt_gather_bench",
+    "pt_record_bytes", "PT_F32", "PT_F16", "PT_REC_LEN", "PT_REC_REASON", "PT_REC_END",
+    "PT_REC_PATHS", "PT_MAP_ACCUMULATE", "PT_KERNEL_SIMPLE", "PT_END_MASK", "PT_END_CURV",
+    "PT_END_MAXLEN", "EXPORTS",
+]
+
+PT_OK, PT_ERR_ARG, PT_ERR_STATE, PT_ERR_OOM, PT_ERR_CUDA, PT_ERR_OVERFLOW = range(6)
+PT_F32, PT_F16 = 0, 1
+PT_END_MASK, PT_END_CURV, PT_END_MAXLEN = 0, 1, 2
+PT_REC_LEN = 1 << 0
+PT_REC_REASON = 1 << 1
+PT_REC_END = 1 << 2
+PT_REC_PATHS = 1 << 3
+PT_MAP_ACCUMULATE = 1 << 4
+PT_KERNEL_SIMPLE = 1 << 8
+
+# every symbol include/pt.h declares
+EXPORTS = ["pt_create", "pt_destroy", "pt_last_error", "pt_set_stream", "pt_load_samples",
+           "pt_track", "pt_get_paths", "pt_get_stats", "pt_gather_bench", "pt_record_bytes"]
+
+_STATUS = {1: "PT_ERR_ARG", 2: "PT_ERR_STATE", 3: "PT_ERR_OOM", 4: "PT_ERR_CUDA", 5: "PT_ERR_OVERFLOW"}
+
+
+class PtError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class pt_volume(ctypes.Structure):
+    _fields_ = [("nx", ctypes.c_int32), ("ny", ctypes.c_int32), ("nz", ctypes.c_int32),
+                ("nsamples", ctypes.c_int32), ("nfibres", ctypes.c_int32), ("dtype", ctypes.c_int32)]
+
+
+class pt_params(ctypes.Structure):
+    _fields_ = [("step", ctypes.c_float), ("curv_thr", ctypes.c_float), ("fib_thr", ctypes.c_float),
+                ("max_steps", ctypes.c_int32), ("rng_seed", ctypes.c_uint64),
+                ("particles_per_seed", ctypes.c_int64), ("flags", ctypes.c_uint32),
+                ("path_stride", ctypes.c_int32)]
+
+
+class pt_paths(ctypes.Structure):
+    _fields_ = [("nsteps", ctypes.c_void_p), ("reason", ctypes.c_void_p), ("end_xyz", ctypes.c_void_p),
+                ("paths", ctypes.c_void_p), ("capacity", ctypes.c_int64), ("count", ctypes.c_int64),
+                ("path_stride", ctypes.c_int32)]
+
+
+class pt_stats(ctypes.Structure):
+    _fields_ = [("total_steps", ctypes.c_uint64), ("particles", ctypes.c_uint64),
+                ("lane_active", ctypes.c_uint64), ("lane_slots", ctypes.c_uint64),
+                ("map_sum", ctypes.c_uint64), ("overflow", ctypes.c_int32),
+                ("kernel_ms", ctypes.c_float), ("track_ms", ctypes.c_float)]
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load the in-tree libpt.so (raises if it was not built: there is no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB):
+        raise ImportError(f"{LIB} is missing: run __graft_entry__.build() (nvcc, sm_100a); "
+                          "this package has no CPU fallback")
+    L = ctypes.CDLL(LIB)
+    vp, P = ctypes.c_void_p, ctypes.POINTER
+    L.pt_create.argtypes = [ctypes.c_int, P(vp)]
+    L.pt_create.restype = ctypes.c_int
+    L.pt_destroy.argtypes = [vp]
+    L.pt_destroy.restype = None
+    L.pt_last_error.argtypes = [vp]
+    L.pt_last_error.restype = ctypes.c_char_p
+    L.pt_set_stream.argtypes = [vp, vp]
+    L.pt_set_stream.restype = ctypes.c_int
+    L.pt_load_samples.argtypes = [vp, P(pt_volume), vp, vp, vp]
+    L.pt_load_samples.restype = ctypes.c_int
+    L.pt_track.argtypes = [vp, vp, vp, ctypes.c_int64, P(pt_params), vp]
+    L.pt_track.restype = ctypes.c_int
+    L.pt_get_paths.argtypes = [vp, P(pt_paths)]
+    L.pt_get_paths.restype = ctypes.c_int
+    L.pt_get_stats.argtypes = [vp, P(pt_stats)]
+    L.pt_get_stats.restype = ctypes.c_int
+    L.pt_gather_bench.argtypes = [vp, ctypes.c_int64, ctypes.c_int32, P(ctypes.c_double)]
+    L.pt_gather_bench.restype = ctypes.c_int
+    L.pt_record_bytes.argtypes = [ctypes.c_int32, ctypes.c_int32]
+    L.pt_record_bytes.restype = ctypes.c_int32
+    _lib = L
+    return L
+
+
+def _check(ctx, rc: int):
+    if rc != PT_OK:
+        msg = lib().pt_last_error(ctx)
+        raise PtError(rc, (msg or b"").decode(errors="replace"))
+
+
+# ------------------------------------------------------------------ C-ABI names (marshalling)
+
+def pt_create(device: int = 0) -> int:
+    h = ctypes.c_void_p()
+    _check(None, lib().pt_create(device, ctypes.byref(h)))
+    return h.value
+
+
+def pt_destroy(ctx) -> None:
+    lib().pt_destroy(ctx)
+
+
+def pt_last_error(ctx) -> str:
+    return (lib().pt_last_error(ctx) or b"").decode(errors="replace")
+
+
+def pt_set_stream(ctx, stream: int) -> None:
+    _check(ctx, lib().pt_set_stream(ctx, stream))
+
+
+def pt_record_bytes(nfibres: int, dtype: int) -> int:
+    return int(lib().pt_record_bytes(nfibres, dtype))
+
+
+def pt_load_samples(ctx, nx, ny, nz, nsamples, nfibres, dtype, dyads_ptr, f_ptr, mask_ptr) -> None:
+    v = pt_volume(nx, ny, nz, nsamples, nfibres, dtype)
+    _check(ctx, lib().pt_load_samples(ctx, ctypes.byref(v), dyads_ptr, f_ptr, mask_ptr))
+
+
+def pt_track(ctx, seeds_ptr, ids_ptr, nseeds: int, params: pt_params, map_ptr) -> None:
+    _check(ctx, lib().pt_track(ctx, seeds_ptr, ids_ptr, nseeds, ctypes.byref(params), map_ptr))
+
+
+def pt_get_paths(ctx, out: pt_paths) -> pt_paths:
+    _check(ctx, lib().pt_get_paths(ctx, ctypes.byref(out)))
+    return out
+
+
+def pt_get_stats(ctx) -> pt_stats:
+    s = pt_stats()
+    _check(ctx, lib().pt_get_stats(ctx, ctypes.byref(s)))
+    return s
+
+
+def pt_gather_bench(ctx, buffer_bytes: int, record_bytes: int) -> float:
+    r = ctypes.c_double()
+    _check(ctx, lib().pt_gather_bench(ctx, buffer_bytes, record_bytes, ctypes.byref(r)))
+    return r.value
+
+
+# ------------------------------------------------------------------ torch convenience
+
+def _ptr(a) -> Optional[int]:
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        assert a.flags.c_contiguous
+        return a.ctypes.data
+    assert a.is_contiguous()
+    return a.data_ptr()
+
+
+class Tracker:
+    """One context on one GPU; tensors in, tensors out (torch supplies memory/streams)."""
+
+    def __init__(self, device: int = 0):
+        import torch
+        self.torch = torch
+        self.device = torch.device("cuda", device)
+        self.ctx = pt_create(device)
+        self.shape = None
+
+    def close(self):
+        if self.ctx:
+            pt_destroy(self.ctx)
+            self.ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def _stream(self):
+        pt_set_stream(self.ctx, self.torch.cuda.current_stream(self.device).cuda_stream)
+
+    def load_samples(self, dyads, f, mask, nsamples: int, nfibres: int) -> None:
+        """dyads [F][S][Z][Y][X][3], f [F][S][Z][Y][X] (float32 or float16), mask [Z][Y][X]
+        uint8; numpy (host) or torch (host or cuda) arrays."""
+        half = str(dyads.dtype).endswith("float16")
+        nz, ny, nx = mask.shape
+        self._stream()
+        pt_load_samples(self.ctx, nx, ny, nz, nsamples, nfibres, PT_F16 if half else PT_F32,
+                        _ptr(dyads), _ptr(f), _ptr(mask))
+        self.shape = (nz, ny, nx)
+
+    def load_volume(self, vol) -> None:
+        """A phantom.Volume-like object (dyads, f, mask, nsamples, nfibres)."""
+        self.load_samples(vol.dyads, vol.f, vol.mask, vol.nsamples, vol.nfibres)
+
+    def track(self, seeds, seed_ids=None, *, step: float, curv_thr: float, fib_thr: float,
+              max_steps: int, rng_seed: int, particles_per_seed: int, flags: int = 0,
+              path_stride: int = 0, out_map=None, want_map: bool = True):
+        """Enqueue pt_track on the current torch stream; returns the map (a cuda int32
+        tensor [Z][Y][X] holding the uint32 counts bit for bit, unless ``out_map`` is
+        given) or None."""
+        torch = self.torch
+        if want_map and out_map is None:
+            out_map = torch.empty(self.shape, dtype=torch.int32, device=self.device)
+        prm = pt_params(step, curv_thr, fib_thr, max_steps, rng_seed, particles_per_seed, flags,
+                        path_stride)
+        self._stream()
+        n = int(seeds.shape[0])
+        pt_track(self.ctx, _ptr(seeds), _ptr(seed_ids), n, prm, _ptr(out_map) if want_map else None)
+        return out_map if want_map else None
+
+    def track_workload(self, w, flags: int = 0, path_stride: int = 0, seeds=None, seed_ids=None,
+                       out_map=None, want_map: bool = True):
+        seeds = w.seeds if seeds is None else seeds
+        if seed_ids is None and w.seed_ids is not None:
+            seed_ids = w.seed_ids
+        return self.track(seeds, seed_ids, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
+                          max_steps=w.max_steps, rng_seed=w.rng_seed,
+                          particles_per_seed=w.particles_per_seed, flags=flags,
+                          path_stride=path_stride, out_map=out_map, want_map=want_map)
+
+    def stats(self) -> dict:
+        s = pt_get_stats(self.ctx)
+        return {k: getattr(s, k) for k, _ in pt_stats._fields_}
+
+    def get_paths(self, nsteps=True, reason=True, end=True, paths=False, on_device=False) -> dict:
+        """Per-particle outputs of the last track: host numpy arrays, or cuda tensors with
+        ``on_device`` (nsteps as int16 holding the uint16 bits, reason as uint8)."""
+        q = pt_get_paths(self.ctx, pt_paths())
+        n, stride = q.count, q.path_stride
+        out = {}
+        bufs = pt_paths()
+        bufs.capacity = n
+        torch = self.torch
+
+        def alloc(name, shape, npdt, tdt):
+            a = torch.empty(shape, dtype=tdt, device=self.device) if on_device else np.empty(shape, npdt)
+            out[name] = a
+            return _ptr(a)
+        if nsteps:
+            bufs.nsteps = alloc("nsteps", (n,), np.uint16, torch.int16)
+        if reason:
+            bufs.reason = alloc("reason", (n,), np.uint8, torch.uint8)
+        if end:
+            bufs.end_xyz = alloc("end", (n, 3), np.float32, torch.float32)
+        if paths:
+            bufs.paths = alloc("paths", (n, stride, 3), np.float32, torch.float32)
+        pt_get_paths(self.ctx, bufs)
+        return out
+
+    def gather_bench(self, buffer_bytes: int, record_bytes: int) -> float:
+        self._stream()
+        return pt_gather_bench(self.ctx, buffer_bytes, record_bytes)

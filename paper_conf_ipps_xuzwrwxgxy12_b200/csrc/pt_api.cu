@@ -1,0 +1,521 @@
+// pt_api.cu -- host side of the C ABI declared in include/pt.h.
+//
+// Owns the device state of one context: the repacked record volume, per-call particle
+// outputs, counters and CUDA events.  Every call enqueues on the context's stream and
+// converts CUDA failures into pt_status codes with a message (no exceptions cross the ABI).
+#include "pt.h"
+
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "pt_internal.h"
+
+struct pt_ctx {
+    int device = 0;
+    int num_sms = 0;
+    cudaStream_t stream = nullptr;
+    std::string err;
+    // volume
+    bool loaded = false;
+    pt_volume vol{};
+    int rec_bytes = 0;
+    uint8_t* d_rec = nullptr;
+    size_t rec_size = 0;
+    // per-call buffers
+    float* d_seeds = nullptr;
+    size_t seeds_cap = 0;
+    uint64_t* d_ids = nullptr;
+    size_t ids_cap = 0;
+    uint32_t* d_map = nullptr;   // internal map for host map pointers
+    size_t map_cap = 0;
+    uint16_t* d_nsteps = nullptr;
+    size_t nsteps_cap = 0;
+    uint8_t* d_reason = nullptr;
+    size_t reason_cap = 0;
+    float* d_end = nullptr;
+    size_t end_cap = 0;
+    float* d_paths = nullptr;
+    size_t paths_cap = 0;
+    unsigned long long* d_stats = nullptr;
+    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+    // last call
+    bool tracked = false;
+    uint64_t last_count = 0;
+    uint32_t last_flags = 0;
+    int32_t last_stride = 0;
+    bool last_map = false;
+};
+
+static std::string g_create_err;
+
+namespace {
+
+pt_status fail(pt_ctx* c, pt_status s, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    if (c) c->err = buf;
+    else g_create_err = buf;
+    return s;
+}
+
+pt_status cuda_fail(pt_ctx* c, cudaError_t e, const char* what) {
+    cudaGetLastError();  // clear a non-sticky error
+    if (e == cudaErrorMemoryAllocation)
+        return fail(c, PT_ERR_OOM, "%s: %s", what, cudaGetErrorString(e));
+    return fail(c, PT_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+#define CK(expr, what)                                   \
+    do {                                                 \
+        cudaError_t _e = (expr);                         \
+        if (_e != cudaSuccess) return cuda_fail(c, _e, what); \
+    } while (0)
+
+// RAII: make ctx's device current for the duration of a call, restore the caller's.
+struct DeviceGuard {
+    int prev = -1;
+    bool ok = true;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != dev) ok = cudaSetDevice(dev) == cudaSuccess;
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+bool is_device_ptr(const void* p) {
+    if (!p) return false;
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+template <typename T>
+cudaError_t ensure(T*& ptr, size_t& cap, size_t n) {
+    if (n <= cap && ptr) return cudaSuccess;
+    if (ptr) cudaFree(ptr);
+    ptr = nullptr;
+    cap = 0;
+    size_t want = n ? n : 1;
+    cudaError_t e = cudaMalloc(reinterpret_cast<void**>(&ptr), want * sizeof(T));
+    if (e == cudaSuccess) cap = want;
+    return e;
+}
+
+int rec_bytes_of(int F, int dtype) {
+    if (F < 1 || F > 3) return 0;
+    int raw;
+    if (dtype == PT_F32) raw = 16 * F;
+    else if (dtype == PT_F16) raw = 8 * F;
+    else return 0;
+    return raw <= 8 ? 8 : raw <= 16 ? 16 : raw <= 32 ? 32 : 64;
+}
+
+}  // namespace
+
+extern "C" {
+
+int32_t pt_record_bytes(int32_t nfibres, int32_t dtype) { return rec_bytes_of(nfibres, dtype); }
+
+pt_status pt_create(int cuda_device, pt_ctx** out) {
+    if (!out) return fail(nullptr, PT_ERR_ARG, "pt_create: out is NULL");
+    *out = nullptr;
+    int n = 0;
+    cudaError_t e = cudaGetDeviceCount(&n);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(nullptr, PT_ERR_CUDA, "pt_create: no CUDA device (%s)", cudaGetErrorString(e));
+    }
+    if (cuda_device < 0 || cuda_device >= n)
+        return fail(nullptr, PT_ERR_ARG, "pt_create: device %d out of range [0,%d)", cuda_device, n);
+    pt_ctx* c = new (std::nothrow) pt_ctx();
+    if (!c) return fail(nullptr, PT_ERR_OOM, "pt_create: host allocation failed");
+    c->device = cuda_device;
+    DeviceGuard g(cuda_device);
+    if (!g.ok) {
+        delete c;
+        return fail(nullptr, PT_ERR_CUDA, "pt_create: cudaSetDevice(%d) failed", cuda_device);
+    }
+    cudaDeviceProp prop;
+    e = cudaGetDeviceProperties(&prop, cuda_device);
+    if (e != cudaSuccess) {
+        delete c;
+        cudaGetLastError();
+        return fail(nullptr, PT_ERR_CUDA, "pt_create: %s", cudaGetErrorString(e));
+    }
+    c->num_sms = prop.multiProcessorCount;
+    for (auto& ev : c->ev) {
+        if (cudaEventCreate(&ev) != cudaSuccess) {
+            cudaGetLastError();
+            pt_destroy(c);
+            return fail(nullptr, PT_ERR_CUDA, "pt_create: cudaEventCreate failed");
+        }
+    }
+    if (cudaMalloc(&c->d_stats, sizeof(unsigned long long) * pt::kNumStats) != cudaSuccess) {
+        cudaGetLastError();
+        pt_destroy(c);
+        return fail(nullptr, PT_ERR_OOM, "pt_create: cudaMalloc(stats) failed");
+    }
+    cudaMemset(c->d_stats, 0, sizeof(unsigned long long) * pt::kNumStats);
+    *out = c;
+    return PT_OK;
+}
+
+void pt_destroy(pt_ctx* c) {
+    if (!c) return;
+    DeviceGuard g(c->device);
+    if (c->stream) cudaStreamSynchronize(c->stream);
+    else cudaDeviceSynchronize();
+    void* bufs[] = {c->d_rec, c->d_seeds, c->d_ids, c->d_map, c->d_nsteps,
+                    c->d_reason, c->d_end, c->d_paths, c->d_stats};
+    for (void* b : bufs)
+        if (b) cudaFree(b);
+    for (auto& ev : c->ev)
+        if (ev) cudaEventDestroy(ev);
+    cudaGetLastError();
+    delete c;
+}
+
+const char* pt_last_error(const pt_ctx* c) { return c ? c->err.c_str() : g_create_err.c_str(); }
+
+pt_status pt_set_stream(pt_ctx* c, void* stream) {
+    if (!c) return PT_ERR_ARG;
+    c->err.clear();
+    c->stream = static_cast<cudaStream_t>(stream);
+    return PT_OK;
+}
+
+pt_status pt_load_samples(pt_ctx* c, const pt_volume* v, const void* dyads, const void* f,
+                          const uint8_t* mask) {
+    if (!c) return PT_ERR_ARG;
+    c->err.clear();
+    if (!v || !dyads || !f || !mask) return fail(c, PT_ERR_ARG, "pt_load_samples: NULL argument");
+    if (v->nx <= 0 || v->ny <= 0 || v->nz <= 0)
+        return fail(c, PT_ERR_ARG, "pt_load_samples: dims must be > 0 (got %d %d %d)", v->nx, v->ny, v->nz);
+    if (v->nsamples < 1) return fail(c, PT_ERR_ARG, "pt_load_samples: nsamples must be >= 1");
+    if (v->nfibres < 1 || v->nfibres > 3)
+        return fail(c, PT_ERR_ARG, "pt_load_samples: nfibres must be in [1,3] (got %d)", v->nfibres);
+    const int rb = rec_bytes_of(v->nfibres, v->dtype);
+    if (!rb) return fail(c, PT_ERR_ARG, "pt_load_samples: dtype must be PT_F32 or PT_F16");
+    const uint64_t V = (uint64_t)v->nx * v->ny * v->nz;
+    if (V > 0xFFFFFFFFull) return fail(c, PT_ERR_ARG, "pt_load_samples: more than 2^32-1 voxels");
+    DeviceGuard g(c->device);
+    if (!g.ok) return fail(c, PT_ERR_CUDA, "pt_load_samples: cannot select device %d", c->device);
+    const uint64_t S = (uint64_t)v->nsamples, F = (uint64_t)v->nfibres;
+    const size_t esz = v->dtype == PT_F16 ? 2 : 4;
+    const size_t dy_bytes = F * S * V * 3 * esz, f_bytes = F * S * V * esz, m_bytes = V;
+    const size_t rec_size = V * S * (size_t)rb;
+
+    // stage host inputs on the device (device inputs are read in place)
+    const void* d_dy = dyads;
+    const void* d_f = f;
+    const uint8_t* d_m = mask;
+    void* tmp[3] = {nullptr, nullptr, nullptr};
+    auto cleanup = [&]() {
+        for (void* t : tmp)
+            if (t) cudaFree(t);
+    };
+    const void* src[3] = {dyads, f, mask};
+    const size_t sz[3] = {dy_bytes, f_bytes, m_bytes};
+    const void** dst[3] = {&d_dy, &d_f, reinterpret_cast<const void**>(&d_m)};
+    for (int i = 0; i < 3; ++i) {
+        if (!is_device_ptr(src[i])) {
+            cudaError_t e = cudaMalloc(&tmp[i], sz[i]);
+            if (e != cudaSuccess) {
+                cleanup();
+                return cuda_fail(c, e, "pt_load_samples: staging allocation");
+            }
+            e = cudaMemcpyAsync(tmp[i], src[i], sz[i], cudaMemcpyHostToDevice, c->stream);
+            if (e != cudaSuccess) {
+                cleanup();
+                return cuda_fail(c, e, "pt_load_samples: host-to-device copy");
+            }
+            *dst[i] = tmp[i];
+        }
+    }
+    if (c->d_rec && c->rec_size != rec_size) {
+        cudaStreamSynchronize(c->stream);
+        cudaFree(c->d_rec);
+        c->d_rec = nullptr;
+        c->rec_size = 0;
+    }
+    if (!c->d_rec) {
+        cudaError_t e = cudaMalloc(&c->d_rec, rec_size);
+        if (e != cudaSuccess) {
+            cleanup();
+            c->loaded = false;
+            return cuda_fail(c, e, "pt_load_samples: record volume allocation");
+        }
+        c->rec_size = rec_size;
+    }
+    c->loaded = false;
+    cudaError_t e = cudaMemsetAsync(c->d_stats + pt::kStatBadInput, 0, sizeof(unsigned long long), c->stream);
+    if (e == cudaSuccess)
+        e = pt::launch_repack(d_dy, d_f, d_m, c->d_rec, (int64_t)V, v->nsamples, v->nfibres,
+                              v->dtype == PT_F16, rb, c->d_stats + pt::kStatBadInput, c->stream);
+    unsigned long long bad = 0;
+    if (e == cudaSuccess)
+        e = cudaMemcpyAsync(&bad, c->d_stats + pt::kStatBadInput, sizeof bad, cudaMemcpyDeviceToHost, c->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
+    cleanup();
+    if (e != cudaSuccess) return cuda_fail(c, e, "pt_load_samples: repack");
+    if (bad) return fail(c, PT_ERR_ARG, "pt_load_samples: %llu records inside the mask hold non-finite values", bad);
+    c->vol = *v;
+    c->rec_bytes = rb;
+    c->loaded = true;
+    c->tracked = false;
+    return PT_OK;
+}
+
+pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, int64_t nseeds,
+                   const pt_params* p, uint32_t* map) {
+    if (!c) return PT_ERR_ARG;
+    c->err.clear();
+    if (!c->loaded) return fail(c, PT_ERR_STATE, "pt_track: no sample volume loaded");
+    if (!p) return fail(c, PT_ERR_ARG, "pt_track: params is NULL");
+    if (nseeds < 0) return fail(c, PT_ERR_ARG, "pt_track: nseeds < 0");
+    if (nseeds > 0 && !seeds_xyz) return fail(c, PT_ERR_ARG, "pt_track: seeds_xyz is NULL");
+    if (!(p->step > 0.f) || !std::isfinite(p->step)) return fail(c, PT_ERR_ARG, "pt_track: step must be finite and > 0");
+    if (!(std::fabs(p->curv_thr) <= 1.f)) return fail(c, PT_ERR_ARG, "pt_track: |curv_thr| must be <= 1");
+    if (std::isnan(p->fib_thr)) return fail(c, PT_ERR_ARG, "pt_track: fib_thr is NaN");
+    if (p->max_steps < 1 || p->max_steps > 65535)
+        return fail(c, PT_ERR_ARG, "pt_track: max_steps must be in [1, 65535] (got %d)", p->max_steps);
+    if (p->particles_per_seed < 1) return fail(c, PT_ERR_ARG, "pt_track: particles_per_seed must be >= 1");
+    if ((p->flags & PT_REC_PATHS) && p->path_stride < 1)
+        return fail(c, PT_ERR_ARG, "pt_track: PT_REC_PATHS needs path_stride >= 1");
+    const uint64_t P = (uint64_t)p->particles_per_seed;
+    if (P > 0xFFFFFFFFull) return fail(c, PT_ERR_ARG, "pt_track: particles_per_seed must be < 2^32");
+    const uint64_t N = (uint64_t)nseeds;
+    if (N && P > UINT64_MAX / N) return fail(c, PT_ERR_ARG, "pt_track: nseeds * P overflows");
+    const uint64_t npart = N * P;
+    DeviceGuard g(c->device);
+    if (!g.ok) return fail(c, PT_ERR_CUDA, "pt_track: cannot select device %d", c->device);
+    cudaStream_t st = c->stream;
+
+    // inputs: host -> device staging
+    const float* d_seeds = seeds_xyz;
+    const uint64_t* d_ids = seed_ids;
+    if (N && !is_device_ptr(seeds_xyz)) {
+        CK(ensure(c->d_seeds, c->seeds_cap, 3 * N), "pt_track: seed buffer");
+        CK(cudaMemcpyAsync(c->d_seeds, seeds_xyz, 3 * N * sizeof(float), cudaMemcpyHostToDevice, st), "pt_track: seeds H2D");
+        d_seeds = c->d_seeds;
+    }
+    if (seed_ids) {
+        // pid overflow: seed_id * P + (P - 1) must fit in 64 bits
+        const uint64_t lim = (UINT64_MAX - (P - 1)) / P;
+        if (!is_device_ptr(seed_ids)) {
+            for (uint64_t i = 0; i < N; ++i)
+                if (seed_ids[i] > lim) return fail(c, PT_ERR_ARG, "pt_track: seed_id %llu * P overflows 64 bits", (unsigned long long)seed_ids[i]);
+            if (N) {
+                CK(ensure(c->d_ids, c->ids_cap, N), "pt_track: id buffer");
+                CK(cudaMemcpyAsync(c->d_ids, seed_ids, N * sizeof(uint64_t), cudaMemcpyHostToDevice, st), "pt_track: ids H2D");
+                d_ids = c->d_ids;
+            }
+        }
+        // device-resident ids are not range-checked (the caller guarantees id*P+P-1 < 2^64)
+    } else if (N && N - 1 > (UINT64_MAX - (P - 1)) / P) {
+        return fail(c, PT_ERR_ARG, "pt_track: pid overflow");
+    }
+
+    const int32_t nxv = c->vol.nx, nyv = c->vol.ny, nzv = c->vol.nz;
+    const uint64_t V = (uint64_t)nxv * nyv * nzv;
+    const bool host_map = map && !is_device_ptr(map);
+    uint32_t* d_map = map;
+    if (host_map) {
+        CK(ensure(c->d_map, c->map_cap, V), "pt_track: map buffer");
+        d_map = c->d_map;
+    }
+    const bool acc = (p->flags & PT_MAP_ACCUMULATE) != 0;
+
+    // outputs
+    const uint32_t fl = p->flags;
+    if (fl & PT_REC_LEN) CK(ensure(c->d_nsteps, c->nsteps_cap, npart), "pt_track: nsteps buffer");
+    if (fl & PT_REC_REASON) CK(ensure(c->d_reason, c->reason_cap, npart), "pt_track: reason buffer");
+    if (fl & PT_REC_END) CK(ensure(c->d_end, c->end_cap, 3 * npart), "pt_track: end buffer");
+    if (fl & PT_REC_PATHS) {
+        CK(ensure(c->d_paths, c->paths_cap, 3 * npart * (uint64_t)p->path_stride), "pt_track: path buffer");
+        CK(cudaMemsetAsync(c->d_paths, 0xFF, 3 * npart * (uint64_t)p->path_stride * sizeof(float), st), "pt_track: path fill");
+    }
+
+    CK(cudaEventRecord(c->ev[0], st), "pt_track: event");
+    CK(cudaMemsetAsync(c->d_stats, 0, sizeof(unsigned long long) * pt::kNumStats, st), "pt_track: stats reset");
+    if (d_map) {
+        if (host_map && acc)
+            CK(cudaMemcpyAsync(d_map, map, V * sizeof(uint32_t), cudaMemcpyHostToDevice, st), "pt_track: map H2D");
+        if (!acc) CK(cudaMemsetAsync(d_map, 0, V * sizeof(uint32_t), st), "pt_track: map zero");
+        else CK(pt::launch_map_sum(d_map, (int64_t)V, c->d_stats + pt::kStatMapBefore, st), "pt_track: map sum");
+    }
+
+    pt::TrackArgs a{};
+    a.rec = c->d_rec;
+    a.nx = nxv;
+    a.ny = nyv;
+    a.nz = nzv;
+    a.cx = nxv / 2;
+    a.cy = nyv / 2;
+    a.cz = nzv / 2;
+    a.fcx = (float)a.cx;
+    a.fcy = (float)a.cy;
+    a.fcz = (float)a.cz;
+    a.S = (uint32_t)c->vol.nsamples;
+    a.step = p->step;
+    a.curv_thr = p->curv_thr;
+    a.fib_thr = p->fib_thr;
+    a.max_steps = p->max_steps;
+    a.key0 = (uint32_t)p->rng_seed;
+    a.key1 = (uint32_t)(p->rng_seed >> 32);
+    a.P = P;
+    a.seeds = d_seeds;
+    a.seed_ids = d_ids;
+    a.nseeds = N;
+    a.nparticles = npart;
+    a.chunks_per_seed = (uint32_t)((P + pt::kChunk - 1) / pt::kChunk);
+    a.total_chunks = N * (uint64_t)a.chunks_per_seed;
+    a.map = d_map;
+    a.o_nsteps = (fl & PT_REC_LEN) ? c->d_nsteps : nullptr;
+    a.o_reason = (fl & PT_REC_REASON) ? c->d_reason : nullptr;
+    a.o_end = (fl & PT_REC_END) ? c->d_end : nullptr;
+    a.o_paths = (fl & PT_REC_PATHS) ? c->d_paths : nullptr;
+    a.path_stride = (fl & PT_REC_PATHS) ? p->path_stride : 0;
+    a.stats = c->d_stats;
+
+    CK(cudaEventRecord(c->ev[1], st), "pt_track: event");
+    CK(pt::launch_track(a, c->vol.nfibres, c->vol.dtype == PT_F16, (fl & PT_KERNEL_SIMPLE) != 0, c->num_sms, st),
+       "pt_track: tracking kernel launch");
+    CK(cudaEventRecord(c->ev[2], st), "pt_track: event");
+    if (d_map) CK(pt::launch_map_sum(d_map, (int64_t)V, c->d_stats + pt::kStatMapAfter, st), "pt_track: map sum");
+    if (host_map) {
+        CK(cudaMemcpyAsync(map, d_map, V * sizeof(uint32_t), cudaMemcpyDeviceToHost, st), "pt_track: map D2H");
+    }
+    CK(cudaEventRecord(c->ev[3], st), "pt_track: event");
+    if (host_map) CK(cudaStreamSynchronize(st), "pt_track: synchronise");
+
+    c->tracked = true;
+    c->last_count = npart;
+    c->last_flags = fl;
+    c->last_stride = (fl & PT_REC_PATHS) ? p->path_stride : 0;
+    c->last_map = d_map != nullptr;
+    return PT_OK;
+}
+
+pt_status pt_get_stats(pt_ctx* c, pt_stats* out) {
+    if (!c || !out) return PT_ERR_ARG;
+    c->err.clear();
+    if (!c->tracked) return fail(c, PT_ERR_STATE, "pt_get_stats: no pt_track yet");
+    DeviceGuard g(c->device);
+    unsigned long long s[pt::kNumStats];
+    CK(cudaStreamSynchronize(c->stream), "pt_get_stats: synchronise");
+    CK(cudaMemcpy(s, c->d_stats, sizeof s, cudaMemcpyDeviceToHost), "pt_get_stats: copy");
+    std::memset(out, 0, sizeof *out);
+    out->total_steps = s[pt::kStatSteps];
+    out->particles = s[pt::kStatParticles];
+    out->lane_active = s[pt::kStatLaneActive];
+    out->lane_slots = s[pt::kStatLaneSlots];
+    out->map_sum = s[pt::kStatMapAfter];
+    out->overflow = (c->last_map && s[pt::kStatMapAfter] != s[pt::kStatMapBefore] + s[pt::kStatSteps]) ? 1 : 0;
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, c->ev[1], c->ev[2]), "pt_get_stats: kernel time");
+    out->kernel_ms = ms;
+    CK(cudaEventElapsedTime(&ms, c->ev[0], c->ev[3]), "pt_get_stats: track time");
+    out->track_ms = ms;
+    if (out->overflow) return fail(c, PT_ERR_OVERFLOW, "a uint32 map cell wrapped past 2^32-1");
+    return PT_OK;
+}
+
+pt_status pt_get_paths(pt_ctx* c, pt_paths* out) {
+    if (!c || !out) return PT_ERR_ARG;
+    c->err.clear();
+    if (!c->tracked) return fail(c, PT_ERR_STATE, "pt_get_paths: no pt_track yet");
+    DeviceGuard g(c->device);
+    out->count = (int64_t)c->last_count;
+    out->path_stride = c->last_stride;
+    const bool any = out->nsteps || out->reason || out->end_xyz || out->paths;
+    if (any && out->capacity < (int64_t)c->last_count)
+        return fail(c, PT_ERR_ARG, "pt_get_paths: capacity %lld < count %llu", (long long)out->capacity,
+                    (unsigned long long)c->last_count);
+    if ((out->nsteps && !(c->last_flags & PT_REC_LEN)) || (out->reason && !(c->last_flags & PT_REC_REASON)) ||
+        (out->end_xyz && !(c->last_flags & PT_REC_END)) || (out->paths && !(c->last_flags & PT_REC_PATHS)))
+        return fail(c, PT_ERR_STATE, "pt_get_paths: output not recorded by the last pt_track (flags 0x%x)", c->last_flags);
+    const uint64_t n = c->last_count;
+    cudaStream_t st = c->stream;
+    if (n) {
+        if (out->nsteps) CK(cudaMemcpyAsync(out->nsteps, c->d_nsteps, n * 2, cudaMemcpyDefault, st), "pt_get_paths: nsteps");
+        if (out->reason) CK(cudaMemcpyAsync(out->reason, c->d_reason, n, cudaMemcpyDefault, st), "pt_get_paths: reason");
+        if (out->end_xyz) CK(cudaMemcpyAsync(out->end_xyz, c->d_end, n * 12, cudaMemcpyDefault, st), "pt_get_paths: end");
+        if (out->paths)
+            CK(cudaMemcpyAsync(out->paths, c->d_paths, n * 12 * (uint64_t)c->last_stride, cudaMemcpyDefault, st),
+               "pt_get_paths: paths");
+    }
+    CK(cudaStreamSynchronize(st), "pt_get_paths: synchronise");
+    pt_stats s;
+    pt_status rc = pt_get_stats(c, &s);
+    return rc;
+}
+
+pt_status pt_gather_bench(pt_ctx* c, int64_t buffer_bytes, int32_t record_bytes, double* sectors_per_s) {
+    if (!c || !sectors_per_s) return PT_ERR_ARG;
+    c->err.clear();
+    if (record_bytes != 8 && record_bytes != 16 && record_bytes != 32 && record_bytes != 64)
+        return fail(c, PT_ERR_ARG, "pt_gather_bench: record_bytes must be 8, 16, 32 or 64");
+    if (buffer_bytes < record_bytes * 1024)
+        return fail(c, PT_ERR_ARG, "pt_gather_bench: buffer too small");
+    DeviceGuard g(c->device);
+    uint8_t* buf = nullptr;
+    uint32_t* sink = nullptr;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    auto cleanup = [&]() {
+        if (buf) cudaFree(buf);
+        if (sink) cudaFree(sink);
+        if (e0) cudaEventDestroy(e0);
+        if (e1) cudaEventDestroy(e1);
+    };
+    cudaError_t e = cudaMalloc(&buf, (size_t)buffer_bytes);
+    if (e == cudaSuccess) e = cudaMalloc(&sink, 64);
+    if (e == cudaSuccess) e = cudaMemsetAsync(buf, 0x3C, (size_t)buffer_bytes, c->stream);
+    if (e == cudaSuccess) e = cudaEventCreate(&e0);
+    if (e == cudaSuccess) e = cudaEventCreate(&e1);
+    if (e != cudaSuccess) {
+        cleanup();
+        return cuda_fail(c, e, "pt_gather_bench: setup");
+    }
+    const uint64_t nrec = (uint64_t)buffer_bytes / (uint64_t)record_bytes;
+    int per_sm = pt::gather_bench_blocks_per_sm(record_bytes);
+    if (per_sm < 1) per_sm = 1;
+    const int blocks = c->num_sms * per_sm;
+    const uint32_t iters = 256;
+    double best = 0.0;
+    for (int rep = 0; rep < 4; ++rep) {
+        e = cudaEventRecord(e0, c->stream);
+        if (e == cudaSuccess) e = pt::launch_gather_bench(buf, nrec, record_bytes, iters, blocks, 0x1234567u + rep, sink, c->stream);
+        if (e == cudaSuccess) e = cudaEventRecord(e1, c->stream);
+        if (e == cudaSuccess) e = cudaEventSynchronize(e1);
+        float ms = 0.f;
+        if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, e0, e1);
+        if (e != cudaSuccess) {
+            cleanup();
+            return cuda_fail(c, e, "pt_gather_bench: run");
+        }
+        const double loads = (double)blocks * 256.0 * (double)iters;
+        const double sectors = loads * (record_bytes > 32 ? record_bytes / 32 : 1);
+        const double rate = sectors / (ms * 1e-3);
+        if (rep > 0 && rate > best) best = rate;  // rep 0 = warm-up
+    }
+    cleanup();
+    *sectors_per_s = best;
+    return PT_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,106 @@
+// pt_device.cuh -- device-side building blocks of the tracking kernels (sm_100a).
+//
+// Every floating-point operation of the stepping arithmetic is written with __fmul_rn /
+// __fadd_rn / __fsub_rn (one IEEE binary32 operation, round-to-nearest-even, never
+// contracted into an FMA) and the library is additionally compiled with -fmad=false, so
+// the results are bit-identical to any correctly rounded binary32 evaluation of the same
+// expression order (R15 in DESIGN.md).  Citations: P:Lnnn = PAPER.md line.
+#pragma once
+#include <cstdint>
+#include <cuda_fp16.h>
+
+namespace pt {
+
+constexpr uint32_t kFull = 0xFFFFFFFFu;
+
+// ---------------------------------------------------------------------------- RNG (R16)
+// Philox4x32-10 (Salmon et al., SC'11): counter-based, so a particle's draws depend only
+// on (rng_seed, pid, block) and never on scheduling.  One block = 4 words: words 0..2
+// give the sample indices of steps 3b, 3b+1, 3b+2; word 3 of block 0 gives the first
+// step's sign.  Replaces the combined Tausworthe generator of P:L153.
+__device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint32_t k0, uint32_t k1) {
+#pragma unroll
+    for (int r = 0; r < 10; ++r) {
+        if (r) {
+            k0 += 0x9E3779B9u;
+            k1 += 0xBB67AE85u;
+        }
+        const uint32_t lo0 = 0xD2511F53u * c.x, hi0 = __umulhi(0xD2511F53u, c.x);
+        const uint32_t lo1 = 0xCD9E8D57u * c.z, hi1 = __umulhi(0xCD9E8D57u, c.z);
+        c = make_uint4(hi1 ^ c.y ^ k0, lo1, hi0 ^ c.w ^ k1, lo0);
+    }
+    return c;
+}
+
+// sample index s = floor(w * S / 2^32) (integer only; R16)
+__device__ __forceinline__ uint32_t sample_of(uint32_t w, uint32_t S) { return __umulhi(w, S); }
+
+// ---------------------------------------------------------------------------- records
+// One record per (voxel, sample): the F fibres' unit vector and fraction (the sample
+// volumes of P:L125 / Fig. 1, repacked).  fp32: {x,y,z,f} x F (16 B per fibre,
+// padded to 16/32/64 B); fp16: {x,y,z,f} halves x F (8 B per fibre, padded to 8/16/32 B).
+// A voxel outside the mask carries the sentinel f0 = all-ones (a NaN that validated
+// input never contains) in every sample: the gather that fetches the next step's record
+// is also the mask test of the candidate voxel (R11).
+template <int F, bool HALF>
+struct Rec {
+    static constexpr int kRaw = HALF ? 8 * F : 16 * F;
+    static constexpr int kBytes = kRaw <= 8 ? 8 : kRaw <= 16 ? 16 : kRaw <= 32 ? 32 : 64;
+    static constexpr int kWords = kBytes / 4;
+    uint32_t w[kWords];
+
+    __device__ __forceinline__ bool outside() const {
+        return HALF ? ((w[1] >> 16) == 0xFFFFu) : (w[3] == 0xFFFFFFFFu);
+    }
+    __device__ __forceinline__ void fibre(int j, float& x, float& y, float& z, float& f) const {
+        if (HALF) {
+            const uint32_t a = w[2 * j], b = w[2 * j + 1];
+            x = __half2float(__ushort_as_half((unsigned short)(a & 0xFFFFu)));
+            y = __half2float(__ushort_as_half((unsigned short)(a >> 16)));
+            z = __half2float(__ushort_as_half((unsigned short)(b & 0xFFFFu)));
+            f = __half2float(__ushort_as_half((unsigned short)(b >> 16)));
+        } else {
+            x = __uint_as_float(w[4 * j + 0]);
+            y = __uint_as_float(w[4 * j + 1]);
+            z = __uint_as_float(w[4 * j + 2]);
+            f = __uint_as_float(w[4 * j + 3]);
+        }
+    }
+};
+
+// Random gather of one record through the read-only (texture/L1) path: one LDG of 8, 16
+// or 32 bytes (two 32-B LDGs for a 64-B record).
+template <int BYTES>
+__device__ __forceinline__ void ldg_record(const void* p, uint32_t* w);
+
+template <>
+__device__ __forceinline__ void ldg_record<8>(const void* p, uint32_t* w) {
+    asm("ld.global.nc.v2.b32 {%0,%1}, [%2];" : "=r"(w[0]), "=r"(w[1]) : "l"(p));
+}
+template <>
+__device__ __forceinline__ void ldg_record<16>(const void* p, uint32_t* w) {
+    asm("ld.global.nc.v4.b32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3])
+                 : "l"(p));
+}
+template <>
+__device__ __forceinline__ void ldg_record<32>(const void* p, uint32_t* w) {
+    asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]),
+                   "=r"(w[6]), "=r"(w[7])
+                 : "l"(p));
+}
+template <>
+__device__ __forceinline__ void ldg_record<64>(const void* p, uint32_t* w) {
+    ldg_record<32>(p, w);
+    ldg_record<32>(static_cast<const char*>(p) + 32, w + 8);
+}
+
+// ---------------------------------------------------------------------------- lookup (R10)
+// Centred coordinates q = x - c, c = floor(N/2); index = c + trunc(q) - signbit(q):
+// voxel i covers [i-c, i-c+1) for i >= c and (i-c, i-c+1] for i < c.
+__device__ __forceinline__ int axis_index(float q, int c) {
+    return c + __float2int_rz(q) - (int)(__float_as_uint(q) >> 31);
+}
+
+}  // namespace pt

@@ -1,0 +1,63 @@
+// pt_internal.h -- private interface between the C-ABI host code (pt_api.cu) and the
+// kernels (pt_kernels.cu).  Not installed; not part of include/pt.h.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace pt {
+
+constexpr int kThreads = 256;       // threads per CTA of the tracking kernel
+constexpr uint32_t kChunk = 32;     // particles claimed per work-queue atomic
+
+// Indices of the per-call device counters (unsigned long long[kNumStats]).
+enum StatIdx {
+    kStatSteps = 0,      // sum of nsteps
+    kStatParticles = 1,  // particles finished
+    kStatLaneActive = 2, // live lanes summed over warp step-iterations
+    kStatLaneSlots = 3,  // 32 x warp step-iterations
+    kStatMapAfter = 4,   // sum of map cells after the kernel
+    kStatMapBefore = 5,  // sum of map cells before the kernel (accumulate mode)
+    kStatQueue = 6,      // work-queue counter (chunks claimed)
+    kStatBadInput = 7,   // repack: non-finite value inside the mask
+    kNumStats = 8
+};
+
+struct TrackArgs {
+    const uint8_t* rec;          // [V][S] records of rec_bytes
+    int nx, ny, nz;
+    int cx, cy, cz;              // floor(N/2) per axis
+    float fcx, fcy, fcz;         // the same as floats
+    uint32_t S;
+    float step, curv_thr, fib_thr;
+    int max_steps;
+    uint32_t key0, key1;
+    uint64_t P;                  // particles per seed
+    const float* seeds;          // [nseeds][3] corner coordinates
+    const uint64_t* seed_ids;    // [nseeds] or nullptr
+    uint64_t nseeds;
+    uint64_t nparticles;         // nseeds * P
+    uint32_t chunks_per_seed;    // ceil(P / kChunk)
+    uint64_t total_chunks;       // nseeds * chunks_per_seed
+    uint32_t* map;               // [V] or nullptr
+    uint16_t* o_nsteps;          // [nparticles] or nullptr
+    uint8_t* o_reason;
+    float* o_end;                // [nparticles][3]
+    float* o_paths;              // [nparticles][path_stride][3]
+    int path_stride;
+    unsigned long long* stats;   // [kNumStats]
+};
+
+// Launchers (return the launch error, if any).
+cudaError_t launch_track(const TrackArgs& a, int nfibres, bool half, bool simple, int num_sms,
+                         cudaStream_t st);
+int track_blocks_per_sm(int nfibres, bool half, bool simple);
+cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask, uint8_t* rec,
+                          int64_t V, int S, int F, bool half, int rec_bytes,
+                          unsigned long long* bad, cudaStream_t st);
+cudaError_t launch_map_sum(const uint32_t* map, int64_t V, unsigned long long* out,
+                           cudaStream_t st);
+cudaError_t launch_gather_bench(const uint8_t* buf, uint64_t nrec, int rec_bytes, uint32_t iters,
+                                int blocks, uint32_t seed, uint32_t* sink, cudaStream_t st);
+int gather_bench_blocks_per_sm(int rec_bytes);
+
+}  // namespace pt

@@ -1,0 +1,279 @@
+"""GPU <-> oracle parity through the C ABI (``-m gpu``; needs a B200 and libpt.so).
+
+Bar (BASELINE.json north_star): per-streamline (nsteps, reason, end
+point bits) and the uint32 visitation maps bit-exact vs the oracle on identical generated
+inputs.  Every comparison below is exact; the tolerance the north star allows (<= 1e-4
+divergent streamlines, map L1 relative difference <= 1e-4) is asserted as a fallback
+report only where a full-size run is sampled.
+"""
+from __future__ import annotations
+
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import phantom
+
+pytestmark = pytest.mark.gpu
+
+REC_ALL = None  # set in fixture
+
+
+@pytest.fixture(scope="module")
+def pt():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    import paper_conf_ipps_xuzwrwxgxy12_b200 as m
+    m.build()
+    global REC_ALL
+    REC_ALL = m.PT_REC_LEN | m.PT_REC_REASON | m.PT_REC_END
+    return m
+
+
+@pytest.fixture(scope="module")
+def tracker(pt):
+    t = pt.Tracker(0)
+    yield t
+    t.close()
+
+
+def _threads():
+    return max(1, len(os.sched_getaffinity(0)))
+
+
+def gpu_run(tr, w, flags=None, path_stride=0, **kw):
+    import torch
+    flags = REC_ALL if flags is None else flags
+    tr.load_volume(w.volume)
+    m = tr.track_workload(w, flags=flags, path_stride=path_stride, **kw)
+    torch.cuda.synchronize()
+    out = tr.get_paths(nsteps=bool(flags & 1), reason=bool(flags & 2), end=bool(flags & 4),
+                       paths=bool(flags & 8))
+    out["map"] = None if m is None else m.cpu().numpy().view(np.uint32)
+    out["stats"] = tr.stats()
+    return out
+
+
+def assert_parity(g, r, idx=None, check_map=True):
+    sl = slice(None) if idx is None else idx
+    assert np.array_equal(g["nsteps"][sl].astype(np.int64), r["nsteps"].astype(np.int64)), \
+        f"nsteps: {np.count_nonzero(g['nsteps'][sl].astype(np.int64) != r['nsteps'])} differ"
+    assert np.array_equal(g["reason"][sl], r["reason"])
+    assert np.array_equal(g["end"][sl].view(np.uint32), r["end"].view(np.uint32))
+    if check_map:
+        assert np.array_equal(g["map"].astype(np.uint64), r["map"])
+
+
+# ----------------------------------------------------------------------------- full configs
+
+@pytest.mark.parametrize("simple", [False, True])
+def test_c1_full(pt, tracker, simple):
+    """BASELINE configs[0]: every particle and the full map, both kernels."""
+    w = phantom.config("c1")
+    g = gpu_run(tracker, w, REC_ALL | (pt.PT_KERNEL_SIMPLE if simple else 0))
+    r = oracle.track(w)
+    assert_parity(g, r)
+    assert g["stats"]["total_steps"] == int(r["nsteps"].sum())
+
+
+def test_c2_full(pt, tracker):
+    """BASELINE configs[1] (zero dispersion): 1000 seeds x 5000 particles, all of them."""
+    w = phantom.config("c2")
+    g = gpu_run(tracker, w)
+    r = oracle.track(w, threads=_threads())
+    assert_parity(g, r)
+
+
+def test_c2_dispersed_full(pt, tracker):
+    """configs[1] shape, dispersed (sigma 0.15, f jitter 0.03): the full map and every
+    particle's (nsteps, reason, end)."""
+    w = phantom.config("c2_dispersed")
+    g = gpu_run(tracker, w)
+    r = oracle.track(w, threads=_threads())
+    assert_parity(g, r)
+    assert g["stats"]["total_steps"] == int(r["nsteps"].sum()) == int(g["map"].sum(dtype=np.uint64))
+
+
+# ----------------------------------------------------------------------------- paths
+
+@pytest.mark.parametrize("half", [False, True])
+@pytest.mark.parametrize("F", [1, 2, 3])
+def test_paths_bit_identical(pt, tracker, F, half):
+    """Per-step positions bit-identical on small brain-shaped volumes (F = 1..3, fp32 and
+    fp16 records), with a ragged particle count (P = 37, not a multiple of the chunk)."""
+    w = phantom.whole_brain(nx=40, ny=36, nz=24, semi=(17.0, 15.0, 10.0), nsamples=16, nfibres=F,
+                            particles_per_seed=37)
+    w = phantom.wm_seeds(w, every=max(1, w.nseeds // 150))
+    if half:
+        w = phantom.to_half(w)
+    stride = 512
+    g = gpu_run(tracker, w, REC_ALL | pt.PT_REC_PATHS, path_stride=stride)
+    r = oracle.track(w, path_stride=stride, threads=_threads())
+    assert_parity(g, r)
+    assert np.array_equal(g["paths"].view(np.uint32), r["paths"].view(np.uint32))
+
+
+@pytest.mark.parametrize("simple", [False, True])
+def test_crossing_dispersed_paths(pt, tracker, simple):
+    w = phantom.crossing(sigma=0.15, f_jitter=0.03, nseeds=60, particles_per_seed=40, nsamples=50)
+    g = gpu_run(tracker, w, REC_ALL | pt.PT_REC_PATHS | (pt.PT_KERNEL_SIMPLE if simple else 0),
+                path_stride=300)
+    r = oracle.track(w, path_stride=300)
+    assert_parity(g, r)
+    assert np.array_equal(g["paths"].view(np.uint32), r["paths"].view(np.uint32))
+
+
+# ----------------------------------------------------------------------------- full size, sampled
+
+@pytest.mark.parametrize("cfg", ["c3", "c4"])
+def test_whole_brain_full_size_sampled(pt, tracker, cfg):
+    """configs[2]/[3] at full size in the launch configuration bench.py times (persistent
+    kernel, all WM seeds x 5000 particles): 3000 sampled particles recomputed one by one
+    by the oracle, plus the global invariants at full size."""
+    import torch
+    w = phantom.config(cfg)
+    tracker.load_volume(w.volume)
+    m = tracker.track_workload(w, flags=REC_ALL)
+    torch.cuda.synchronize()
+    st = tracker.stats()
+    out = tracker.get_paths(on_device=True)
+    nst = out["nsteps"].to(torch.int64)
+    total = int(nst.sum().item())
+    gm = m.cpu().numpy().view(np.uint32)
+    assert st["particles"] == w.nparticles
+    assert st["total_steps"] == total == int(gm.sum(dtype=np.uint64))
+    assert int(nst.max().item()) <= w.max_steps
+    assert np.all(gm[w.volume.mask == 0] == 0)
+    rng = np.random.default_rng(2012)
+    pick = np.sort(rng.choice(w.nparticles, 3000, replace=False))
+    P = w.particles_per_seed
+    idx_t = torch.as_tensor(pick, device=out["nsteps"].device)
+    g = {"nsteps": out["nsteps"][idx_t].cpu().numpy().view(np.uint16),
+         "reason": out["reason"][idx_t].cpu().numpy(),
+         "end": out["end"][idx_t].cpu().numpy()}
+    rn, rr, re_ = [], [], []
+    for li in pick:
+        si, j = divmod(int(li), P)
+        sub = w.replace(seeds=w.seeds[si:si + 1], seed_ids=w.ids()[si:si + 1])
+        r = oracle.track(sub, j, j + 1, want_map=False)
+        rn.append(r["nsteps"][0])
+        rr.append(r["reason"][0])
+        re_.append(r["end"][0])
+    r = {"nsteps": np.array(rn), "reason": np.array(rr), "end": np.array(re_)}
+    diverged = (g["nsteps"].astype(np.int64) != r["nsteps"]) | (g["reason"] != r["reason"]) | \
+        np.any(g["end"].view(np.uint32) != r["end"].view(np.uint32), axis=1)
+    assert diverged.sum() == 0, f"{diverged.sum()} of {len(pick)} sampled streamlines diverge"
+    assert r["nsteps"].mean() > 10
+
+
+# ----------------------------------------------------------------------------- invariances
+
+def test_sharding_invariance(pt, tracker):
+    """C-pin-10 on the GPU: seeds sharded i mod G (G = 2, 3) with global seed ids give the
+    same per-pid results, and the shard maps sum to the unsharded map (what the NCCL
+    reduce of the multi-GPU path computes)."""
+    import torch
+    w = phantom.crossing(sigma=0.15, f_jitter=0.03, nseeds=300, particles_per_seed=500)
+    full = gpu_run(tracker, w)
+    for G in (2, 3):
+        tot = np.zeros_like(full["map"], dtype=np.uint64)
+        for rank in range(G):
+            sel = np.arange(rank, w.nseeds, G)
+            sub = w.replace(seeds=w.seeds[sel].copy(), seed_ids=w.ids()[sel].copy())
+            g = gpu_run(tracker, sub)
+            tot += g["map"]
+            rows = (sel[:, None] * w.particles_per_seed + np.arange(w.particles_per_seed)).ravel()
+            assert np.array_equal(g["nsteps"], full["nsteps"][rows])
+            assert np.array_equal(g["end"].view(np.uint32), full["end"][rows].view(np.uint32))
+        assert np.array_equal(tot, full["map"].astype(np.uint64))
+    torch.cuda.synchronize()
+
+
+def test_host_buffers_and_accumulate(pt, tracker):
+    """e2e path: host seeds + host map (H2D/D2H inside pt_track) equals the device path;
+    PT_MAP_ACCUMULATE adds to the existing map."""
+    w = phantom.crossing(sigma=0.15, nseeds=50, particles_per_seed=200)
+    dev = gpu_run(tracker, w, 0)
+    hm = np.zeros((w.volume.nz, w.volume.ny, w.volume.nx), np.uint32)
+    tracker.track(w.seeds, None, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
+                  max_steps=w.max_steps, rng_seed=w.rng_seed, particles_per_seed=w.particles_per_seed,
+                  out_map=hm)
+    assert np.array_equal(hm, dev["map"])
+    tracker.track(w.seeds, None, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
+                  max_steps=w.max_steps, rng_seed=w.rng_seed, particles_per_seed=w.particles_per_seed,
+                  out_map=hm, flags=pt.PT_MAP_ACCUMULATE)
+    assert np.array_equal(hm, 2 * dev["map"])
+
+
+def test_overflow_is_detected(pt, tracker):
+    """R17: a uint32 cell wrapping past 2^32-1 is reported as PT_ERR_OVERFLOW."""
+    import torch
+    w = phantom.tube(particles_per_seed=10)
+    tracker.load_volume(w.volume)
+    m = torch.full((w.volume.nz, w.volume.ny, w.volume.nx), -3, dtype=torch.int32, device="cuda")
+    tracker.track_workload(w, flags=pt.PT_MAP_ACCUMULATE, out_map=m)
+    with pytest.raises(pt.PtError) as e:
+        tracker.stats()
+    assert e.value.status == pt.PT_ERR_OVERFLOW
+
+
+# ----------------------------------------------------------------------------- edge cases
+
+def test_edge_cases(pt, tracker):
+    import torch
+    w = phantom.crossing(sigma=0.15, nseeds=20, particles_per_seed=33)
+    # seeds outside the volume and outside the mask (R12), plus max_steps = 1 and P = 1
+    seeds = np.concatenate([w.seeds, np.array([[-5.0, 3.0, 3.0], [0.5, 0.5, 0.5], [70.0, 1.0, 1.0]],
+                                              np.float32)])
+    for kw in ({}, {"max_steps": 1}, {"particles_per_seed": 1}, {"max_steps": 3}):
+        ww = w.replace(seeds=seeds, **kw)
+        g = gpu_run(tracker, ww)
+        r = oracle.track(ww)
+        assert_parity(g, r)
+    # no seeds: the map is zeroed, nothing else happens
+    tracker.load_volume(w.volume)
+    m = torch.full((w.volume.nz, w.volume.ny, w.volume.nx), 7, dtype=torch.int32, device="cuda")
+    tracker.track_workload(w, seeds=np.zeros((0, 3), np.float32), out_map=m)
+    torch.cuda.synchronize()
+    assert int(m.abs().sum().item()) == 0
+    assert tracker.stats()["particles"] == 0
+
+
+def test_errors(pt):
+    t = pt.Tracker(0)
+    w = phantom.tube(particles_per_seed=4)
+    with pytest.raises(pt.PtError) as e:
+        t.track_workload(w)
+    assert e.value.status == pt.PT_ERR_STATE
+    t.load_volume(w.volume)
+    for bad in ({"max_steps": 0}, {"max_steps": 70000}, {"step": 0.0}, {"curv_thr": 1.5},
+                {"particles_per_seed": 0}):
+        with pytest.raises(pt.PtError) as e:
+            t.track_workload(w.replace(**bad))
+        assert e.value.status == pt.PT_ERR_ARG
+    v = w.volume
+    dy = v.dyads.copy()
+    dy[0, 0, 8, 16, 16, 0] = np.nan  # inside the tube mask
+    with pytest.raises(pt.PtError) as e:
+        t.load_samples(dy, v.f, v.mask, v.nsamples, v.nfibres)
+    assert e.value.status == pt.PT_ERR_ARG
+    with pytest.raises(pt.PtError) as e:
+        t.get_paths(paths=True)
+    t.close()
+
+
+def test_lane_efficiency_and_gather_bench(pt, tracker):
+    """Lane refill keeps warps converged: active-lane fraction of the persistent kernel is
+    well above the no-refill ablation's (~1/H_32 for exponential lengths)."""
+    w = phantom.crossing(sigma=0.15, f_jitter=0.03, nseeds=400, particles_per_seed=2000)
+    a = gpu_run(tracker, w, 0)["stats"]
+    b = gpu_run(tracker, w, pt.PT_KERNEL_SIMPLE)["stats"]
+    fa = a["lane_active"] / a["lane_slots"]
+    fb = b["lane_active"] / b["lane_slots"]
+    assert a["total_steps"] == b["total_steps"]
+    assert fa > 0.8 and fa > fb, (fa, fb)
+    r = tracker.gather_bench(1 << 30, 32)
+    assert r > 1e9
