@@ -182,23 +182,20 @@ int oracle_track(const oracle_volume* vol, const oracle_params* prm,
                     /* maximum number of steps (R14) -- checked first */
                     if (n == prm->max_steps) { why = ORACLE_END_MAXLEN; break; }
 
-                    /* R1/R16: a fresh random sample index every step.  Block b = n/4 of
-                     * the sample stream: ctr = {b, pid_lo, pid_hi, 0}; word n%4. */
-                    blk_ctr[0] = (uint32_t)(n / 4); blk_ctr[1] = plo; blk_ctr[2] = phi; blk_ctr[3] = 0u;
+                    /* R1/R16: a fresh random sample index every step.  Block b = n/3 of
+                     * the particle's stream: ctr = {b, pid_lo, pid_hi, 0}; word n%3. */
+                    blk_ctr[0] = (uint32_t)(n / 3); blk_ctr[1] = plo; blk_ctr[2] = phi; blk_ctr[3] = 0u;
                     oracle_philox4x32_10(blk_ctr, key, w);
-                    s = oracle_sample_index(w[n % 4], S);
+                    s = oracle_sample_index(w[n % 3], S);
 
                     /* Interpolation() (R2): the sample's fibres at this voxel */
                     for (j = 0; j < F; ++j) fetch(vol, vox, s, j, v[j], &fv[j]);
 
                     if (n == 0) {
-                        /* R5, R6: first step follows fibre 0 with a random sign drawn from
-                         * the particle's init stream ctr = {0, pid_lo, pid_hi, 1}. */
-                        uint32_t ictr[4], iw[4];
-                        ictr[0] = 0u; ictr[1] = plo; ictr[2] = phi; ictr[3] = 1u;
-                        oracle_philox4x32_10(ictr, key, iw);
+                        /* R5, R6: first step follows fibre 0 with a random sign: the top
+                         * bit of word 3 of block 0 (w holds block 0 here). */
                         jstar = 0;
-                        sgn = (iw[0] >> 31) ? -1.0f : 1.0f;
+                        sgn = (w[3] >> 31) ? -1.0f : 1.0f;
                     } else {
                         /* choose the fibre closest to the previous direction
                          * (R7 eligibility f_j > fib_thr, R8 strict >, lowest j on ties). */

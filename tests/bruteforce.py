@@ -66,14 +66,13 @@ def track(w, seed_index: int, j: int, max_points: int = 10**9):
     while True:
         if n == w.max_steps:
             return n, 2, np.array(pos, np.float32)
-        wd = philox4x32_10([n // 4, pid & _M, pid >> 32, 0], key)
-        s = (wd[n % 4] * S) >> 32
+        wd = philox4x32_10([n // 3, pid & _M, pid >> 32, 0], key)
+        s = (wd[n % 3] * S) >> 32
         vv = [[dy[jj, s, vox[0], vox[1], vox[2], a] for a in range(3)] for jj in range(F)]
         ff = [fr[jj, s, vox[0], vox[1], vox[2]] for jj in range(F)]
         if n == 0:
-            iw = philox4x32_10([0, pid & _M, pid >> 32, 1], key)
             js = 0
-            sg = np.float32(-1.0) if (iw[0] >> 31) else np.float32(1.0)
+            sg = np.float32(-1.0) if (wd[3] >> 31) else np.float32(1.0)
         else:
             dots = [(vv[jj][0] * p[0] + vv[jj][1] * p[1]) + vv[jj][2] * p[2] for jj in range(F)]
             js = None
