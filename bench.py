@@ -133,11 +133,9 @@ def _workload(cfg):
 
 
 def _shard(w, rank, world):
-    import numpy as np
-    if world == 1:
-        return w
-    sel = np.arange(rank, w.nseeds, world)
-    return w.replace(seeds=w.seeds[sel].copy(), seed_ids=w.ids()[sel].copy())
+    from paper_conf_ipps_xuzwrwxgxy12_b200 import sharding
+    seeds, ids = sharding.shard_seeds(w.seeds, w.seed_ids, rank, world)
+    return w.replace(seeds=seeds, seed_ids=ids)
 
 
 def _cpu_sample(w, target_s: float, threads: int):
@@ -212,6 +210,7 @@ def run_ours(args):
     import torch.distributed as dist
 
     import paper_conf_ipps_xuzwrwxgxy12_b200 as pt
+    from paper_conf_ipps_xuzwrwxgxy12_b200 import sharding
 
     world = _env_int("WORLD_SIZE", 1)
     rank = _env_int("RANK", 0)
@@ -237,9 +236,9 @@ def run_ours(args):
         flush_buf.fill_(1)  # evict L2 between steps
         tr.track(seeds_d, ids_d, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
                  max_steps=w.max_steps, rng_seed=w.rng_seed,
-                 particles_per_seed=w.particles_per_seed, out_map=out_map)
+                 particles_per_seed=w.particles_per_seed, out_map=out_map, flags=args.track_flags)
         if world > 1:
-            dist.reduce(out_map, dst=0, op=dist.ReduceOp.SUM)  # modular int32 sum == uint32 sum
+            sharding.reduce_map(out_map, dst=0)  # one NCCL reduce; int32 sum == uint32 sum
 
     for _ in range(args.warmup):
         one_step()
@@ -300,11 +299,11 @@ def run_ours(args):
         flush_buf.fill_(1)
         tr.track(seeds_h, ids_h, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
                  max_steps=w.max_steps, rng_seed=w.rng_seed,
-                 particles_per_seed=w.particles_per_seed, out_map=map_h)
+                 particles_per_seed=w.particles_per_seed, out_map=map_h, flags=args.track_flags)
         if world > 1:
             # the host map is reduced over the process group as the step's result
             mt = map_h.to(dev, non_blocking=True)
-            dist.reduce(mt, dst=0, op=dist.ReduceOp.SUM)
+            sharding.reduce_map(mt, dst=0)
             if rank == 0:
                 map_h.copy_(mt)
     torch.cuda.synchronize()
@@ -394,6 +393,9 @@ def main(argv=None):
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-gather-bench", action="store_true")
     ap.add_argument("--no-per-step-stats", dest="per_step_stats", action="store_false")
+    ap.add_argument("--track-flags", type=int, default=0,
+                    help="extra pt_params.flags for ablations (e.g. 256 = PT_KERNEL_SIMPLE, "
+                         "512 = PT_SEED_ORDER_INPUT)")
     args = ap.parse_args(argv)
     if args.warmup < 3 and args.impl == "ours" and not os.environ.get("BENCH_ALLOW_FEW_WARMUP"):
         args.warmup = 3

@@ -51,6 +51,9 @@ typedef enum { PT_END_MASK = 0, PT_END_CURV = 1, PT_END_MAXLEN = 2 } pt_reason;
 #define PT_MAP_ACCUMULATE (1u << 4)  /* add to the map instead of zeroing it first      */
 #define PT_KERNEL_SIMPLE  (1u << 8)  /* ablation: one thread per particle, no lane
                                         refill (the paper's "Extreme case 1")   */
+#define PT_SEED_ORDER_INPUT (1u << 9) /* ablation: claim seeds in input order instead of
+                                        the default Z-order (Morton) of their voxels;
+                                        results are identical either way (R16)           */
 
 /* Create a context on CUDA device `cuda_device` (the caller's current device is left
  * unchanged).  *out receives the context or NULL.  The stream defaults to the legacy
@@ -95,7 +98,8 @@ typedef struct {
     int32_t max_steps;          /* 1..65535 (maximum number of steps; R14)        */
     uint64_t rng_seed;          /* Philox-4x32-10 key (R16)                               */
     int64_t particles_per_seed; /* P >= 1; particle j of seed id k has pid = k*P + j      */
-    uint32_t flags;             /* PT_REC_* | PT_MAP_ACCUMULATE | PT_KERNEL_SIMPLE        */
+    uint32_t flags;             /* PT_REC_* | PT_MAP_ACCUMULATE | PT_KERNEL_SIMPLE |
+                                   PT_SEED_ORDER_INPUT                                    */
     int32_t path_stride;        /* points stored per particle with PT_REC_PATHS (>= 1)    */
 } pt_params;
 

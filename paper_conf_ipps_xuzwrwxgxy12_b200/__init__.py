@@ -24,7 +24,7 @@ __all__ = [
     "PtError", "lib", "Tracker", "pt_create", "pt_destroy", "pt_last_error", "pt_set_stream",
     "pt_load_samples", "pt_track", "pt_get_paths", "pt_get_stats", "pt_gather_bench",
     "pt_record_bytes", "PT_F32", "PT_F16", "PT_REC_LEN", "PT_REC_REASON", "PT_REC_END",
-    "PT_REC_PATHS", "PT_MAP_ACCUMULATE", "PT_KERNEL_SIMPLE", "PT_END_MASK", "PT_END_CURV",
+    "PT_REC_PATHS", "PT_MAP_ACCUMULATE", "PT_KERNEL_SIMPLE", "PT_SEED_ORDER_INPUT", "PT_END_MASK", "PT_END_CURV",
     "PT_END_MAXLEN", "EXPORTS",
 ]
 
@@ -37,6 +37,7 @@ PT_REC_END = 1 << 2
 PT_REC_PATHS = 1 << 3
 PT_MAP_ACCUMULATE = 1 << 4
 PT_KERNEL_SIMPLE = 1 << 8
+PT_SEED_ORDER_INPUT = 1 << 9
 
 # every symbol include/pt.h declares
 EXPORTS = ["pt_create", "pt_destroy", "pt_last_error", "pt_set_stream", "pt_load_samples",
@@ -175,10 +176,20 @@ def _ptr(a) -> Optional[int]:
     if a is None:
         return None
     if isinstance(a, np.ndarray):
-        assert a.flags.c_contiguous
+        if not a.flags.c_contiguous:
+            raise ValueError("array must be C-contiguous")
         return a.ctypes.data
-    assert a.is_contiguous()
+    if not a.is_contiguous():
+        raise ValueError("tensor must be contiguous")
     return a.data_ptr()
+
+
+def _contig(a):
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        return np.ascontiguousarray(a)
+    return a.contiguous()
 
 
 class Tracker:
@@ -226,10 +237,11 @@ class Tracker:
         tensor [Z][Y][X] holding the uint32 counts bit for bit, unless ``out_map`` is
         given) or None."""
         torch = self.torch
-        if want_map and out_map is None:
+        if want_map and out_map is None and self.shape is not None:
             out_map = torch.empty(self.shape, dtype=torch.int32, device=self.device)
         prm = pt_params(step, curv_thr, fib_thr, max_steps, rng_seed, particles_per_seed, flags,
                         path_stride)
+        seeds, seed_ids = _contig(seeds), _contig(seed_ids)
         self._stream()
         n = int(seeds.shape[0])
         pt_track(self.ctx, _ptr(seeds), _ptr(seed_ids), n, prm, _ptr(out_map) if want_map else None)

@@ -9,7 +9,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
-LIB = os.path.join(PKG, "libpt.so")
+LIB = os.environ.get("PT_LIB") or os.path.join(PKG, "libpt.so")  # PT_LIB: experiment builds
 SOURCES = ["pt_api.cu", "pt_kernels.cu"]
 HEADERS = ["pt_device.cuh", "pt_internal.h"]
 

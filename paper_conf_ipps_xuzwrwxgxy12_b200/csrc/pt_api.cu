@@ -31,6 +31,10 @@ struct pt_ctx {
     size_t seeds_cap = 0;
     uint64_t* d_ids = nullptr;
     size_t ids_cap = 0;
+    uint64_t* d_keys = nullptr;  // seed-order sort keys
+    size_t keys_cap = 0;
+    uint32_t* d_perm = nullptr;  // seed processing order
+    size_t perm_cap = 0;
     uint32_t* d_map = nullptr;   // internal map for host map pointers
     size_t map_cap = 0;
     uint16_t* d_nsteps = nullptr;
@@ -179,7 +183,7 @@ void pt_destroy(pt_ctx* c) {
     DeviceGuard g(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
     else cudaDeviceSynchronize();
-    void* bufs[] = {c->d_rec, c->d_seeds, c->d_ids, c->d_map, c->d_nsteps,
+    void* bufs[] = {c->d_rec, c->d_seeds, c->d_ids, c->d_keys, c->d_perm, c->d_map, c->d_nsteps,
                     c->d_reason, c->d_end, c->d_paths, c->d_stats};
     for (void* b : bufs)
         if (b) cudaFree(b);
@@ -359,6 +363,15 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         else CK(pt::launch_map_sum(d_map, (int64_t)V, c->d_stats + pt::kStatMapBefore, st), "pt_track: map sum");
     }
 
+    const uint32_t* d_order = nullptr;
+    if (!(fl & (PT_SEED_ORDER_INPUT | PT_KERNEL_SIMPLE)) && N > 1) {
+        if (N > 0xFFFFFFFFull) return fail(c, PT_ERR_ARG, "pt_track: more than 2^32-1 seeds");
+        CK(ensure(c->d_keys, c->keys_cap, N), "pt_track: order keys");
+        CK(ensure(c->d_perm, c->perm_cap, N), "pt_track: order buffer");
+        CK(pt::launch_seed_order(d_seeds, N, c->d_keys, c->d_perm, st), "pt_track: seed order");
+        d_order = c->d_perm;
+    }
+
     pt::TrackArgs a{};
     a.rec = c->d_rec;
     a.nx = nxv;
@@ -380,6 +393,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.P = P;
     a.seeds = d_seeds;
     a.seed_ids = d_ids;
+    a.order = d_order;
     a.nseeds = N;
     a.nparticles = npart;
     a.chunks_per_seed = (uint32_t)((P + pt::kChunk - 1) / pt::kChunk);

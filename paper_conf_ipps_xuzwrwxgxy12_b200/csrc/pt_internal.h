@@ -34,6 +34,7 @@ struct TrackArgs {
     uint64_t P;                  // particles per seed
     const float* seeds;          // [nseeds][3] corner coordinates
     const uint64_t* seed_ids;    // [nseeds] or nullptr
+    const uint32_t* order;       // [nseeds] processing order (Morton) or nullptr
     uint64_t nseeds;
     uint64_t nparticles;         // nseeds * P
     uint32_t chunks_per_seed;    // ceil(P / kChunk)
@@ -54,6 +55,10 @@ int track_blocks_per_sm(int nfibres, bool half, bool simple);
 cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask, uint8_t* rec,
                           int64_t V, int S, int F, bool half, int rec_bytes,
                           unsigned long long* bad, cudaStream_t st);
+// Z-order processing permutation of the seeds: perm[k] = index of the k-th seed in Morton
+// order of its voxel (ties by input index).  keys/perm/tmp are device buffers of nseeds.
+cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint64_t* keys, uint32_t* perm,
+                              cudaStream_t st);
 cudaError_t launch_map_sum(const uint32_t* map, int64_t V, unsigned long long* out,
                            cudaStream_t st);
 cudaError_t launch_gather_bench(const uint8_t* buf, uint64_t nrec, int rec_bytes, uint32_t iters,

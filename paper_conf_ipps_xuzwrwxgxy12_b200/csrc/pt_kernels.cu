@@ -17,18 +17,24 @@
 // the third step's gather is deferred to the next round's start, where it is issued by
 // the same instruction as the first gather of freshly refilled lanes.
 #include <cuda_runtime.h>
+#include <thrust/execution_policy.h>
+#include <thrust/sort.h>
 
 #include <cstdint>
 
 #include "pt_device.cuh"
 #include "pt_internal.h"
 
+#ifndef PT_MIN_BLOCKS
+#define PT_MIN_BLOCKS 1
+#endif
+
 namespace pt {
 
 enum { kEndMask = 0, kEndCurv = 1, kEndMaxlen = 2 };
 
 template <int F, bool HALF, bool REFILL>
-__global__ void __launch_bounds__(kThreads) track_kernel(const __grid_constant__ TrackArgs a) {
+__global__ void __launch_bounds__(kThreads, PT_MIN_BLOCKS) track_kernel(const __grid_constant__ TrackArgs a) {
     using R = Rec<F, HALF>;
     constexpr int RB = R::kBytes;
     const uint32_t lane = threadIdx.x & 31u;
@@ -151,8 +157,9 @@ __global__ void __launch_bounds__(kThreads) track_kernel(const __grid_constant__
                         exhausted = true;
                         break;
                     }
-                    cseed = c / a.chunks_per_seed;
-                    cnext = (uint32_t)(c - cseed * a.chunks_per_seed) * kChunk;
+                    const uint64_t k = c / a.chunks_per_seed;
+                    cnext = (uint32_t)(c - k * a.chunks_per_seed) * kChunk;
+                    cseed = a.order ? (uint64_t)a.order[k] : k;
                     const uint64_t e = (uint64_t)cnext + kChunk;
                     cend = (uint32_t)(e < a.P ? e : a.P);
                 }
@@ -340,6 +347,45 @@ __global__ void repack_kernel(const void* __restrict__ dyads, const void* __rest
                 reinterpret_cast<uint4*>(out)[k] = make_uint4(w[4 * k], w[4 * k + 1], w[4 * k + 2], w[4 * k + 3]);
         }
     }
+}
+
+// ------------------------------------------------------------------------- seed order
+// Morton key of the seed's voxel (10 bits per axis; coordinates clamped to [0, 1023]),
+// with the input index in the low 32 bits so the sort is a total order.
+__device__ __forceinline__ uint64_t spread3(uint32_t v) {
+    uint64_t x = v & 0x3FFu;
+    x = (x | (x << 16)) & 0x030000FFull;
+    x = (x | (x << 8)) & 0x0300F00Full;
+    x = (x | (x << 4)) & 0x030C30C3ull;
+    x = (x | (x << 2)) & 0x09249249ull;
+    return x;
+}
+
+__global__ void seed_keys_kernel(const float* __restrict__ seeds, uint64_t n, uint64_t* keys,
+                                 uint32_t* perm) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t c[3];
+#pragma unroll
+        for (int a = 0; a < 3; ++a) {
+            const float x = seeds[3 * i + a];
+            c[a] = x <= 0.f ? 0u : (x >= 1023.f ? 1023u : (uint32_t)x);
+        }
+        const uint64_t m = spread3(c[0]) | (spread3(c[1]) << 1) | (spread3(c[2]) << 2);
+        keys[i] = (m << 32) | (uint64_t)(uint32_t)i;
+        perm[i] = (uint32_t)i;
+    }
+}
+
+cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint64_t* keys, uint32_t* perm,
+                              cudaStream_t st) {
+    if (nseeds == 0) return cudaSuccess;
+    uint64_t blocks = (nseeds + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    seed_keys_kernel<<<(unsigned)blocks, 256, 0, st>>>(seeds, nseeds, keys, perm);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+    thrust::sort_by_key(thrust::cuda::par.on(st), keys, keys + nseeds, perm);
+    return cudaGetLastError();
 }
 
 // ------------------------------------------------------------------------- map sum

@@ -1,0 +1,44 @@
+"""Seed sharding and the map combine of the multi-GPU path.
+
+Particles are independent and the RNG is keyed by the *global* particle id
+(seed_id * P + j, R16), so a rank can track any subset of seeds as long as it passes their
+global ids: the union of the ranks' results equals the single-GPU result bit for bit.  The
+only exchange is the final combine of the per-rank uint32 visitation maps: one
+``reduce(SUM)`` (NCCL on GPUs) of the maps viewed as int32 -- two's-complement addition is
+the same bit pattern as uint32 addition mod 2^32, so the combined map is bit-identical.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+
+def shard_indices(nseeds: int, rank: int, world: int) -> np.ndarray:
+    """Interleaved sharding: seed i -> rank i mod world (spatially uniform, so the per-rank
+    work balances statistically for raster-ordered seeds)."""
+    if world < 1 or not (0 <= rank < world):
+        raise ValueError(f"bad rank {rank} / world {world}")
+    return np.arange(rank, nseeds, world, dtype=np.int64)
+
+
+def shard_seeds(seeds: np.ndarray, seed_ids, rank: int, world: int):
+    """(seeds, global seed ids) of this rank's shard."""
+    n = int(seeds.shape[0])
+    ids = np.arange(n, dtype=np.uint64) if seed_ids is None else np.asarray(seed_ids, np.uint64)
+    sel = shard_indices(n, rank, world)
+    return np.ascontiguousarray(seeds[sel]), np.ascontiguousarray(ids[sel])
+
+
+def reduce_map(map_i32, dst: int = 0, group=None, all_ranks: bool = False):
+    """Combine the ranks' maps in place: reduce to ``dst`` (or all-reduce) with SUM over
+    the int32 view.  ``map_i32`` is a torch int32 tensor holding uint32 counts."""
+    import torch
+    import torch.distributed as dist
+    if map_i32.dtype != torch.int32:
+        raise TypeError("the map must be an int32 view of the uint32 counts")
+    if not dist.is_available() or not dist.is_initialized() or dist.get_world_size(group) == 1:
+        return map_i32
+    if all_ranks:
+        dist.all_reduce(map_i32, op=dist.ReduceOp.SUM, group=group)
+    else:
+        dist.reduce(map_i32, dst=dst, op=dist.ReduceOp.SUM, group=group)
+    return map_i32

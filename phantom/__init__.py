@@ -108,7 +108,7 @@ def _normalize(v: np.ndarray) -> np.ndarray:
 
 def _centres(idx: np.ndarray) -> np.ndarray:
     """Voxel-centre corner coordinates (i + 0.5) for integer indices [n][3] (x,y,z)."""
-    return (idx.astype(np.float32) + np.float32(0.5)).astype(np.float32)
+    return np.ascontiguousarray((idx.astype(np.float32) + np.float32(0.5)).astype(np.float32))
 
 
 def _empty(nx, ny, nz, S, F):

@@ -1,5 +1,3 @@
 set -x
-nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv
-python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -20
-timeout 900 python -m pytest tests -m gpu -x -q -k "not whole_brain" 2>&1 | tail -30
-timeout 600 python bench.py --steps 3 --warmup 3 --cpu-seconds 10 > gpurun_out/bench1.json 2> gpurun_out/bench1.err; tail -5 gpurun_out/bench1.err; cat gpurun_out/bench1.json
+timeout 1500 python -m pytest tests -m gpu -q -k "not whole_brain" > gpurun_out/pytest_gpu.log 2>&1; tail -15 gpurun_out/pytest_gpu.log
+CFG=c3 TAG=r01 timeout 1200 bash scripts/profile.sh

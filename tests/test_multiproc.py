@@ -1,0 +1,77 @@
+"""World-size-2 (and 3) gloo tests of the multi-GPU host logic on CPU: seed sharding with
+global ids + one reduce(SUM) of the int32-viewed maps reproduce the single-process map
+bit for bit.  The per-rank tracker here is the oracle (test infrastructure); on GPUs the
+same shard/reduce code drives libpt.so over NCCL (bench.py)."""
+from __future__ import annotations
+
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        import phantom
+        from paper_conf_ipps_xuzwrwxgxy12_b200 import sharding
+        w = phantom.crossing(sigma=0.15, f_jitter=0.03, nseeds=48, particles_per_seed=60, nsamples=20)
+        seeds, ids = sharding.shard_seeds(w.seeds, w.seed_ids, rank, world)
+        r = oracle.track(w.replace(seeds=seeds, seed_ids=ids))
+        m = torch.from_numpy(r["map"].astype(np.uint32).view(np.int32).copy())
+        sharding.reduce_map(m, dst=0)
+        # uint32 wrap-around survives the int32 reduce: each rank adds 2^31 + rank to cell 0
+        wrap = torch.tensor([np.int32(-2**31 + rank)], dtype=torch.int32)
+        sharding.reduce_map(wrap, all_ranks=True)
+        steps = torch.tensor([int(r["nsteps"].sum())], dtype=torch.int64)
+        dist.all_reduce(steps)
+        if rank == 0:
+            full = oracle.track(w)
+            q.put((m.numpy().view(np.uint32).copy(), full["map"].astype(np.uint32),
+                   int(wrap[0].item()) & 0xFFFFFFFF, int(steps[0]), int(full["nsteps"].sum())))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_sharded_reduce_matches_single_process(world):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got, full, wrap, steps, full_steps = q.get(timeout=600)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    assert np.array_equal(got, full)
+    assert steps == full_steps == int(full.sum(dtype=np.uint64))
+    expect = sum((2**31 + r) for r in range(world)) & 0xFFFFFFFF
+    assert wrap == expect
+
+
+def test_shard_indices_partition():
+    from paper_conf_ipps_xuzwrwxgxy12_b200 import sharding
+    for n in (0, 1, 7, 100):
+        for world in (1, 2, 3, 8):
+            parts = [sharding.shard_indices(n, r, world) for r in range(world)]
+            allp = np.sort(np.concatenate(parts)) if n else np.array([], np.int64)
+            assert np.array_equal(allp, np.arange(n))
+    with pytest.raises(ValueError):
+        sharding.shard_indices(5, 2, 2)
