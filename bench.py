@@ -236,8 +236,9 @@ def run_ours(args):
         flush_buf.fill_(1)  # evict L2 between steps
         tr.track(seeds_d, ids_d, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
                  max_steps=w.max_steps, rng_seed=w.rng_seed,
-                 particles_per_seed=w.particles_per_seed, out_map=out_map, flags=args.track_flags)
-        if world > 1:
+                 particles_per_seed=w.particles_per_seed, out_map=out_map, flags=args.track_flags,
+                 want_map=not args.no_map)
+        if world > 1 and not args.no_map:
             sharding.reduce_map(out_map, dst=0)  # one NCCL reduce; int32 sum == uint32 sum
 
     for _ in range(args.warmup):
@@ -393,6 +394,8 @@ def main(argv=None):
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-gather-bench", action="store_true")
     ap.add_argument("--no-per-step-stats", dest="per_step_stats", action="store_false")
+    ap.add_argument("--no-map", action="store_true", help="diagnostic: no visitation map")
+    ap.add_argument("--tag", default="", help="free-form label echoed by experiment scripts")
     ap.add_argument("--track-flags", type=int, default=0,
                     help="extra pt_params.flags for ablations (e.g. 256 = PT_KERNEL_SIMPLE, "
                          "512 = PT_SEED_ORDER_INPUT)")

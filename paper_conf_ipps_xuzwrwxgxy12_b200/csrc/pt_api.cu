@@ -396,7 +396,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.order = d_order;
     a.nseeds = N;
     a.nparticles = npart;
-    a.chunks_per_seed = (uint32_t)((P + pt::kChunk - 1) / pt::kChunk);
+    a.chunks_per_seed = (uint32_t)((P + pt::kCtaChunk - 1) / pt::kCtaChunk);
     a.total_chunks = N * (uint64_t)a.chunks_per_seed;
     a.map = d_map;
     a.o_nsteps = (fl & PT_REC_LEN) ? c->d_nsteps : nullptr;

@@ -6,8 +6,21 @@
 
 namespace pt {
 
-constexpr int kThreads = 256;       // threads per CTA of the tracking kernel
-constexpr uint32_t kChunk = 32;     // particles claimed per work-queue atomic
+#ifndef PT_CTA_THREADS
+#define PT_CTA_THREADS 1024
+#endif
+#ifndef PT_CTA_CHUNK
+#define PT_CTA_CHUNK PT_CTA_THREADS
+#endif
+// Persistent kernel: one CTA of kThreads per SM; a CTA claims kCtaChunk particles of one
+// seed per global atomic and hands kSub-particle sub-chunks to its warps (shared-memory
+// atomics), so each seed's particles run on few SMs (L1 locality) while the chip as a
+// whole works on a few Morton-adjacent seeds at a time (L2 locality).
+constexpr int kThreads = PT_CTA_THREADS;
+constexpr int kSimpleThreads = 256;  // no-refill ablation kernel
+constexpr uint32_t kCtaChunk = PT_CTA_CHUNK;
+constexpr uint32_t kSub = 32;
+static_assert(kCtaChunk % kSub == 0, "CTA chunk must be a multiple of the sub-chunk");
 
 // Indices of the per-call device counters (unsigned long long[kNumStats]).
 enum StatIdx {
@@ -37,7 +50,7 @@ struct TrackArgs {
     const uint32_t* order;       // [nseeds] processing order (Morton) or nullptr
     uint64_t nseeds;
     uint64_t nparticles;         // nseeds * P
-    uint32_t chunks_per_seed;    // ceil(P / kChunk)
+    uint32_t chunks_per_seed;    // ceil(P / kCtaChunk)
     uint64_t total_chunks;       // nseeds * chunks_per_seed
     uint32_t* map;               // [V] or nullptr
     uint16_t* o_nsteps;          // [nparticles] or nullptr

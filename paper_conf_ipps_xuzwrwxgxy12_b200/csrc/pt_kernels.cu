@@ -28,61 +28,143 @@
 #ifndef PT_MIN_BLOCKS
 #define PT_MIN_BLOCKS 1
 #endif
+#ifndef PT_MAP_CACHE
+#define PT_MAP_CACHE 4096   // entries of the per-CTA shared-memory count cache (power of 2; 0 = off)
+#endif
 
 namespace pt {
 
 enum { kEndMask = 0, kEndCurv = 1, kEndMaxlen = 2 };
 
+// Per-CTA shared-memory cache of visitation counts (REFILL kernel).  Entry = (voxel+1) << 32
+// | count; direct-mapped by a multiplicative hash.  A flush adds to the entry of its voxel
+// or replaces a different voxel's entry, whose count then goes to the global map with one
+// RED; the CTA drains the table at exit.  Integer sums commute, so the map is unchanged.
+constexpr uint32_t kMapCache = PT_MAP_CACHE;
+
+__device__ __forceinline__ void cache_add(unsigned long long* tab, uint32_t* map, uint32_t v, uint32_t c) {
+    constexpr uint32_t kBits = kMapCache > 1 ? 31 - __builtin_clz(kMapCache) : 0;
+    const uint32_t h = kBits ? (v * 0x9E3779B1u) >> (32 - kBits) : 0u;
+    unsigned long long* e = tab + h;
+    const uint32_t key = v + 1u;
+    unsigned long long old = *reinterpret_cast<volatile unsigned long long*>(e);
+    for (;;) {
+        const uint32_t ok = (uint32_t)(old >> 32), oc = (uint32_t)old;
+        const bool same = ok == key && oc < 0x80000000u;
+        const unsigned long long want = same ? old + c : (((unsigned long long)key << 32) | c);
+        const unsigned long long prev = atomicCAS(e, old, want);
+        if (prev == old) {
+            if (!same && ok != 0u) atomicAdd(map + (ok - 1u), oc);
+            return;
+        }
+        old = prev;
+    }
+}
+
+// CTA work distribution (REFILL kernel): s_work packs (CTA chunk index << 24 | tickets
+// taken).  A warp takes ticket t: t < subs(chunk) -> sub-chunk t of the CTA chunk;
+// t == subs -> this warp claims the next global chunk and publishes it; t > subs -> wait
+// for the publication and retry.  Returns (seed index << 32 | first j) or kNoWork.
+constexpr unsigned long long kNoWork = ~0ull;
+constexpr unsigned long long kNoChunk = (1ull << 40) - 1;  // initial "empty" chunk id
+
+__device__ __forceinline__ unsigned long long cta_take(unsigned long long* s_work, const TrackArgs& a) {
+    for (;;) {
+        const unsigned long long old = atomicAdd(s_work, 1ull);
+        const unsigned long long chunk = old >> 24;
+        const uint32_t t = (uint32_t)(old & 0xFFFFFFull);
+        uint32_t subs = 0;
+        uint64_t k = 0, jbase = 0;
+        if (chunk != kNoChunk) {
+            if (chunk >= a.total_chunks) return kNoWork;
+            k = chunk / a.chunks_per_seed;
+            jbase = (chunk - k * a.chunks_per_seed) * (uint64_t)kCtaChunk;
+            const uint64_t cnt = a.P - jbase < kCtaChunk ? a.P - jbase : kCtaChunk;
+            subs = (uint32_t)((cnt + kSub - 1) / kSub);
+        }
+        if (t < subs) {
+            const uint32_t seed = a.order ? a.order[k] : (uint32_t)k;
+            return ((unsigned long long)seed << 32) | (jbase + (uint64_t)t * kSub);
+        }
+        if (t == subs) {
+            const unsigned long long c = atomicAdd(a.stats + kStatQueue, 1ull);
+            atomicExch(s_work, (c << 24) | 1ull);
+            if (c >= a.total_chunks) return kNoWork;
+            const uint64_t k2 = c / a.chunks_per_seed;
+            const uint64_t jb2 = (c - k2 * a.chunks_per_seed) * (uint64_t)kCtaChunk;
+            const uint32_t seed = a.order ? a.order[k2] : (uint32_t)k2;
+            return ((unsigned long long)seed << 32) | jb2;
+        }
+        while ((*reinterpret_cast<volatile unsigned long long*>(s_work) >> 24) == chunk) __nanosleep(64);
+    }
+}
+
 template <int F, bool HALF, bool REFILL>
-__global__ void __launch_bounds__(kThreads, PT_MIN_BLOCKS) track_kernel(const __grid_constant__ TrackArgs a) {
+__global__ void __launch_bounds__(REFILL ? kThreads : kSimpleThreads, PT_MIN_BLOCKS)
+track_kernel(const __grid_constant__ TrackArgs a) {
     using R = Rec<F, HALF>;
     constexpr int RB = R::kBytes;
+    constexpr int TPB = REFILL ? kThreads : kSimpleThreads;
+    // rarely used state lives in shared memory to keep the hot loop's register count low
+    __shared__ unsigned long long s_li[TPB];     // particle index of this call (outputs)
+    __shared__ uint32_t s_q[TPB / 32][3];        // per-warp sub-chunk: seed, next j, end j
+    __shared__ unsigned long long s_work;        // CTA chunk + tickets (see cta_take)
     const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t wib = threadIdx.x >> 5;
     const uint32_t lt_mask = (1u << lane) - 1u;
+    extern __shared__ unsigned long long s_cache[];  // kMapCache entries when REFILL && map
+    constexpr bool kCache = REFILL && kMapCache > 0;
+    const bool use_cache = kCache && a.map != nullptr;
+    if (threadIdx.x == 0) s_work = kNoChunk << 24;
+    if (use_cache)
+        for (uint32_t i = threadIdx.x; i < kMapCache; i += TPB) s_cache[i] = 0ull;
+    __syncthreads();
 
     // ---- per-lane particle state
     bool alive = false;   // lane holds a particle in flight
-    bool pend = false;    // a candidate step waits for the round-start gather (mask test)
+    bool pend = false;    // the round's 3rd candidate step waits for the next round's gather
     float qx = 0.f, qy = 0.f, qz = 0.f;   // committed position, centred coordinates (R10)
     float px = 0.f, py = 0.f, pz = 0.f;   // direction of the last (candidate) step
-    float cqx = 0.f, cqy = 0.f, cqz = 0.f;  // pending candidate position
-    uint32_t gvox = 0;    // voxel read by the round-start gather
+    uint32_t gvox = 0;    // voxel read by the round-start gather (seed or pending candidate)
     int n = 0;            // committed steps
     uint64_t pid = 0;     // global particle id = seed_id * P + j (RNG key, R16)
-    uint64_t li = 0;      // particle index of this call = seed_index * P + j (outputs)
-    uint32_t sign0 = 0;   // first step's sign bit
     uint32_t run_vox = 0, run_cnt = 0;  // run-length merge of consecutive visits
     R rv;                 // record of the current step
     uint4 W = make_uint4(0u, 0u, 0u, 0u);
 
-    // ---- per-lane counters
-    unsigned long long my_steps = 0, my_particles = 0, my_active = 0;
-    unsigned long long rounds = 0;
-
-    // ---- warp-uniform work-queue state
-    uint64_t cseed = 0;
-    uint32_t cnext = 0, cend = 0;
-    bool exhausted = false;
+    // ---- per-lane counters (a lane never sees 2^32 steps in one launch)
+    uint32_t my_steps = 0, my_particles = 0, my_active = 0, rounds = 0;
+    bool exhausted = false;  // warp-uniform
+    if (lane == 0) {
+        s_q[wib][0] = 0u;
+        s_q[wib][1] = 0u;
+        s_q[wib][2] = 0u;
+    }
+    __syncwarp();
 
     auto flush = [&]() {
         if (run_cnt) {
-            atomicAdd(a.map + run_vox, run_cnt);  // no return value used -> RED
+            if (kCache && use_cache) cache_add(s_cache, a.map, run_vox, run_cnt);
+            else atomicAdd(a.map + run_vox, run_cnt);  // no return value used -> RED
             run_cnt = 0;
         }
     };
     // SetEndPoint()
     auto finish = [&](int why) {
-        if (a.o_nsteps) a.o_nsteps[li] = (uint16_t)n;
-        if (a.o_reason) a.o_reason[li] = (uint8_t)why;
-        if (a.o_end) {
-            float* e = a.o_end + 3 * li;
-            e[0] = __fadd_rn(qx, a.fcx);
-            e[1] = __fadd_rn(qy, a.fcy);
-            e[2] = __fadd_rn(qz, a.fcz);
+        if (a.o_nsteps || a.o_reason || a.o_end) {
+            const uint64_t li = s_li[threadIdx.x];
+            if (a.o_nsteps) a.o_nsteps[li] = (uint16_t)n;
+            if (a.o_reason) a.o_reason[li] = (uint8_t)why;
+            if (a.o_end) {
+                float* e = a.o_end + 3 * li;
+                e[0] = __fadd_rn(qx, a.fcx);
+                e[1] = __fadd_rn(qy, a.fcy);
+                e[2] = __fadd_rn(qz, a.fcz);
+            }
         }
         if (a.map) flush();
-        my_steps += (unsigned long long)n;
-        my_particles += 1ull;
+        my_steps += (uint32_t)n;
+        my_particles += 1u;
         alive = false;
         pend = false;
     };
@@ -102,7 +184,7 @@ __global__ void __launch_bounds__(kThreads, PT_MIN_BLOCKS) track_kernel(const __
             }
         }
         if (a.o_paths && n < a.path_stride) {
-            float* pp = a.o_paths + (li * (uint64_t)a.path_stride + (uint64_t)n) * 3u;
+            float* pp = a.o_paths + (s_li[threadIdx.x] * (uint64_t)a.path_stride + (uint64_t)n) * 3u;
             pp[0] = __fadd_rn(qx, a.fcx);
             pp[1] = __fadd_rn(qy, a.fcy);
             pp[2] = __fadd_rn(qz, a.fcz);
@@ -110,7 +192,8 @@ __global__ void __launch_bounds__(kThreads, PT_MIN_BLOCKS) track_kernel(const __
     };
     // GetStartPoint(): centred seed position, seed voxel (R10, R12)
     auto start = [&](uint64_t si, uint64_t j) {
-        li = si * a.P + j;
+        const uint64_t li = si * a.P + j;
+        s_li[threadIdx.x] = li;
         const uint64_t sid = a.seed_ids ? a.seed_ids[si] : si;
         pid = sid * a.P + j;
         qx = __fsub_rn(a.seeds[3 * si + 0], a.fcx);
@@ -136,7 +219,7 @@ __global__ void __launch_bounds__(kThreads, PT_MIN_BLOCKS) track_kernel(const __
     };
 
     if (!REFILL) {
-        const uint64_t g = (uint64_t)blockIdx.x * kThreads + threadIdx.x;
+        const uint64_t g = (uint64_t)blockIdx.x * TPB + threadIdx.x;
         if (g < a.nparticles) {
             const uint64_t si = g / a.P;
             start(si, g - si * a.P);
@@ -148,31 +231,40 @@ __global__ void __launch_bounds__(kThreads, PT_MIN_BLOCKS) track_kernel(const __
         // paper's CPU Reduction()/segment relaunch)
         if (REFILL) {
             uint32_t need = __ballot_sync(kFull, !alive);
-            while (need != 0u && !exhausted) {
-                if (cnext == cend) {
-                    unsigned long long c = 0;
-                    if (lane == 0) c = atomicAdd(a.stats + kStatQueue, 1ull);
-                    c = __shfl_sync(kFull, c, 0);
-                    if (c >= a.total_chunks) {
-                        exhausted = true;
-                        break;
+            if (need != 0u && !exhausted) {
+                uint32_t cseed = s_q[wib][0], cnext = s_q[wib][1], cend = s_q[wib][2];
+                while (need != 0u) {
+                    if (cnext == cend) {
+                        unsigned long long r = 0;
+                        if (lane == 0) r = cta_take(&s_work, a);
+                        r = __shfl_sync(kFull, r, 0);
+                        if (r == kNoWork) {
+                            exhausted = true;
+                            break;
+                        }
+                        cseed = (uint32_t)(r >> 32);
+                        cnext = (uint32_t)r;
+                        const uint64_t e = (uint64_t)cnext + kSub;
+                        cend = (uint32_t)(e < a.P ? e : a.P);
                     }
-                    const uint64_t k = c / a.chunks_per_seed;
-                    cnext = (uint32_t)(c - k * a.chunks_per_seed) * kChunk;
-                    cseed = a.order ? (uint64_t)a.order[k] : k;
-                    const uint64_t e = (uint64_t)cnext + kChunk;
-                    cend = (uint32_t)(e < a.P ? e : a.P);
+                    const uint32_t avail = cend - cnext;
+                    const uint32_t rank = __popc(need & lt_mask);
+                    if (!alive && rank < avail) start(cseed, (uint64_t)(cnext + rank));
+                    const uint32_t cnt = (uint32_t)__popc(need);
+                    cnext += cnt < avail ? cnt : avail;
+                    need = __ballot_sync(kFull, !alive);
                 }
-                const uint32_t avail = cend - cnext;
-                const uint32_t rank = __popc(need & lt_mask);
-                if (!alive && rank < avail) start(cseed, (uint64_t)(cnext + rank));
-                const uint32_t cnt = (uint32_t)__popc(need);
-                cnext += cnt < avail ? cnt : avail;
-                need = __ballot_sync(kFull, !alive);
+                __syncwarp();
+                if (lane == 0) {
+                    s_q[wib][0] = cseed;
+                    s_q[wib][1] = cnext;
+                    s_q[wib][2] = cend;
+                }
+                __syncwarp();
             }
         }
         if (!__any_sync(kFull, alive)) break;
-        rounds += 1ull;
+        rounds += 1u;
 
         // ------------------------------------------------ round start: one Philox block,
         // gather of (pending candidate | seed) voxel = mask test + first step's record
@@ -183,19 +275,18 @@ __global__ void __launch_bounds__(kThreads, PT_MIN_BLOCKS) track_kernel(const __
             ldg_record<RB>(a.rec + ((uint64_t)gvox * a.S + sample_of(W.x, a.S)) * RB, rv.w);
             if (rv.outside()) {
                 finish(kEndMask);  // seed outside the mask (R12) or candidate rejected (R11)
-            } else {
-                if (pend) {
-                    commit(cqx, cqy, cqz, gvox);
-                    pend = false;
-                }
-                if (n == 0) sign0 = W.w >> 31;
+            } else if (pend) {
+                // the candidate is recomputed bit-identically from (q, d) instead of kept
+                commit(__fadd_rn(qx, __fmul_rn(a.step, px)), __fadd_rn(qy, __fmul_rn(a.step, py)),
+                       __fadd_rn(qz, __fmul_rn(a.step, pz)), gvox);
+                pend = false;
             }
         }
 
         // ------------------------------------------------ three steps
 #pragma unroll
         for (int k = 0; k < 3; ++k) {
-            my_active += alive ? 1ull : 0ull;
+            my_active += alive ? 1u : 0u;
             if (alive) {
                 if (n == a.max_steps) {
                     finish(kEndMaxlen);  // maximum number of steps (R14)
@@ -204,8 +295,10 @@ __global__ void __launch_bounds__(kThreads, PT_MIN_BLOCKS) track_kernel(const __
                     bool go = true;
                     float sg;
                     if (n == 0) {
-                        rv.fibre(0, vx, vy, vz, fj);  // R5, R6
-                        sg = sign0 ? -1.f : 1.f;
+                        // first step (always k == 0 of a lane's first round, W = block 0):
+                        // fibre 0, sign = top bit of word 3 (R5, R6, R16)
+                        rv.fibre(0, vx, vy, vz, fj);
+                        sg = (W.w >> 31) ? -1.f : 1.f;
                     } else {
                         // choose the fibre closest to the previous direction:
                         // eligible iff f_j > fib_thr (R7), strict >, lowest j wins (R8)
@@ -240,15 +333,12 @@ __global__ void __launch_bounds__(kThreads, PT_MIN_BLOCKS) track_kernel(const __
                     }
                     if (go) {
                         // StepToNextPoint(): q' = q + h * (sign * v), no FMA
-                        const float dx = sg < 0.f ? -vx : vx;
-                        const float dy = sg < 0.f ? -vy : vy;
-                        const float dz = sg < 0.f ? -vz : vz;
-                        px = dx;
-                        py = dy;
-                        pz = dz;
-                        const float nqx = __fadd_rn(qx, __fmul_rn(a.step, dx));
-                        const float nqy = __fadd_rn(qy, __fmul_rn(a.step, dy));
-                        const float nqz = __fadd_rn(qz, __fmul_rn(a.step, dz));
+                        px = sg < 0.f ? -vx : vx;
+                        py = sg < 0.f ? -vy : vy;
+                        pz = sg < 0.f ? -vz : vz;
+                        const float nqx = __fadd_rn(qx, __fmul_rn(a.step, px));
+                        const float nqy = __fadd_rn(qy, __fmul_rn(a.step, py));
+                        const float nqz = __fadd_rn(qz, __fmul_rn(a.step, pz));
                         const int ix = axis_index(nqx, a.cx), iy = axis_index(nqy, a.cy),
                                   iz = axis_index(nqz, a.cz);
                         if (!((unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny &&
@@ -267,15 +357,21 @@ __global__ void __launch_bounds__(kThreads, PT_MIN_BLOCKS) track_kernel(const __
                                 }
                             } else {
                                 pend = true;  // next round's start gathers and tests it
-                                cqx = nqx;
-                                cqy = nqy;
-                                cqz = nqz;
                                 gvox = v;
                             }
                         }
                     }
                 }
             }
+        }
+    }
+
+    // ---- drain the count cache
+    if (kCache && use_cache) {
+        __syncthreads();
+        for (uint32_t i = threadIdx.x; i < kMapCache; i += TPB) {
+            const unsigned long long e = s_cache[i];
+            if (e >> 32) atomicAdd(a.map + ((uint32_t)(e >> 32) - 1u), (uint32_t)e);
         }
     }
 
@@ -287,10 +383,10 @@ __global__ void __launch_bounds__(kThreads, PT_MIN_BLOCKS) track_kernel(const __
         my_active += __shfl_xor_sync(kFull, my_active, o);
     }
     if (lane == 0) {
-        atomicAdd(a.stats + kStatSteps, my_steps);
-        atomicAdd(a.stats + kStatParticles, my_particles);
-        atomicAdd(a.stats + kStatLaneActive, my_active);
-        atomicAdd(a.stats + kStatLaneSlots, rounds * 3ull * 32ull);
+        atomicAdd(a.stats + kStatSteps, (unsigned long long)my_steps);
+        atomicAdd(a.stats + kStatParticles, (unsigned long long)my_particles);
+        atomicAdd(a.stats + kStatLaneActive, (unsigned long long)my_active);
+        atomicAdd(a.stats + kStatLaneSlots, (unsigned long long)rounds * 3ull * 32ull);
     }
 }
 
@@ -425,20 +521,25 @@ __global__ void __launch_bounds__(256) gather_bench_kernel(const uint8_t* __rest
 template <int F, bool HALF, bool REFILL>
 static cudaError_t launch_t(const TrackArgs& a, int num_sms, cudaStream_t st) {
     auto k = track_kernel<F, HALF, REFILL>;
+    constexpr int TPB = REFILL ? kThreads : kSimpleThreads;
     if (a.nparticles == 0) return cudaSuccess;
     unsigned grid;
+    const size_t dyn = (REFILL && kMapCache > 0 && a.map) ? kMapCache * sizeof(unsigned long long) : 0;
     if (REFILL) {
         int per_sm = 0;
-        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kThreads, 0);
+        cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)(kMapCache * sizeof(unsigned long long)));
         if (e != cudaSuccess) return e;
-        if (per_sm < 1) per_sm = 1;
-        const uint64_t need = (a.nparticles + kThreads - 1) / kThreads;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, TPB, dyn);
+        if (e != cudaSuccess) return e;
+        if (per_sm < 1) return cudaErrorInvalidConfiguration;
+        const uint64_t need = (a.nparticles + TPB - 1) / TPB;
         const uint64_t full = (uint64_t)num_sms * (uint64_t)per_sm;
         grid = (unsigned)(need < full ? need : full);
     } else {
-        grid = (unsigned)((a.nparticles + kThreads - 1) / kThreads);
+        grid = (unsigned)((a.nparticles + TPB - 1) / TPB);
     }
-    k<<<grid, kThreads, 0, st>>>(a);
+    k<<<grid, TPB, dyn, st>>>(a);
     return cudaGetLastError();
 }
 
@@ -463,7 +564,8 @@ cudaError_t launch_track(const TrackArgs& a, int nfibres, bool half, bool simple
 template <int F, bool HALF, bool REFILL>
 static int bps() {
     int per_sm = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, track_kernel<F, HALF, REFILL>, kThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, track_kernel<F, HALF, REFILL>,
+                                                  REFILL ? kThreads : kSimpleThreads, 0);
     return per_sm;
 }
 

@@ -1,0 +1,7 @@
+set -x
+PT_LIB=$PWD/scripts/libpt_mc16384.so timeout 900 python -m pytest tests -m gpu -q -x -k "not whole_brain" > gpurun_out/pytest_gpu.log 2>&1; tail -3 gpurun_out/pytest_gpu.log
+run() { timeout 300 python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-gather-bench "$@" 2>&1 | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('RES', sys.argv[1:], d['value']/1e9, d['roofline']['kernel_ms'])" "$@"; }
+for T in 16384 8192 4096; do
+PT_LIB=$PWD/scripts/libpt_mc$T.so run --config c3 --tag mc$T
+PT_LIB=$PWD/scripts/libpt_mc$T.so run --config c4 --tag mc$T
+done
