@@ -222,6 +222,9 @@ def run_ours(args):
     torch.cuda.set_device(dev)
 
     w = _workload(args.config)
+    if args.seed_every > 1:
+        import phantom
+        w = phantom.wm_seeds(w, every=args.seed_every)
     mine = _shard(w, rank, world)
     tr = pt.Tracker(local)
     tr.load_volume(w.volume)
@@ -253,7 +256,7 @@ def run_ours(args):
     torch.cuda.synchronize()
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
-    kern_ms = []
+    kern_ms, track_ms = [], []
     steps_done = 0
     e0.record()
     for _ in range(args.steps):
@@ -261,6 +264,7 @@ def run_ours(args):
         s = tr.stats() if args.per_step_stats else None
         if s:
             kern_ms.append(s["kernel_ms"])
+            track_ms.append(s["track_ms"])
             steps_done += s["total_steps"]
     e1.record()
     torch.cuda.synchronize()
@@ -323,7 +327,8 @@ def run_ours(args):
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": achieved / peak, "traffic": _ncu_traffic(args.config),
             "peak_source": "measured (MEASURED_PEAKS.json hbm_gbs)" if peaks else "fallback 6.65 TB/s",
-            "bytes_per_step": rb + 8, "kernel_ms": kms}
+            "bytes_per_step": rb + 8, "kernel_ms": kms,
+            "kernel_ms_steps": kern_ms, "track_ms_steps": track_ms}
     gather = None
     if rank == 0 and not args.no_gather_bench:
         rec_bytes_total = V * w.volume.nsamples * rb
@@ -396,6 +401,8 @@ def main(argv=None):
     ap.add_argument("--no-per-step-stats", dest="per_step_stats", action="store_false")
     ap.add_argument("--no-map", action="store_true", help="diagnostic: no visitation map")
     ap.add_argument("--tag", default="", help="free-form label echoed by experiment scripts")
+    ap.add_argument("--seed-every", type=int, default=1,
+                    help="diagnostic (profiling only): every k-th seed of the workload")
     ap.add_argument("--track-flags", type=int, default=0,
                     help="extra pt_params.flags for ablations (e.g. 256 = PT_KERNEL_SIMPLE, "
                          "512 = PT_SEED_ORDER_INPUT)")

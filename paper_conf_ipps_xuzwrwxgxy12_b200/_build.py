@@ -18,7 +18,7 @@ NVCC_FLAGS = [
     "-O3", "-lineinfo", "-std=c++17",
     "-fmad=false",          # no FMA contraction anywhere in the library (R15)
     "-Xcompiler", "-fPIC", "-shared",
-    "-Xptxas", "-warn-spills",
+    "-Xptxas", "-warn-spills", "-diag-suppress", "186",
 ]
 
 

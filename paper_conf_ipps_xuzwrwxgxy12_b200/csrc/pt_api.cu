@@ -31,10 +31,10 @@ struct pt_ctx {
     size_t seeds_cap = 0;
     uint64_t* d_ids = nullptr;
     size_t ids_cap = 0;
-    uint64_t* d_keys = nullptr;  // seed-order sort keys
-    size_t keys_cap = 0;
-    uint32_t* d_perm = nullptr;  // seed processing order
-    size_t perm_cap = 0;
+    uint32_t* d_order = nullptr;  // seed order: 4 x nseeds u32 (keys, sorted keys, idx, perm)
+    size_t order_cap = 0;
+    uint8_t* d_temp = nullptr;    // radix-sort temp storage
+    size_t temp_cap = 0;
     uint32_t* d_map = nullptr;   // internal map for host map pointers
     size_t map_cap = 0;
     uint16_t* d_nsteps = nullptr;
@@ -183,7 +183,7 @@ void pt_destroy(pt_ctx* c) {
     DeviceGuard g(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
     else cudaDeviceSynchronize();
-    void* bufs[] = {c->d_rec, c->d_seeds, c->d_ids, c->d_keys, c->d_perm, c->d_map, c->d_nsteps,
+    void* bufs[] = {c->d_rec, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_nsteps,
                     c->d_reason, c->d_end, c->d_paths, c->d_stats};
     for (void* b : bufs)
         if (b) cudaFree(b);
@@ -366,10 +366,13 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     const uint32_t* d_order = nullptr;
     if (!(fl & (PT_SEED_ORDER_INPUT | PT_KERNEL_SIMPLE)) && N > 1) {
         if (N > 0xFFFFFFFFull) return fail(c, PT_ERR_ARG, "pt_track: more than 2^32-1 seeds");
-        CK(ensure(c->d_keys, c->keys_cap, N), "pt_track: order keys");
-        CK(ensure(c->d_perm, c->perm_cap, N), "pt_track: order buffer");
-        CK(pt::launch_seed_order(d_seeds, N, c->d_keys, c->d_perm, st), "pt_track: seed order");
-        d_order = c->d_perm;
+        CK(ensure(c->d_order, c->order_cap, 4 * N), "pt_track: order buffers");
+        const size_t tb = pt::seed_order_temp_bytes(N);
+        CK(ensure(c->d_temp, c->temp_cap, tb), "pt_track: sort temp storage");
+        CK(pt::launch_seed_order(d_seeds, N, c->d_order, c->d_order + N, c->d_order + 2 * N, c->d_order + 3 * N,
+                                 c->d_temp, c->temp_cap, st),
+           "pt_track: seed order");
+        d_order = c->d_order + 3 * N;
     }
 
     pt::TrackArgs a{};

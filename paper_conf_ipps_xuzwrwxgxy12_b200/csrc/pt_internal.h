@@ -69,9 +69,11 @@ cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask,
                           int64_t V, int S, int F, bool half, int rec_bytes,
                           unsigned long long* bad, cudaStream_t st);
 // Z-order processing permutation of the seeds: perm[k] = index of the k-th seed in Morton
-// order of its voxel (ties by input index).  keys/perm/tmp are device buffers of nseeds.
-cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint64_t* keys, uint32_t* perm,
-                              cudaStream_t st);
+// order of its voxel (ties by input index; stable radix sort).  keys, keys_out, idx, perm:
+// device buffers of nseeds; temp: seed_order_temp_bytes(nseeds) bytes.
+size_t seed_order_temp_bytes(uint64_t nseeds);
+cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint32_t* keys, uint32_t* keys_out,
+                              uint32_t* idx, uint32_t* perm, void* temp, size_t temp_bytes, cudaStream_t st);
 cudaError_t launch_map_sum(const uint32_t* map, int64_t V, unsigned long long* out,
                            cudaStream_t st);
 cudaError_t launch_gather_bench(const uint8_t* buf, uint64_t nrec, int rec_bytes, uint32_t iters,

@@ -17,8 +17,7 @@
 // the third step's gather is deferred to the next round's start, where it is issued by
 // the same instruction as the first gather of freshly refilled lanes.
 #include <cuda_runtime.h>
-#include <thrust/execution_policy.h>
-#include <thrust/sort.h>
+#include <cub/device/device_radix_sort.cuh>
 
 #include <cstdint>
 
@@ -29,7 +28,7 @@
 #define PT_MIN_BLOCKS 1
 #endif
 #ifndef PT_MAP_CACHE
-#define PT_MAP_CACHE 4096   // entries of the per-CTA shared-memory count cache (power of 2; 0 = off)
+#define PT_MAP_CACHE 0      // entries of the per-CTA shared-memory count cache (power of 2; 0 = off)
 #endif
 
 namespace pt {
@@ -116,8 +115,10 @@ track_kernel(const __grid_constant__ TrackArgs a) {
     constexpr bool kCache = REFILL && kMapCache > 0;
     const bool use_cache = kCache && a.map != nullptr;
     if (threadIdx.x == 0) s_work = kNoChunk << 24;
-    if (use_cache)
-        for (uint32_t i = threadIdx.x; i < kMapCache; i += TPB) s_cache[i] = 0ull;
+    if constexpr (kCache) {
+        if (use_cache)
+            for (uint32_t i = threadIdx.x; i < kMapCache; i += TPB) s_cache[i] = 0ull;
+    }
     __syncthreads();
 
     // ---- per-lane particle state
@@ -142,15 +143,21 @@ track_kernel(const __grid_constant__ TrackArgs a) {
     }
     __syncwarp();
 
-    auto flush = [&]() {
-        if (run_cnt) {
-            if (kCache && use_cache) cache_add(s_cache, a.map, run_vox, run_cnt);
-            else atomicAdd(a.map + run_vox, run_cnt);  // no return value used -> RED
-            run_cnt = 0;
-        }
+    int why = -1;  // >= 0: the particle ended with this reason; outputs pending (finish())
+
+    auto red = [&](uint32_t v, uint32_t c) {
+        if (kCache && use_cache) cache_add(s_cache, a.map, v, c);
+        else atomicAdd(a.map + v, c);  // no return value used -> RED
+    };
+    // a termination only records the reason; the outputs are written once per round for
+    // all ended lanes at the top of the loop (one divergent block instead of one per site)
+    auto end = [&](int w) {
+        why = w;
+        alive = false;
+        pend = false;
     };
     // SetEndPoint()
-    auto finish = [&](int why) {
+    auto finish = [&]() {
         if (a.o_nsteps || a.o_reason || a.o_end) {
             const uint64_t li = s_li[threadIdx.x];
             if (a.o_nsteps) a.o_nsteps[li] = (uint16_t)n;
@@ -162,26 +169,24 @@ track_kernel(const __grid_constant__ TrackArgs a) {
                 e[2] = __fadd_rn(qz, a.fcz);
             }
         }
-        if (a.map) flush();
+        if (a.map && run_cnt) red(run_vox, run_cnt);
+        run_cnt = 0;
         my_steps += (uint32_t)n;
         my_particles += 1u;
-        alive = false;
-        pend = false;
+        why = -1;
     };
-    // commit a step: new position, one visit of the new voxel (R13)
+    // commit a step: new position, one visit of the new voxel (R13); consecutive
+    // visits of the same voxel are merged (run length) and flushed when the voxel changes
     auto commit = [&](float x, float y, float z, uint32_t v) {
         qx = x;
         qy = y;
         qz = z;
         n += 1;
         if (a.map) {
-            if (run_cnt != 0u && v == run_vox) {
-                run_cnt += 1u;
-            } else {
-                flush();
-                run_vox = v;
-                run_cnt = 1u;
-            }
+            const bool change = v != run_vox;
+            if (change && run_cnt != 0u) red(run_vox, run_cnt);
+            run_cnt = change ? 1u : run_cnt + 1u;
+            run_vox = v;
         }
         if (a.o_paths && n < a.path_stride) {
             float* pp = a.o_paths + (s_li[threadIdx.x] * (uint64_t)a.path_stride + (uint64_t)n) * 3u;
@@ -214,7 +219,8 @@ track_kernel(const __grid_constant__ TrackArgs a) {
             (unsigned)iz < (unsigned)a.nz) {
             gvox = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
         } else {
-            finish(kEndMask);
+            end(kEndMask);  // seed outside the volume (R12): finished right away, so the
+            finish();       // refill loop may hand this lane another particle
         }
     };
 
@@ -227,6 +233,8 @@ track_kernel(const __grid_constant__ TrackArgs a) {
     }
 
     for (;;) {
+        if (why >= 0) finish();  // particles that ended during the previous round
+
         // ------------------------------------------------ lane refill (replaces the
         // paper's CPU Reduction()/segment relaunch)
         if (REFILL) {
@@ -274,7 +282,7 @@ track_kernel(const __grid_constant__ TrackArgs a) {
                               a.key0, a.key1);
             ldg_record<RB>(a.rec + ((uint64_t)gvox * a.S + sample_of(W.x, a.S)) * RB, rv.w);
             if (rv.outside()) {
-                finish(kEndMask);  // seed outside the mask (R12) or candidate rejected (R11)
+                end(kEndMask);  // seed outside the mask (R12) or candidate rejected (R11)
             } else if (pend) {
                 // the candidate is recomputed bit-identically from (q, d) instead of kept
                 commit(__fadd_rn(qx, __fmul_rn(a.step, px)), __fadd_rn(qy, __fmul_rn(a.step, py)),
@@ -289,11 +297,11 @@ track_kernel(const __grid_constant__ TrackArgs a) {
             my_active += alive ? 1u : 0u;
             if (alive) {
                 if (n == a.max_steps) {
-                    finish(kEndMaxlen);  // maximum number of steps (R14)
+                    end(kEndMaxlen);  // maximum number of steps (R14)
                 } else {
                     float vx, vy, vz, fj;
-                    bool go = true;
                     float sg;
+                    bool go = true;
                     if (n == 0) {
                         // first step (always k == 0 of a lane's first round, W = block 0):
                         // fibre 0, sign = top bit of word 3 (R5, R6, R16)
@@ -302,14 +310,11 @@ track_kernel(const __grid_constant__ TrackArgs a) {
                     } else {
                         // choose the fibre closest to the previous direction:
                         // eligible iff f_j > fib_thr (R7), strict >, lowest j wins (R8)
-                        float bc = 0.f, best = -1.f;
+                        float best = -1.f;
                         rv.fibre(0, vx, vy, vz, fj);
-                        {
-                            const float c0 = __fadd_rn(__fadd_rn(__fmul_rn(vx, px), __fmul_rn(vy, py)),
-                                                       __fmul_rn(vz, pz));
-                            bc = c0;
-                            if (fj > a.fib_thr) best = fabsf(c0);
-                        }
+                        float bc = __fadd_rn(__fadd_rn(__fmul_rn(vx, px), __fmul_rn(vy, py)),
+                                             __fmul_rn(vz, pz));
+                        if (fj > a.fib_thr) best = fabsf(bc);
 #pragma unroll
                         for (int j = 1; j < F; ++j) {
                             float ux, uy, uz, fu;
@@ -325,10 +330,8 @@ track_kernel(const __grid_constant__ TrackArgs a) {
                             }
                         }
                         // maximum angle, measured by the dot product (R4)
-                        if (!(fabsf(bc) > a.curv_thr)) {
-                            finish(kEndCurv);
-                            go = false;
-                        }
+                        go = fabsf(bc) > a.curv_thr;
+                        if (!go) end(kEndCurv);
                         sg = bc > 0.f ? 1.f : -1.f;  // keep the orientation (R9)
                     }
                     if (go) {
@@ -343,18 +346,15 @@ track_kernel(const __grid_constant__ TrackArgs a) {
                                   iz = axis_index(nqz, a.cz);
                         if (!((unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny &&
                               (unsigned)iz < (unsigned)a.nz)) {
-                            finish(kEndMask);  // left the volume (R11)
+                            end(kEndMask);  // left the volume (R11)
                         } else {
                             const uint32_t v =
                                 ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
                             if (k < 2) {
                                 const uint32_t w = (k == 0) ? W.y : W.z;
                                 ldg_record<RB>(a.rec + ((uint64_t)v * a.S + sample_of(w, a.S)) * RB, rv.w);
-                                if (rv.outside()) {
-                                    finish(kEndMask);  // candidate outside the mask (R11)
-                                } else {
-                                    commit(nqx, nqy, nqz, v);
-                                }
+                                if (rv.outside()) end(kEndMask);  // candidate outside the mask (R11)
+                                else commit(nqx, nqy, nqz, v);
                             } else {
                                 pend = true;  // next round's start gathers and tests it
                                 gvox = v;
@@ -367,11 +367,13 @@ track_kernel(const __grid_constant__ TrackArgs a) {
     }
 
     // ---- drain the count cache
-    if (kCache && use_cache) {
-        __syncthreads();
-        for (uint32_t i = threadIdx.x; i < kMapCache; i += TPB) {
-            const unsigned long long e = s_cache[i];
-            if (e >> 32) atomicAdd(a.map + ((uint32_t)(e >> 32) - 1u), (uint32_t)e);
+    if constexpr (kCache) {
+        if (use_cache) {
+            __syncthreads();
+            for (uint32_t i = threadIdx.x; i < kMapCache; i += TPB) {
+                const unsigned long long e = s_cache[i];
+                if (e >> 32) atomicAdd(a.map + ((uint32_t)(e >> 32) - 1u), (uint32_t)e);
+            }
         }
     }
 
@@ -457,8 +459,8 @@ __device__ __forceinline__ uint64_t spread3(uint32_t v) {
     return x;
 }
 
-__global__ void seed_keys_kernel(const float* __restrict__ seeds, uint64_t n, uint64_t* keys,
-                                 uint32_t* perm) {
+__global__ void seed_keys_kernel(const float* __restrict__ seeds, uint64_t n, uint32_t* keys,
+                                 uint32_t* idx) {
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
         uint32_t c[3];
 #pragma unroll
@@ -466,22 +468,28 @@ __global__ void seed_keys_kernel(const float* __restrict__ seeds, uint64_t n, ui
             const float x = seeds[3 * i + a];
             c[a] = x <= 0.f ? 0u : (x >= 1023.f ? 1023u : (uint32_t)x);
         }
-        const uint64_t m = spread3(c[0]) | (spread3(c[1]) << 1) | (spread3(c[2]) << 2);
-        keys[i] = (m << 32) | (uint64_t)(uint32_t)i;
-        perm[i] = (uint32_t)i;
+        keys[i] = (uint32_t)(spread3(c[0]) | (spread3(c[1]) << 1) | (spread3(c[2]) << 2));
+        idx[i] = (uint32_t)i;
     }
 }
 
-cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint64_t* keys, uint32_t* perm,
-                              cudaStream_t st) {
+size_t seed_order_temp_bytes(uint64_t nseeds) {
+    size_t bytes = 0;
+    cub::DeviceRadixSort::SortPairs(nullptr, bytes, (const uint32_t*)nullptr, (uint32_t*)nullptr,
+                                    (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)nseeds, 0, 30);
+    return bytes;
+}
+
+cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint32_t* keys, uint32_t* keys_out,
+                              uint32_t* idx, uint32_t* perm, void* temp, size_t temp_bytes, cudaStream_t st) {
     if (nseeds == 0) return cudaSuccess;
     uint64_t blocks = (nseeds + 255) / 256;
     if (blocks > 148 * 16) blocks = 148 * 16;
-    seed_keys_kernel<<<(unsigned)blocks, 256, 0, st>>>(seeds, nseeds, keys, perm);
+    seed_keys_kernel<<<(unsigned)blocks, 256, 0, st>>>(seeds, nseeds, keys, idx);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
-    thrust::sort_by_key(thrust::cuda::par.on(st), keys, keys + nseeds, perm);
-    return cudaGetLastError();
+    // stable radix sort on the 30-bit Morton code: ties keep the input order
+    return cub::DeviceRadixSort::SortPairs(temp, temp_bytes, keys, keys_out, idx, perm, (int)nseeds, 0, 30, st);
 }
 
 // ------------------------------------------------------------------------- map sum

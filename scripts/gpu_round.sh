@@ -1,3 +1,2 @@
 set -x
-timeout 1500 python -m pytest tests -m gpu -q -k "not whole_brain" > gpurun_out/pytest_gpu.log 2>&1; tail -15 gpurun_out/pytest_gpu.log
-CFG=c3 TAG=r01 timeout 1200 bash scripts/profile.sh
+CFG=c3 TAG=r01b timeout 1500 bash scripts/profile.sh
