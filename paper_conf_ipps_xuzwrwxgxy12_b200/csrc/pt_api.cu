@@ -399,7 +399,17 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.order = d_order;
     a.nseeds = N;
     a.nparticles = npart;
-    a.chunks_per_seed = (uint32_t)((P + pt::kCtaChunk - 1) / pt::kCtaChunk);
+    {
+        // a whole seed per CTA claim when there are >= 8 claims per SM, else smaller chunks
+        const uint64_t P32 = (P + pt::kSub - 1) / pt::kSub * pt::kSub;
+        uint64_t ch = npart / (8ull * (uint64_t)(c->num_sms > 0 ? c->num_sms : 1));
+        ch = (ch + pt::kSub - 1) / pt::kSub * pt::kSub;
+        if (ch < pt::kMinCtaChunk) ch = pt::kMinCtaChunk;
+        if (ch > P32) ch = P32;
+        if (ch > (1ull << 27)) ch = 1ull << 27;  // keeps tickets per chunk < 2^22 (cta_take)
+        a.cta_chunk = (uint32_t)ch;
+    }
+    a.chunks_per_seed = (uint32_t)((P + a.cta_chunk - 1) / a.cta_chunk);
     a.total_chunks = N * (uint64_t)a.chunks_per_seed;
     a.map = d_map;
     a.o_nsteps = (fl & PT_REC_LEN) ? c->d_nsteps : nullptr;

@@ -9,18 +9,15 @@ namespace pt {
 #ifndef PT_CTA_THREADS
 #define PT_CTA_THREADS 1024
 #endif
-#ifndef PT_CTA_CHUNK
-#define PT_CTA_CHUNK PT_CTA_THREADS
-#endif
-// Persistent kernel: one CTA of kThreads per SM; a CTA claims kCtaChunk particles of one
-// seed per global atomic and hands kSub-particle sub-chunks to its warps (shared-memory
-// atomics), so each seed's particles run on few SMs (L1 locality) while the chip as a
-// whole works on a few Morton-adjacent seeds at a time (L2 locality).
+// Persistent kernel: one CTA of kThreads per SM; a CTA claims a chunk of cta_chunk particles
+// of one seed per global atomic (cta_chunk chosen per call, see pt_track: a whole seed when
+// there is enough work) and hands kSub-particle sub-chunks to its warps (shared-memory
+// tickets), so a seed's particles run on one SM (L1 locality) while the chip as a whole
+// works on a compact set of Morton-adjacent seeds (L2 locality).
 constexpr int kThreads = PT_CTA_THREADS;
 constexpr int kSimpleThreads = 256;  // no-refill ablation kernel
-constexpr uint32_t kCtaChunk = PT_CTA_CHUNK;
 constexpr uint32_t kSub = 32;
-static_assert(kCtaChunk % kSub == 0, "CTA chunk must be a multiple of the sub-chunk");
+constexpr uint32_t kMinCtaChunk = 1024;
 
 // Indices of the per-call device counters (unsigned long long[kNumStats]).
 enum StatIdx {
@@ -50,7 +47,8 @@ struct TrackArgs {
     const uint32_t* order;       // [nseeds] processing order (Morton) or nullptr
     uint64_t nseeds;
     uint64_t nparticles;         // nseeds * P
-    uint32_t chunks_per_seed;    // ceil(P / kCtaChunk)
+    uint32_t cta_chunk;          // particles per CTA claim (multiple of kSub)
+    uint32_t chunks_per_seed;    // ceil(P / cta_chunk)
     uint64_t total_chunks;       // nseeds * chunks_per_seed
     uint32_t* map;               // [V] or nullptr
     uint16_t* o_nsteps;          // [nparticles] or nullptr
@@ -64,7 +62,6 @@ struct TrackArgs {
 // Launchers (return the launch error, if any).
 cudaError_t launch_track(const TrackArgs& a, int nfibres, bool half, bool simple, int num_sms,
                          cudaStream_t st);
-int track_blocks_per_sm(int nfibres, bool half, bool simple);
 cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask, uint8_t* rec,
                           int64_t V, int S, int F, bool half, int rec_bytes,
                           unsigned long long* bad, cudaStream_t st);

@@ -77,8 +77,8 @@ __device__ __forceinline__ unsigned long long cta_take(unsigned long long* s_wor
         if (chunk != kNoChunk) {
             if (chunk >= a.total_chunks) return kNoWork;
             k = chunk / a.chunks_per_seed;
-            jbase = (chunk - k * a.chunks_per_seed) * (uint64_t)kCtaChunk;
-            const uint64_t cnt = a.P - jbase < kCtaChunk ? a.P - jbase : kCtaChunk;
+            jbase = (chunk - k * a.chunks_per_seed) * (uint64_t)a.cta_chunk;
+            const uint64_t cnt = a.P - jbase < a.cta_chunk ? a.P - jbase : a.cta_chunk;
             subs = (uint32_t)((cnt + kSub - 1) / kSub);
         }
         if (t < subs) {
@@ -90,7 +90,7 @@ __device__ __forceinline__ unsigned long long cta_take(unsigned long long* s_wor
             atomicExch(s_work, (c << 24) | 1ull);
             if (c >= a.total_chunks) return kNoWork;
             const uint64_t k2 = c / a.chunks_per_seed;
-            const uint64_t jb2 = (c - k2 * a.chunks_per_seed) * (uint64_t)kCtaChunk;
+            const uint64_t jb2 = (c - k2 * a.chunks_per_seed) * (uint64_t)a.cta_chunk;
             const uint32_t seed = a.order ? a.order[k2] : (uint32_t)k2;
             return ((unsigned long long)seed << 32) | jb2;
         }
@@ -98,7 +98,8 @@ __device__ __forceinline__ unsigned long long cta_take(unsigned long long* s_wor
     }
 }
 
-template <int F, bool HALF, bool REFILL>
+// OUT: per-particle outputs or polylines are recorded (compiled out of the bench path).
+template <int F, bool HALF, bool REFILL, bool OUT>
 __global__ void __launch_bounds__(REFILL ? kThreads : kSimpleThreads, PT_MIN_BLOCKS)
 track_kernel(const __grid_constant__ TrackArgs a) {
     using R = Rec<F, HALF>;
@@ -114,6 +115,7 @@ track_kernel(const __grid_constant__ TrackArgs a) {
     extern __shared__ unsigned long long s_cache[];  // kMapCache entries when REFILL && map
     constexpr bool kCache = REFILL && kMapCache > 0;
     const bool use_cache = kCache && a.map != nullptr;
+    const bool has_map = a.map != nullptr;
     if (threadIdx.x == 0) s_work = kNoChunk << 24;
     if constexpr (kCache) {
         if (use_cache)
@@ -158,7 +160,7 @@ track_kernel(const __grid_constant__ TrackArgs a) {
     };
     // SetEndPoint()
     auto finish = [&]() {
-        if (a.o_nsteps || a.o_reason || a.o_end) {
+        if (OUT && (a.o_nsteps || a.o_reason || a.o_end)) {
             const uint64_t li = s_li[threadIdx.x];
             if (a.o_nsteps) a.o_nsteps[li] = (uint16_t)n;
             if (a.o_reason) a.o_reason[li] = (uint8_t)why;
@@ -169,7 +171,7 @@ track_kernel(const __grid_constant__ TrackArgs a) {
                 e[2] = __fadd_rn(qz, a.fcz);
             }
         }
-        if (a.map && run_cnt) red(run_vox, run_cnt);
+        if (has_map && run_cnt) red(run_vox, run_cnt);
         run_cnt = 0;
         my_steps += (uint32_t)n;
         my_particles += 1u;
@@ -182,13 +184,13 @@ track_kernel(const __grid_constant__ TrackArgs a) {
         qy = y;
         qz = z;
         n += 1;
-        if (a.map) {
+        if (has_map) {
             const bool change = v != run_vox;
             if (change && run_cnt != 0u) red(run_vox, run_cnt);
             run_cnt = change ? 1u : run_cnt + 1u;
             run_vox = v;
         }
-        if (a.o_paths && n < a.path_stride) {
+        if (OUT && a.o_paths && n < a.path_stride) {
             float* pp = a.o_paths + (s_li[threadIdx.x] * (uint64_t)a.path_stride + (uint64_t)n) * 3u;
             pp[0] = __fadd_rn(qx, a.fcx);
             pp[1] = __fadd_rn(qy, a.fcy);
@@ -198,7 +200,7 @@ track_kernel(const __grid_constant__ TrackArgs a) {
     // GetStartPoint(): centred seed position, seed voxel (R10, R12)
     auto start = [&](uint64_t si, uint64_t j) {
         const uint64_t li = si * a.P + j;
-        s_li[threadIdx.x] = li;
+        if (OUT) s_li[threadIdx.x] = li;
         const uint64_t sid = a.seed_ids ? a.seed_ids[si] : si;
         pid = sid * a.P + j;
         qx = __fsub_rn(a.seeds[3 * si + 0], a.fcx);
@@ -208,7 +210,7 @@ track_kernel(const __grid_constant__ TrackArgs a) {
         pend = false;
         run_cnt = 0;
         alive = true;
-        if (a.o_paths) {
+        if (OUT && a.o_paths) {
             float* pp = a.o_paths + li * (uint64_t)a.path_stride * 3u;
             pp[0] = __fadd_rn(qx, a.fcx);
             pp[1] = __fadd_rn(qy, a.fcy);
@@ -526,17 +528,19 @@ __global__ void __launch_bounds__(256) gather_bench_kernel(const uint8_t* __rest
 }
 
 // ------------------------------------------------------------------------- launchers
-template <int F, bool HALF, bool REFILL>
+template <int F, bool HALF, bool REFILL, bool OUT>
 static cudaError_t launch_t(const TrackArgs& a, int num_sms, cudaStream_t st) {
-    auto k = track_kernel<F, HALF, REFILL>;
+    auto k = track_kernel<F, HALF, REFILL, OUT>;
     constexpr int TPB = REFILL ? kThreads : kSimpleThreads;
     if (a.nparticles == 0) return cudaSuccess;
-    unsigned grid;
     const size_t dyn = (REFILL && kMapCache > 0 && a.map) ? kMapCache * sizeof(unsigned long long) : 0;
+    unsigned grid;
     if (REFILL) {
         int per_sm = 0;
         cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              (int)(kMapCache * sizeof(unsigned long long)));
+        if (e == cudaSuccess)  // prefer L1 over shared memory: records are gathered through L1
+            e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, kMapCache ? -1 : 0);
         if (e != cudaSuccess) return e;
         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, TPB, dyn);
         if (e != cudaSuccess) return e;
@@ -553,7 +557,9 @@ static cudaError_t launch_t(const TrackArgs& a, int num_sms, cudaStream_t st) {
 
 template <int F, bool HALF>
 static cudaError_t launch_f(const TrackArgs& a, bool simple, int num_sms, cudaStream_t st) {
-    return simple ? launch_t<F, HALF, false>(a, num_sms, st) : launch_t<F, HALF, true>(a, num_sms, st);
+    const bool out = a.o_nsteps || a.o_reason || a.o_end || a.o_paths;
+    if (simple) return out ? launch_t<F, HALF, false, true>(a, num_sms, st) : launch_t<F, HALF, false, false>(a, num_sms, st);
+    return out ? launch_t<F, HALF, true, true>(a, num_sms, st) : launch_t<F, HALF, true, false>(a, num_sms, st);
 }
 
 cudaError_t launch_track(const TrackArgs& a, int nfibres, bool half, bool simple, int num_sms,
@@ -566,32 +572,6 @@ cudaError_t launch_track(const TrackArgs& a, int nfibres, bool half, bool simple
         case 6: return launch_f<3, false>(a, simple, num_sms, st);
         case 7: return launch_f<3, true>(a, simple, num_sms, st);
         default: return cudaErrorInvalidValue;
-    }
-}
-
-template <int F, bool HALF, bool REFILL>
-static int bps() {
-    int per_sm = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, track_kernel<F, HALF, REFILL>,
-                                                  REFILL ? kThreads : kSimpleThreads, 0);
-    return per_sm;
-}
-
-int track_blocks_per_sm(int nfibres, bool half, bool simple) {
-    switch (nfibres * 4 + (half ? 2 : 0) + (simple ? 1 : 0)) {
-        case 4: return bps<1, false, true>();
-        case 5: return bps<1, false, false>();
-        case 6: return bps<1, true, true>();
-        case 7: return bps<1, true, false>();
-        case 8: return bps<2, false, true>();
-        case 9: return bps<2, false, false>();
-        case 10: return bps<2, true, true>();
-        case 11: return bps<2, true, false>();
-        case 12: return bps<3, false, true>();
-        case 13: return bps<3, false, false>();
-        case 14: return bps<3, true, true>();
-        case 15: return bps<3, true, false>();
-        default: return 0;
     }
 }
 
