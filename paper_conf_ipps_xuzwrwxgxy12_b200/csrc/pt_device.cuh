@@ -96,6 +96,52 @@ __device__ __forceinline__ void ldg_record<64>(const void* p, uint32_t* w) {
     ldg_record<32>(static_cast<const char*>(p) + 32, w + 8);
 }
 
+// Predicated variants for straight-line step code: the load / reduction is issued only by
+// lanes with p != 0; the destination registers of the other lanes keep their values.
+template <int BYTES>
+__device__ __forceinline__ void ldg_record_if(bool p, const void* ptr, uint32_t* w);
+
+template <>
+__device__ __forceinline__ void ldg_record_if<8>(bool p, const void* ptr, uint32_t* w) {
+    asm("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %3, 0;\n\t@q ld.global.nc.v2.b32 {%0,%1}, [%2];\n\t}"
+        : "+r"(w[0]), "+r"(w[1])
+        : "l"(ptr), "r"((int)p));
+}
+template <>
+__device__ __forceinline__ void ldg_record_if<16>(bool p, const void* ptr, uint32_t* w) {
+    asm("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %5, 0;\n\t@q ld.global.nc.v4.b32 {%0,%1,%2,%3}, [%4];\n\t}"
+        : "+r"(w[0]), "+r"(w[1]), "+r"(w[2]), "+r"(w[3])
+        : "l"(ptr), "r"((int)p));
+}
+template <>
+__device__ __forceinline__ void ldg_record_if<32>(bool p, const void* ptr, uint32_t* w) {
+    asm("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %9, 0;\n\t@q ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];\n\t}"
+        : "+r"(w[0]), "+r"(w[1]), "+r"(w[2]), "+r"(w[3]), "+r"(w[4]), "+r"(w[5]), "+r"(w[6]), "+r"(w[7])
+        : "l"(ptr), "r"((int)p));
+}
+template <>
+__device__ __forceinline__ void ldg_record_if<64>(bool p, const void* ptr, uint32_t* w) {
+    ldg_record_if<32>(p, ptr, w);
+    ldg_record_if<32>(p, static_cast<const char*>(ptr) + 32, w + 8);
+}
+
+// The same with an L2 cache-eviction policy (createpolicy ... L2::evict_last): keeps the
+// visitation map resident in L2 while the record stream churns through it.
+__device__ __forceinline__ uint64_t l2_evict_last_policy() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ void red_add_if_hint(bool p, uint32_t* addr, uint32_t v, uint64_t pol) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %3, 0;\n\t@q red.global.add.L2::cache_hint.u32 [%0], %1, %2;\n\t}"
+                 :: "l"(addr), "r"(v), "l"(pol), "r"((int)p) : "memory");
+}
+
+__device__ __forceinline__ void red_add_if(bool p, uint32_t* addr, uint32_t v) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q red.global.add.u32 [%0], %1;\n\t}"
+                 :: "l"(addr), "r"(v), "r"((int)p) : "memory");
+}
+
 // ---------------------------------------------------------------------------- lookup (R10)
 // Centred coordinates q = x - c, c = floor(N/2); index = c + trunc(q) - signbit(q):
 // voxel i covers [i-c, i-c+1) for i >= c and (i-c, i-c+1] for i < c.

@@ -27,6 +27,12 @@
 #ifndef PT_MIN_BLOCKS
 #define PT_MIN_BLOCKS 1
 #endif
+#ifndef PT_MAP_HINT
+#define PT_MAP_HINT 0  // 1: REDs carry an L2 evict_last policy (measured: no effect)
+#endif
+#ifndef PT_MAP_PERSIST
+#define PT_MAP_PERSIST 0  // 1: persisting L2 access-policy window over the map (measured: no effect)
+#endif
 #ifndef PT_MAP_CACHE
 #define PT_MAP_CACHE 0      // entries of the per-CTA shared-memory count cache (power of 2; 0 = off)
 #endif
@@ -109,6 +115,9 @@ track_kernel(const __grid_constant__ TrackArgs a) {
     __shared__ unsigned long long s_li[TPB];     // particle index of this call (outputs)
     __shared__ uint32_t s_q[TPB / 32][3];        // per-warp sub-chunk: seed, next j, end j
     __shared__ unsigned long long s_work;        // CTA chunk + tickets (see cta_take)
+#if defined(PT_DIAG_RED) && PT_DIAG_RED == 1
+    __shared__ uint32_t s_diag[1024];
+#endif
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t wib = threadIdx.x >> 5;
     const uint32_t lt_mask = (1u << lane) - 1u;
@@ -116,6 +125,7 @@ track_kernel(const __grid_constant__ TrackArgs a) {
     constexpr bool kCache = REFILL && kMapCache > 0;
     const bool use_cache = kCache && a.map != nullptr;
     const bool has_map = a.map != nullptr;
+    const uint64_t map_pol = PT_MAP_HINT ? l2_evict_last_policy() : 0ull;
     if (threadIdx.x == 0) s_work = kNoChunk << 24;
     if constexpr (kCache) {
         if (use_cache)
@@ -177,20 +187,32 @@ track_kernel(const __grid_constant__ TrackArgs a) {
         my_particles += 1u;
         why = -1;
     };
-    // commit a step: new position, one visit of the new voxel (R13); consecutive
-    // visits of the same voxel are merged (run length) and flushed when the voxel changes
-    auto commit = [&](float x, float y, float z, uint32_t v) {
-        qx = x;
-        qy = y;
-        qz = z;
-        n += 1;
+    // commit a step (lanes with c): new position, one visit of the new voxel (R13);
+    // consecutive visits of the same voxel are merged (run length) and flushed with a
+    // predicated RED when the voxel changes.  Straight-line, no branch.
+    auto commit_if = [&](bool c, float x, float y, float z, uint32_t v) {
+        qx = c ? x : qx;
+        qy = c ? y : qy;
+        qz = c ? z : qz;
+        n += c ? 1 : 0;
         if (has_map) {
             const bool change = v != run_vox;
-            if (change && run_cnt != 0u) red(run_vox, run_cnt);
-            run_cnt = change ? 1u : run_cnt + 1u;
-            run_vox = v;
+            if (kCache && use_cache) {
+                if (c && change && run_cnt != 0u) red(run_vox, run_cnt);
+            } else {
+#if defined(PT_DIAG_RED) && PT_DIAG_RED == 1  // diagnostic builds only (wrong maps)
+                if (c && change && run_cnt != 0u) atomicAdd(&s_diag[run_vox & 1023u], run_cnt);
+#elif defined(PT_DIAG_RED) && PT_DIAG_RED == 2
+                red_add_if(c && change && run_cnt != 0u, a.map + ((run_vox & 4095u) + blockIdx.x * 4096u), run_cnt);
+#else
+                if (PT_MAP_HINT) red_add_if_hint(c && change && run_cnt != 0u, a.map + run_vox, run_cnt, map_pol);
+                else red_add_if(c && change && run_cnt != 0u, a.map + run_vox, run_cnt);
+#endif
+            }
+            run_cnt = c ? (change ? 1u : run_cnt + 1u) : run_cnt;
+            run_vox = c ? v : run_vox;
         }
-        if (OUT && a.o_paths && n < a.path_stride) {
+        if (OUT && a.o_paths && c && n < a.path_stride) {
             float* pp = a.o_paths + (s_li[threadIdx.x] * (uint64_t)a.path_stride + (uint64_t)n) * 3u;
             pp[0] = __fadd_rn(qx, a.fcx);
             pp[1] = __fadd_rn(qy, a.fcy);
@@ -277,93 +299,78 @@ track_kernel(const __grid_constant__ TrackArgs a) {
         rounds += 1u;
 
         // ------------------------------------------------ round start: one Philox block,
-        // gather of (pending candidate | seed) voxel = mask test + first step's record
-        if (alive) {
+        // gather of (pending candidate | seed) voxel = mask test + first step's record.
+        // Straight-line code: every lane computes, only live lanes load / commit.
+        {
             const uint32_t t0 = (uint32_t)n + (pend ? 1u : 0u);  // a multiple of 3
             W = philox4x32_10(make_uint4(t0 / 3u, (uint32_t)pid, (uint32_t)(pid >> 32), 0u),
                               a.key0, a.key1);
-            ldg_record<RB>(a.rec + ((uint64_t)gvox * a.S + sample_of(W.x, a.S)) * RB, rv.w);
-            if (rv.outside()) {
-                end(kEndMask);  // seed outside the mask (R12) or candidate rejected (R11)
-            } else if (pend) {
-                // the candidate is recomputed bit-identically from (q, d) instead of kept
-                commit(__fadd_rn(qx, __fmul_rn(a.step, px)), __fadd_rn(qy, __fmul_rn(a.step, py)),
-                       __fadd_rn(qz, __fmul_rn(a.step, pz)), gvox);
-                pend = false;
-            }
+            ldg_record_if<RB>(alive, a.rec + ((uint64_t)gvox * a.S + sample_of(W.x, a.S)) * RB, rv.w);
+            // seed outside the mask (R12) or pending candidate rejected (R11)
+            const bool outside = alive && rv.outside();
+            why = outside ? kEndMask : why;
+            alive = alive && !outside;
+            // accepted candidate: recomputed bit-identically from (q, d) instead of kept
+            commit_if(pend && !outside, __fadd_rn(qx, __fmul_rn(a.step, px)),
+                      __fadd_rn(qy, __fmul_rn(a.step, py)), __fadd_rn(qz, __fmul_rn(a.step, pz)), gvox);
+            pend = false;
         }
 
         // ------------------------------------------------ three steps
 #pragma unroll
         for (int k = 0; k < 3; ++k) {
             my_active += alive ? 1u : 0u;
-            if (alive) {
-                if (n == a.max_steps) {
-                    end(kEndMaxlen);  // maximum number of steps (R14)
-                } else {
-                    float vx, vy, vz, fj;
-                    float sg;
-                    bool go = true;
-                    if (n == 0) {
-                        // first step (always k == 0 of a lane's first round, W = block 0):
-                        // fibre 0, sign = top bit of word 3 (R5, R6, R16)
-                        rv.fibre(0, vx, vy, vz, fj);
-                        sg = (W.w >> 31) ? -1.f : 1.f;
-                    } else {
-                        // choose the fibre closest to the previous direction:
-                        // eligible iff f_j > fib_thr (R7), strict >, lowest j wins (R8)
-                        float best = -1.f;
-                        rv.fibre(0, vx, vy, vz, fj);
-                        float bc = __fadd_rn(__fadd_rn(__fmul_rn(vx, px), __fmul_rn(vy, py)),
-                                             __fmul_rn(vz, pz));
-                        if (fj > a.fib_thr) best = fabsf(bc);
+            const bool first = n == 0;
+            // choose the fibre closest to the previous direction: eligible iff
+            // f_j > fib_thr (R7), strict >, lowest j wins (R8); the first step takes fibre 0
+            // (R5).  "Interpolation()" of Alg. 1 = this sample's record at the voxel (R2).
+            float vx, vy, vz, f0;
+            rv.fibre(0, vx, vy, vz, f0);
+            float bc = __fadd_rn(__fadd_rn(__fmul_rn(vx, px), __fmul_rn(vy, py)), __fmul_rn(vz, pz));
+            float best = f0 > a.fib_thr ? fabsf(bc) : -1.f;
 #pragma unroll
-                        for (int j = 1; j < F; ++j) {
-                            float ux, uy, uz, fu;
-                            rv.fibre(j, ux, uy, uz, fu);
-                            const float cj = __fadd_rn(__fadd_rn(__fmul_rn(ux, px), __fmul_rn(uy, py)),
-                                                       __fmul_rn(uz, pz));
-                            if (fu > a.fib_thr && fabsf(cj) > best) {
-                                best = fabsf(cj);
-                                bc = cj;
-                                vx = ux;
-                                vy = uy;
-                                vz = uz;
-                            }
-                        }
-                        // maximum angle, measured by the dot product (R4)
-                        go = fabsf(bc) > a.curv_thr;
-                        if (!go) end(kEndCurv);
-                        sg = bc > 0.f ? 1.f : -1.f;  // keep the orientation (R9)
-                    }
-                    if (go) {
-                        // StepToNextPoint(): q' = q + h * (sign * v), no FMA
-                        px = sg < 0.f ? -vx : vx;
-                        py = sg < 0.f ? -vy : vy;
-                        pz = sg < 0.f ? -vz : vz;
-                        const float nqx = __fadd_rn(qx, __fmul_rn(a.step, px));
-                        const float nqy = __fadd_rn(qy, __fmul_rn(a.step, py));
-                        const float nqz = __fadd_rn(qz, __fmul_rn(a.step, pz));
-                        const int ix = axis_index(nqx, a.cx), iy = axis_index(nqy, a.cy),
-                                  iz = axis_index(nqz, a.cz);
-                        if (!((unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny &&
-                              (unsigned)iz < (unsigned)a.nz)) {
-                            end(kEndMask);  // left the volume (R11)
-                        } else {
-                            const uint32_t v =
-                                ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
-                            if (k < 2) {
-                                const uint32_t w = (k == 0) ? W.y : W.z;
-                                ldg_record<RB>(a.rec + ((uint64_t)v * a.S + sample_of(w, a.S)) * RB, rv.w);
-                                if (rv.outside()) end(kEndMask);  // candidate outside the mask (R11)
-                                else commit(nqx, nqy, nqz, v);
-                            } else {
-                                pend = true;  // next round's start gathers and tests it
-                                gvox = v;
-                            }
-                        }
-                    }
-                }
+            for (int j = 1; j < F; ++j) {
+                float ux, uy, uz, fu;
+                rv.fibre(j, ux, uy, uz, fu);
+                const float cj = __fadd_rn(__fadd_rn(__fmul_rn(ux, px), __fmul_rn(uy, py)), __fmul_rn(uz, pz));
+                const bool pick = !first && fu > a.fib_thr && fabsf(cj) > best;
+                best = pick ? fabsf(cj) : best;
+                bc = pick ? cj : bc;
+                vx = pick ? ux : vx;
+                vy = pick ? uy : vy;
+                vz = pick ? uz : vz;
+            }
+            // maximum angle, measured by the dot product (R4); orientation
+            // kept (R9); first step: sign = top bit of word 3 of block 0 (R6, R16)
+            const bool curv_ok = first || fabsf(bc) > a.curv_thr;
+            const bool neg = first ? (W.w >> 31) != 0u : !(bc > 0.f);
+            // StepToNextPoint(): q' = q + h * (sign * v), no FMA
+            const float dx = neg ? -vx : vx, dy = neg ? -vy : vy, dz = neg ? -vz : vz;
+            const float nqx = __fadd_rn(qx, __fmul_rn(a.step, dx));
+            const float nqy = __fadd_rn(qy, __fmul_rn(a.step, dy));
+            const float nqz = __fadd_rn(qz, __fmul_rn(a.step, dz));
+            const int ix = axis_index(nqx, a.cx), iy = axis_index(nqy, a.cy), iz = axis_index(nqz, a.cz);
+            const bool inb = (unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny &&
+                             (unsigned)iz < (unsigned)a.nz;
+            const uint32_t v = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
+            // stop criteria in order: maximum steps (R14), angle, volume (R11)
+            const bool maxed = n == a.max_steps;
+            const bool go = alive && !maxed && curv_ok && inb;
+            why = (alive && !go) ? (maxed ? kEndMaxlen : (!curv_ok ? kEndCurv : kEndMask)) : why;
+            alive = go;
+            px = go ? dx : px;
+            py = go ? dy : py;
+            pz = go ? dz : pz;
+            if (k < 2) {
+                const uint32_t w = (k == 0) ? W.y : W.z;
+                ldg_record_if<RB>(go, a.rec + ((uint64_t)v * a.S + sample_of(w, a.S)) * RB, rv.w);
+                const bool outside = go && rv.outside();  // candidate outside the mask (R11)
+                why = outside ? kEndMask : why;
+                alive = go && !outside;
+                commit_if(alive, nqx, nqy, nqz, v);
+            } else {
+                pend = go;  // next round's start gathers and tests it
+                gvox = go ? v : gvox;
             }
         }
     }
@@ -550,6 +557,28 @@ static cudaError_t launch_t(const TrackArgs& a, int num_sms, cudaStream_t st) {
         grid = (unsigned)(need < full ? need : full);
     } else {
         grid = (unsigned)((a.nparticles + TPB - 1) / TPB);
+    }
+    if (PT_MAP_PERSIST && REFILL && a.map) {
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(grid);
+        cfg.blockDim = dim3(TPB);
+        cfg.dynamicSmemBytes = dyn;
+        cfg.stream = st;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeAccessPolicyWindow;
+        at[0].val.accessPolicyWindow.base_ptr = a.map;
+        at[0].val.accessPolicyWindow.num_bytes = (size_t)a.nx * a.ny * a.nz * sizeof(uint32_t);
+        at[0].val.accessPolicyWindow.hitRatio = 1.0f;
+        at[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        at[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        size_t lim = 0;
+        cudaDeviceGetLimit(&lim, cudaLimitPersistingL2CacheSize);
+        if (lim < at[0].val.accessPolicyWindow.num_bytes)
+            cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, at[0].val.accessPolicyWindow.num_bytes);
+        cudaGetLastError();
+        return cudaLaunchKernelEx(&cfg, k, a);
     }
     k<<<grid, TPB, dyn, st>>>(a);
     return cudaGetLastError();
