@@ -15,6 +15,13 @@
 
 #include "pt_internal.h"
 
+#ifndef PT_SEEDS_PER_CLAIM
+// Whole seeds per CTA claim when every seed fits one claim: a CTA walks 32 consecutive
+// (Morton-adjacent) seeds, so its L1 keeps serving the shared tract voxels (sweep 1..64:
+// c3 74.6/75.3/76.0/76.4/77.0/77.2/76.9 G steps/s; 32 is the default).
+#define PT_SEEDS_PER_CLAIM 32
+#endif
+
 struct pt_ctx {
     int device = 0;
     int num_sms = 0;
@@ -411,6 +418,15 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     }
     a.chunks_per_seed = (uint32_t)((P + a.cta_chunk - 1) / a.cta_chunk);
     a.total_chunks = N * (uint64_t)a.chunks_per_seed;
+    a.seeds_per_claim = 1;
+    if (a.chunks_per_seed == 1 && PT_SEEDS_PER_CLAIM > 1) {
+        // whole seeds per claim: G consecutive seeds (tickets per claim must stay < 2^22)
+        uint64_t G = PT_SEEDS_PER_CLAIM;
+        const uint64_t sps = (P + pt::kSub - 1) / pt::kSub;
+        while (G > 1 && (G * sps >= (1ull << 22) || N / G < 8ull * (uint64_t)c->num_sms)) G >>= 1;
+        a.seeds_per_claim = (uint32_t)G;
+        a.total_chunks = (N + G - 1) / G;
+    }
     a.map = d_map;
     a.o_nsteps = (fl & PT_REC_LEN) ? c->d_nsteps : nullptr;
     a.o_reason = (fl & PT_REC_REASON) ? c->d_reason : nullptr;

@@ -47,7 +47,8 @@ struct TrackArgs {
     const uint32_t* order;       // [nseeds] processing order (Morton) or nullptr
     uint64_t nseeds;
     uint64_t nparticles;         // nseeds * P
-    uint32_t cta_chunk;          // particles per CTA claim (multiple of kSub)
+    uint32_t cta_chunk;          // particles per CTA claim within a seed (multiple of kSub)
+    uint32_t seeds_per_claim;    // > 1: a claim is this many whole consecutive seeds
     uint32_t chunks_per_seed;    // ceil(P / cta_chunk)
     uint64_t total_chunks;       // nseeds * chunks_per_seed
     uint32_t* map;               // [V] or nullptr
