@@ -47,7 +47,8 @@ class _Volume(ctypes.Structure):
 class _Params(ctypes.Structure):
     _fields_ = [("step", ctypes.c_float), ("curv_thr", ctypes.c_float),
                 ("fib_thr", ctypes.c_float), ("max_steps", ctypes.c_int32),
-                ("rng_seed", ctypes.c_uint64), ("particles_per_seed", ctypes.c_int64)]
+                ("rng_seed", ctypes.c_uint64), ("particles_per_seed", ctypes.c_int64),
+                ("sample_mode", ctypes.c_int32)]
 
 
 _lib = None
@@ -107,11 +108,11 @@ def sample_index(w: int, nsamples: int) -> int:
 
 # ----------------------------------------------------------------------------- tracking
 
-def _structs(volume, step, curv_thr, fib_thr, max_steps, rng_seed, P):
+def _structs(volume, step, curv_thr, fib_thr, max_steps, rng_seed, P, sample_mode=0):
     v = volume
     vs = _Volume(v.nx, v.ny, v.nz, v.nsamples, v.nfibres, 1 if v.dyads.dtype == np.float16 else 0,
                  v.dyads.ctypes.data, v.f.ctypes.data, v.mask.ctypes.data)
-    ps = _Params(step, curv_thr, fib_thr, max_steps, rng_seed, P)
+    ps = _Params(step, curv_thr, fib_thr, max_steps, rng_seed, P, sample_mode)
     return vs, ps
 
 
@@ -132,7 +133,8 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
     ids = np.ascontiguousarray(w.ids(), np.uint64)
     ns = seeds.shape[0]
     n = ns * npp
-    vs, ps = _structs(v, w.step, w.curv_thr, w.fib_thr, w.max_steps, w.rng_seed, P)
+    vs, ps = _structs(v, w.step, w.curv_thr, w.fib_thr, w.max_steps, w.rng_seed, P,
+                      int(getattr(w, "sample_mode", 0)))
     nsteps = np.zeros(n, np.int32) if want_particles else None
     reason = np.zeros(n, np.uint8) if want_particles else None
     end = np.zeros((n, 3), np.float32) if want_particles else None

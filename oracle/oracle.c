@@ -126,6 +126,7 @@ static int valid_params(const oracle_volume* v, const oracle_params* p) {
     if (isnan(p->fib_thr)) return 0;
     if (p->max_steps < 1 || p->max_steps > 65535) return 0;
     if (p->particles_per_seed < 1) return 0;
+    if (p->sample_mode != 0 && p->sample_mode != 1) return 0;
     return 1;
 }
 
@@ -186,7 +187,11 @@ int oracle_track(const oracle_volume* vol, const oracle_params* prm,
                      * the particle's stream: ctr = {b, pid_lo, pid_hi, 0}; word n%3. */
                     blk_ctr[0] = (uint32_t)(n / 3); blk_ctr[1] = plo; blk_ctr[2] = phi; blk_ctr[3] = 0u;
                     oracle_philox4x32_10(blk_ctr, key, w);
-                    s = oracle_sample_index(w[n % 3], S);
+                    if (prm->sample_mode == 1)
+                        s = (uint32_t)((uint64_t)jj % S);   /* NEXT-1: one sample volume per
+                                                               streamline */
+                    else
+                        s = oracle_sample_index(w[n % 3], S);
 
                     /* Interpolation() (R2): the sample's fibres at this voxel */
                     for (j = 0; j < F; ++j) fetch(vol, vox, s, j, v[j], &fv[j]);

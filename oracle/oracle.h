@@ -40,6 +40,10 @@ typedef struct {
     int32_t max_steps;
     uint64_t rng_seed;
     int64_t particles_per_seed;
+    /* 0: a fresh random sample every step (R1, FSL style, the north star's mode);
+     * 1: paper mode (NEXT-1): particle j of a seed follows sample volume j mod S for its
+     *    whole path (Alg. 1: one sample volume per streamline). */
+    int32_t sample_mode;
 } oracle_params;
 
 enum { ORACLE_END_MASK = 0, ORACLE_END_CURV = 1, ORACLE_END_MAXLEN = 2 };

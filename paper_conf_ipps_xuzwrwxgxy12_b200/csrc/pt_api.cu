@@ -15,6 +15,9 @@
 
 #include "pt_internal.h"
 
+#ifndef PT_MAP_COPIES
+#define PT_MAP_COPIES 1  // private map copies (privatisation; 1 = add into the map directly)
+#endif
 #ifndef PT_SEEDS_PER_CLAIM
 // Whole seeds per CTA claim when every seed fits one claim: a CTA walks 32 consecutive
 // (Morton-adjacent) seeds, so its L1 keeps serving the shared tract voxels (sweep 1..64:
@@ -44,6 +47,8 @@ struct pt_ctx {
     size_t temp_cap = 0;
     uint32_t* d_map = nullptr;   // internal map for host map pointers
     size_t map_cap = 0;
+    uint32_t* d_copies = nullptr;  // private map copies (PT_MAP_COPIES > 1)
+    size_t copies_cap = 0;
     uint16_t* d_nsteps = nullptr;
     size_t nsteps_cap = 0;
     uint8_t* d_reason = nullptr;
@@ -190,7 +195,7 @@ void pt_destroy(pt_ctx* c) {
     DeviceGuard g(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
     else cudaDeviceSynchronize();
-    void* bufs[] = {c->d_rec, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_nsteps,
+    void* bufs[] = {c->d_rec, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_copies, c->d_nsteps,
                     c->d_reason, c->d_end, c->d_paths, c->d_stats};
     for (void* b : bufs)
         if (b) cudaFree(b);
@@ -428,6 +433,16 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         a.total_chunks = (N + G - 1) / G;
     }
     a.map = d_map;
+    a.map_copies = 1;
+    const bool simple = (fl & PT_KERNEL_SIMPLE) != 0;
+    uint32_t copies = (d_map && !simple && npart > 0) ? (uint32_t)PT_MAP_COPIES : 1u;
+    if (copies > (uint32_t)c->num_sms) copies = (uint32_t)c->num_sms;
+    if (copies > 1) {
+        CK(ensure(c->d_copies, c->copies_cap, (size_t)copies * V), "pt_track: map copies");
+        CK(cudaMemsetAsync(c->d_copies, 0, (size_t)copies * V * sizeof(uint32_t), st), "pt_track: map copies zero");
+        a.map = c->d_copies;
+        a.map_copies = copies;
+    }
     a.o_nsteps = (fl & PT_REC_LEN) ? c->d_nsteps : nullptr;
     a.o_reason = (fl & PT_REC_REASON) ? c->d_reason : nullptr;
     a.o_end = (fl & PT_REC_END) ? c->d_end : nullptr;
@@ -439,6 +454,8 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     CK(pt::launch_track(a, c->vol.nfibres, c->vol.dtype == PT_F16, (fl & PT_KERNEL_SIMPLE) != 0, c->num_sms, st),
        "pt_track: tracking kernel launch");
     CK(cudaEventRecord(c->ev[2], st), "pt_track: event");
+    if (a.map_copies > 1)
+        CK(pt::launch_map_combine(a.map, a.map_copies, (int64_t)V, d_map, true, st), "pt_track: map combine");
     if (d_map) CK(pt::launch_map_sum(d_map, (int64_t)V, c->d_stats + pt::kStatMapAfter, st), "pt_track: map sum");
     if (host_map) {
         CK(cudaMemcpyAsync(map, d_map, V * sizeof(uint32_t), cudaMemcpyDeviceToHost, st), "pt_track: map D2H");

@@ -51,7 +51,9 @@ struct TrackArgs {
     uint32_t seeds_per_claim;    // > 1: a claim is this many whole consecutive seeds
     uint32_t chunks_per_seed;    // ceil(P / cta_chunk)
     uint64_t total_chunks;       // nseeds * chunks_per_seed
-    uint32_t* map;               // [V] or nullptr
+    uint32_t* map;               // [V] or nullptr: the map this launch adds into
+    uint32_t map_copies;         // > 1: map points at map_copies private [V] copies;
+                                 //      CTA b adds into copy b % map_copies
     uint16_t* o_nsteps;          // [nparticles] or nullptr
     uint8_t* o_reason;
     float* o_end;                // [nparticles][3]
@@ -72,6 +74,9 @@ cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask,
 size_t seed_order_temp_bytes(uint64_t nseeds);
 cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint32_t* keys, uint32_t* keys_out,
                               uint32_t* idx, uint32_t* perm, void* temp, size_t temp_bytes, cudaStream_t st);
+// out[v] (+)= sum over c of copies[c * V + v]
+cudaError_t launch_map_combine(const uint32_t* copies, uint32_t ncopies, int64_t V, uint32_t* out,
+                               bool accumulate, cudaStream_t st);
 cudaError_t launch_map_sum(const uint32_t* map, int64_t V, unsigned long long* out,
                            cudaStream_t st);
 cudaError_t launch_gather_bench(const uint8_t* buf, uint64_t nrec, int rec_bytes, uint32_t iters,

@@ -147,6 +147,11 @@ track_kernel(const __grid_constant__ TrackArgs a) {
     constexpr bool kCache = REFILL && kMapCache > 0;
     const bool use_cache = kCache && a.map != nullptr;
     const bool has_map = a.map != nullptr;
+    // privatised map: CTA b adds into copy b % map_copies (no cross-SM contention on the
+    // hot lines near the seeds; the copies are summed by map_combine_kernel)
+    uint32_t* const map = has_map ? a.map + (size_t)(blockIdx.x % a.map_copies) *
+                                                  ((size_t)a.nx * a.ny * a.nz)
+                                  : nullptr;
     const uint64_t map_pol = PT_MAP_HINT ? l2_evict_last_policy() : 0ull;
     if (threadIdx.x == 0) s_work = kNoChunk << 24;
     if constexpr (kCache) {
@@ -180,8 +185,8 @@ track_kernel(const __grid_constant__ TrackArgs a) {
     int why = -1;  // >= 0: the particle ended with this reason; outputs pending (finish())
 
     auto red = [&](uint32_t v, uint32_t c) {
-        if (kCache && use_cache) cache_add(s_cache, a.map, v, c);
-        else atomicAdd(a.map + v, c);  // no return value used -> RED
+        if (kCache && use_cache) cache_add(s_cache, map, v, c);
+        else atomicAdd(map + v, c);  // no return value used -> RED
     };
     // a termination only records the reason; the outputs are written once per round for
     // all ended lanes at the top of the loop (one divergent block instead of one per site)
@@ -227,8 +232,8 @@ track_kernel(const __grid_constant__ TrackArgs a) {
 #elif defined(PT_DIAG_RED) && PT_DIAG_RED == 2
                 red_add_if(c && change && run_cnt != 0u, a.map + ((run_vox & 4095u) + blockIdx.x * 4096u), run_cnt);
 #else
-                if (PT_MAP_HINT) red_add_if_hint(c && change && run_cnt != 0u, a.map + run_vox, run_cnt, map_pol);
-                else red_add_if(c && change && run_cnt != 0u, a.map + run_vox, run_cnt);
+                if (PT_MAP_HINT) red_add_if_hint(c && change && run_cnt != 0u, map + run_vox, run_cnt, map_pol);
+                else red_add_if(c && change && run_cnt != 0u, map + run_vox, run_cnt);
 #endif
             }
             run_cnt = c ? (change ? 1u : run_cnt + 1u) : run_cnt;
@@ -403,7 +408,7 @@ track_kernel(const __grid_constant__ TrackArgs a) {
             __syncthreads();
             for (uint32_t i = threadIdx.x; i < kMapCache; i += TPB) {
                 const unsigned long long e = s_cache[i];
-                if (e >> 32) atomicAdd(a.map + ((uint32_t)(e >> 32) - 1u), (uint32_t)e);
+                if (e >> 32) atomicAdd(map + ((uint32_t)(e >> 32) - 1u), (uint32_t)e);
             }
         }
     }
@@ -521,6 +526,25 @@ cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint32_t* key
     if (e != cudaSuccess) return e;
     // stable radix sort on the 30-bit Morton code: ties keep the input order
     return cub::DeviceRadixSort::SortPairs(temp, temp_bytes, keys, keys_out, idx, perm, (int)nseeds, 0, 30, st);
+}
+
+// ------------------------------------------------------------------------- map combine
+__global__ void map_combine_kernel(const uint32_t* __restrict__ copies, uint32_t ncopies, int64_t V,
+                                   uint32_t* __restrict__ out, bool accumulate) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < V; i += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t s = accumulate ? out[i] : 0u;
+        for (uint32_t c = 0; c < ncopies; ++c) s += __ldg(copies + (int64_t)c * V + i);
+        out[i] = s;
+    }
+}
+
+cudaError_t launch_map_combine(const uint32_t* copies, uint32_t ncopies, int64_t V, uint32_t* out,
+                               bool accumulate, cudaStream_t st) {
+    int64_t blocks = (V + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    if (blocks < 1) blocks = 1;
+    map_combine_kernel<<<(unsigned)blocks, 256, 0, st>>>(copies, ncopies, V, out, accumulate);
+    return cudaGetLastError();
 }
 
 // ------------------------------------------------------------------------- map sum

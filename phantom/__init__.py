@@ -80,6 +80,7 @@ class Workload:
     rng_seed: int = 0x5EED_2012
     particles_per_seed: int = 1000
     recipe: str = ""
+    sample_mode: int = 0  # 0: random sample per step (R1); 1: paper mode, s = j mod S (NEXT-1)
 
     @property
     def nseeds(self) -> int:

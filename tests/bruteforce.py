@@ -67,7 +67,7 @@ def track(w, seed_index: int, j: int, max_points: int = 10**9):
         if n == w.max_steps:
             return n, 2, np.array(pos, np.float32)
         wd = philox4x32_10([n // 3, pid & _M, pid >> 32, 0], key)
-        s = (wd[n % 3] * S) >> 32
+        s = (j % S) if getattr(w, "sample_mode", 0) == 1 else (wd[n % 3] * S) >> 32
         vv = [[dy[jj, s, vox[0], vox[1], vox[2], a] for a in range(3)] for jj in range(F)]
         ff = [fr[jj, s, vox[0], vox[1], vox[2]] for jj in range(F)]
         if n == 0:

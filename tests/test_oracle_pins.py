@@ -443,3 +443,56 @@ def test_zero_dot_sign_is_negative():
     assert np.all(r["reason"] == oracle.END_MASK)
     assert np.all(r["end"][fwd, 1] < 1.0)
     assert np.all(r["end"][fwd, 0] >= 40)
+
+
+# ----------------------------------------------------------------------------- NEXT-1 paper mode
+
+def _alternating_tube(nx=40, ny=40, nz=8, S=4, P=24, seed_xy=(20, 20)):
+    """Whole-volume mask; sample s points along x for even s, along y for odd s (F = 1)."""
+    dy = np.zeros((1, S, nz, ny, nx, 3), np.float32)
+    for s in range(S):
+        dy[0, s, ..., 0 if s % 2 == 0 else 1] = 1.0
+    f = np.ones((1, S, nz, ny, nx), np.float32)
+    mask = np.ones((nz, ny, nx), np.uint8)
+    vol = phantom.Volume(nx, ny, nz, S, 1, dy, f, mask)
+    seeds = np.array([[seed_xy[0] + 0.5, seed_xy[1] + 0.5, nz // 2 + 0.5]], np.float32)
+    return phantom.Workload("alt_tube", vol, seeds, None, particles_per_seed=P, rng_seed=99,
+                            sample_mode=1)
+
+
+def test_paper_mode_one_sample_per_streamline():
+    """NEXT-1 (Alg. 1: each streamline follows one sample volume):
+    particle j uses sample j mod S for every step, so with samples alternating between
+    +-x and +-y it runs straight along x (j even) or y (j odd) to the volume face."""
+    w = _alternating_tube()
+    r = oracle.track(w)
+    sg = _signs(w)
+    N = 40
+    for j in range(w.particles_per_seed):
+        path = _exact_path(N, 20, int(sg[j]), 200)
+        k = path.index(-1) if sg[j] < 0 else path.index(N)
+        assert r["nsteps"][j] == k and r["reason"][j] == oracle.END_MASK
+        e = r["end"][j]
+        moved, fixed = (0, 1) if j % 2 == 0 else (1, 0)
+        assert e[fixed] == 20.5
+        assert e[moved] == np.float32(20.5 + 0.5 * sg[j] * k)
+    # the per-step random mode (R1) mixes the two directions instead
+    rr = oracle.track(w.replace(sample_mode=0))
+    assert not np.array_equal(rr["nsteps"], r["nsteps"])
+
+
+@pytest.mark.parametrize("half", [False, True])
+def test_paper_mode_bruteforce(half):
+    w = phantom.whole_brain(nx=14, ny=12, nz=10, semi=(6.0, 5.0, 4.0), nsamples=6, nfibres=2,
+                            particles_per_seed=6, seeds="brain")
+    w = phantom.wm_seeds(w, every=max(1, w.nseeds // 12)).replace(curv_thr=0.3, sample_mode=1)
+    if half:
+        w = phantom.to_half(w)
+    r = oracle.track(w, path_stride=300)
+    for i in range(w.nparticles):
+        n, why, pos = bruteforce.track(w, i // w.particles_per_seed, i % w.particles_per_seed)
+        assert (r["nsteps"][i], r["reason"][i]) == (n, why), i
+        k = min(n + 1, 300)
+        assert np.array_equal(r["paths"][i, :k].view(np.uint32), pos[:k].view(np.uint32)), i
+    with pytest.raises(ValueError):
+        oracle.track(w.replace(sample_mode=2))
