@@ -34,7 +34,16 @@ CONFIG_TEXT = {
     "c2": "configs[1]: 64x64x32 two-bundle 90deg crossing, 50 samples x 2 fibres, 1k seeds x 5000",
     "c2_dispersed": "configs[1] shape, dispersed (sigma 0.15, f jitter 0.03)",
     "c1": "configs[0]: 32x32x16 straight tube, 64 seeds x 1000",
+    "d1": "NEXT-1 paper mode: dataset-1-shaped 96x96x48, every brain voxel x 50 (one streamline per "
+          "sample volume), step 0.1, dot threshold 0.9, MaxStep 1888 (Table II row 1 parameters)",
+    "d2": "NEXT-1 paper mode: dataset-2-shaped 102x102x60, every brain voxel x 50, step 0.1, "
+          "dot threshold 0.9, MaxStep 1888 (Table II row 4 parameters)",
 }
+
+# Table II of the paper, for context beside the NEXT-1 paper-mode workloads:
+# (total fibre length = total steps, longest fibre) on the real CABI datasets, HD 5870.
+PAPER_TABLE2 = {"d1": {"total_steps": 113822762, "longest": 453, "kernel_s": 3.02, "gpu_total_s": 6.74},
+                "d2": {"total_steps": 305396623, "longest": 777, "kernel_s": 6.78, "gpu_total_s": 14.84}}
 
 
 def _env_int(k, d):
@@ -228,6 +237,7 @@ def run_ours(args):
     mine = _shard(w, rank, world)
     tr = pt.Tracker(local)
     tr.load_volume(w.volume)
+    base_flags = args.track_flags | (pt.PT_SAMPLE_PER_STREAMLINE if getattr(w, "sample_mode", 0) else 0)
     V = w.volume.nx * w.volume.ny * w.volume.nz
     rb = pt.pt_record_bytes(w.volume.nfibres, pt.PT_F16 if w.volume.is_half else pt.PT_F32)
     seeds_d = torch.as_tensor(mine.seeds, device=dev).contiguous()
@@ -239,7 +249,7 @@ def run_ours(args):
         flush_buf.fill_(1)  # evict L2 between steps
         tr.track(seeds_d, ids_d, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
                  max_steps=w.max_steps, rng_seed=w.rng_seed,
-                 particles_per_seed=w.particles_per_seed, out_map=out_map, flags=args.track_flags,
+                 particles_per_seed=w.particles_per_seed, out_map=out_map, flags=base_flags,
                  want_map=not args.no_map)
         if world > 1 and not args.no_map:
             sharding.reduce_map(out_map, dst=0)  # one NCCL reduce; int32 sum == uint32 sum
@@ -304,7 +314,7 @@ def run_ours(args):
         flush_buf.fill_(1)
         tr.track(seeds_h, ids_h, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
                  max_steps=w.max_steps, rng_seed=w.rng_seed,
-                 particles_per_seed=w.particles_per_seed, out_map=map_h, flags=args.track_flags)
+                 particles_per_seed=w.particles_per_seed, out_map=map_h, flags=base_flags)
         if world > 1:
             # the host map is reduced over the process group as the step's result
             mt = map_h.to(dev, non_blocking=True)
@@ -354,6 +364,37 @@ def run_ours(args):
                "sample": f"every {every}th WM seed ({sub.nseeds} seeds) x particles j<{J}: "
                          f"{s} steps in {dt:.1f} s"}
 
+    lengths = None
+    if rank == 0 and (args.lengths or args.config in PAPER_TABLE2):
+        # one more (untimed) pass with per-particle lengths: the Eq. 4 / Fig. 5 statistics
+        tr.track(seeds_d, ids_d, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
+                 max_steps=w.max_steps, rng_seed=w.rng_seed, particles_per_seed=w.particles_per_seed,
+                 out_map=out_map, flags=base_flags | pt.PT_REC_LEN)
+        torch.cuda.synchronize()
+        ns = tr.get_paths(nsteps=True, reason=False, end=False, on_device=True)["nsteps"]
+        hist = torch.zeros(65536, dtype=torch.int64, device=dev)
+        for c0 in range(0, ns.numel(), 1 << 27):
+            hist += torch.bincount(ns[c0:c0 + (1 << 27)].to(torch.int32) & 0xFFFF, minlength=65536)
+        h = hist.cpu().numpy()
+        nz = np.nonzero(h)[0]
+        tot = int((h * np.arange(65536)).sum())
+        cnt = int(h.sum())
+        mean = tot / max(1, cnt)
+        # semilog fit of the length histogram between the 5th and 95th percentiles (Fig. 5c)
+        cdf = np.cumsum(h) / max(1, cnt)
+        lo, hi = int(np.searchsorted(cdf, 0.05)), int(np.searchsorted(cdf, 0.95))
+        xs = np.arange(max(lo, 1), max(hi, lo + 2))
+        ys = h[xs]
+        keep = ys > 0
+        slope = float(np.polyfit(xs[keep], np.log(ys[keep]), 1)[0]) if keep.sum() > 2 else None
+        lengths = {"streamlines": cnt, "total_steps": tot, "mean": mean,
+                   "longest": int(nz.max()) if nz.size else 0,
+                   "lambda_mle": 1.0 / mean if mean > 0 else None,
+                   "lambda_semilog_fit": -slope if slope is not None else None,
+                   "fit_range": [int(xs[0]), int(xs[-1])]}
+        if args.config in PAPER_TABLE2:
+            lengths["paper_table2_context"] = PAPER_TABLE2[args.config]
+
     if rank == 0:
         value = total_steps * args.steps / (ms * 1e-3)
         line = {
@@ -372,6 +413,7 @@ def run_ours(args):
                              % (V * w.volume.nsamples * rb / 1e9)},
             "seeds_per_s": total_seeds * args.steps / (ms * 1e-3),
             "active_lane_fraction": lane_frac,
+            "lengths": lengths,
             "roofline": roof,
             "gather_roofline": gather,
             "cpu_baseline": cpu,
@@ -400,6 +442,8 @@ def main(argv=None):
     ap.add_argument("--no-gather-bench", action="store_true")
     ap.add_argument("--no-per-step-stats", dest="per_step_stats", action="store_false")
     ap.add_argument("--no-map", action="store_true", help="diagnostic: no visitation map")
+    ap.add_argument("--lengths", action="store_true",
+                    help="report streamline-length statistics (untimed extra pass with PT_REC_LEN)")
     ap.add_argument("--tag", default="", help="free-form label echoed by experiment scripts")
     ap.add_argument("--seed-every", type=int, default=1,
                     help="diagnostic (profiling only): every k-th seed of the workload")

@@ -54,6 +54,10 @@ typedef enum { PT_END_MASK = 0, PT_END_CURV = 1, PT_END_MAXLEN = 2 } pt_reason;
 #define PT_SEED_ORDER_INPUT (1u << 9) /* ablation: claim seeds in input order instead of
                                         the default Z-order (Morton) of their voxels;
                                         results are identical either way (R16)           */
+#define PT_SAMPLE_PER_STREAMLINE (1u << 10) /* paper mode (NEXT-1): particle j of a seed
+                                        follows sample volume j mod S for its whole path
+                                        (Alg. 1) instead of a fresh
+                                        random sample every step (R1)                    */
 
 /* Create a context on CUDA device `cuda_device` (the caller's current device is left
  * unchanged).  *out receives the context or NULL.  The stream defaults to the legacy
@@ -99,7 +103,7 @@ typedef struct {
     uint64_t rng_seed;          /* Philox-4x32-10 key (R16)                               */
     int64_t particles_per_seed; /* P >= 1; particle j of seed id k has pid = k*P + j      */
     uint32_t flags;             /* PT_REC_* | PT_MAP_ACCUMULATE | PT_KERNEL_SIMPLE |
-                                   PT_SEED_ORDER_INPUT                                    */
+                                   PT_SEED_ORDER_INPUT | PT_SAMPLE_PER_STREAMLINE         */
     int32_t path_stride;        /* points stored per particle with PT_REC_PATHS (>= 1)    */
 } pt_params;
 

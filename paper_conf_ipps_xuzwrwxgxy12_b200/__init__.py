@@ -24,7 +24,8 @@ __all__ = [
     "PtError", "lib", "Tracker", "pt_create", "pt_destroy", "pt_last_error", "pt_set_stream",
     "pt_load_samples", "pt_track", "pt_get_paths", "pt_get_stats", "pt_gather_bench",
     "pt_record_bytes", "PT_F32", "PT_F16", "PT_REC_LEN", "PT_REC_REASON", "PT_REC_END",
-    "PT_REC_PATHS", "PT_MAP_ACCUMULATE", "PT_KERNEL_SIMPLE", "PT_SEED_ORDER_INPUT", "PT_END_MASK", "PT_END_CURV",
+    "PT_REC_PATHS", "PT_MAP_ACCUMULATE", "PT_KERNEL_SIMPLE", "PT_SEED_ORDER_INPUT",
+    "PT_SAMPLE_PER_STREAMLINE", "PT_END_MASK", "PT_END_CURV",
     "PT_END_MAXLEN", "EXPORTS",
 ]
 
@@ -38,6 +39,7 @@ PT_REC_PATHS = 1 << 3
 PT_MAP_ACCUMULATE = 1 << 4
 PT_KERNEL_SIMPLE = 1 << 8
 PT_SEED_ORDER_INPUT = 1 << 9
+PT_SAMPLE_PER_STREAMLINE = 1 << 10
 
 # every symbol include/pt.h declares
 EXPORTS = ["pt_create", "pt_destroy", "pt_last_error", "pt_set_stream", "pt_load_samples",
@@ -249,6 +251,8 @@ class Tracker:
 
     def track_workload(self, w, flags: int = 0, path_stride: int = 0, seeds=None, seed_ids=None,
                        out_map=None, want_map: bool = True):
+        if getattr(w, "sample_mode", 0) == 1:
+            flags |= PT_SAMPLE_PER_STREAMLINE
         seeds = w.seeds if seeds is None else seeds
         if seed_ids is None and w.seed_ids is not None:
             seed_ids = w.seed_ids

@@ -399,6 +399,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.fcy = (float)a.cy;
     a.fcz = (float)a.cz;
     a.S = (uint32_t)c->vol.nsamples;
+    a.sample_mode = (fl & PT_SAMPLE_PER_STREAMLINE) ? 1u : 0u;
     a.step = p->step;
     a.curv_thr = p->curv_thr;
     a.fib_thr = p->fib_thr;

@@ -38,6 +38,7 @@ struct TrackArgs {
     int cx, cy, cz;              // floor(N/2) per axis
     float fcx, fcy, fcz;         // the same as floats
     uint32_t S;
+    uint32_t sample_mode;        // 0: random sample per step (R1); 1: s = j mod S (NEXT-1)
     float step, curv_thr, fib_thr;
     int max_steps;
     uint32_t key0, key1;

@@ -169,6 +169,7 @@ track_kernel(const __grid_constant__ TrackArgs a) {
     int n = 0;            // committed steps
     uint64_t pid = 0;     // global particle id = seed_id * P + j (RNG key, R16)
     uint32_t run_vox = 0, run_cnt = 0;  // run-length merge of consecutive visits
+    uint32_t sfix = 0;    // paper mode (NEXT-1): the particle's sample volume, j mod S
     R rv;                 // record of the current step
     uint4 W = make_uint4(0u, 0u, 0u, 0u);
 
@@ -252,6 +253,7 @@ track_kernel(const __grid_constant__ TrackArgs a) {
         if (OUT) s_li[threadIdx.x] = li;
         const uint64_t sid = a.seed_ids ? a.seed_ids[si] : si;
         pid = sid * a.P + j;
+        sfix = (uint32_t)(j % a.S);
         qx = __fsub_rn(a.seeds[3 * si + 0], a.fcx);
         qy = __fsub_rn(a.seeds[3 * si + 1], a.fcy);
         qz = __fsub_rn(a.seeds[3 * si + 2], a.fcz);
@@ -332,7 +334,8 @@ track_kernel(const __grid_constant__ TrackArgs a) {
             const uint32_t t0 = (uint32_t)n + (pend ? 1u : 0u);  // a multiple of 3
             W = philox4x32_10(make_uint4(t0 / 3u, (uint32_t)pid, (uint32_t)(pid >> 32), 0u),
                               a.key0, a.key1);
-            ldg_record_if<RB>(alive, a.rec + ((uint64_t)gvox * a.S + sample_of(W.x, a.S)) * RB, rv.w);
+            const uint32_t s0 = a.sample_mode ? sfix : sample_of(W.x, a.S);
+            ldg_record_if<RB>(alive, a.rec + ((uint64_t)gvox * a.S + s0) * RB, rv.w);
             // seed outside the mask (R12) or pending candidate rejected (R11)
             const bool outside = alive && rv.outside();
             why = outside ? kEndMask : why;
@@ -390,7 +393,8 @@ track_kernel(const __grid_constant__ TrackArgs a) {
             pz = go ? dz : pz;
             if (k < 2) {
                 const uint32_t w = (k == 0) ? W.y : W.z;
-                ldg_record_if<RB>(go, a.rec + ((uint64_t)v * a.S + sample_of(w, a.S)) * RB, rv.w);
+                const uint32_t sk = a.sample_mode ? sfix : sample_of(w, a.S);
+                ldg_record_if<RB>(go, a.rec + ((uint64_t)v * a.S + sk) * RB, rv.w);
                 const bool outside = go && rv.outside();  // candidate outside the mask (R11)
                 why = outside ? kEndMask : why;
                 alive = go && !outside;

@@ -29,7 +29,7 @@ import numpy as np
 
 __all__ = [
     "Volume", "Workload", "tube", "crossing", "whole_brain", "isotropic", "bent_tube",
-    "t_junction", "fork", "mirror_x", "to_half", "config", "CONFIGS", "wm_seeds",
+    "t_junction", "fork", "paper_dataset", "mirror_x", "to_half", "config", "CONFIGS", "wm_seeds",
 ]
 
 
@@ -411,6 +411,22 @@ def to_half(w: Workload) -> Workload:
     return w.replace(name=w.name + "_f16", volume=vol)
 
 
+# ----------------------------------------------------------------------------- paper mode
+
+def paper_dataset(which: int = 1, step: float = 0.1, curv_thr: float = 0.9, gen_seed: int = 21) -> Workload:
+    """NEXT-1 workload shaped like the paper's datasets: #1 48x96x96, #2 60x102x102
+    (read as 96x96 / 102x102 in-plane, 48 / 60 slices), brain ellipsoid with c3's
+    proportions, seeds = every brain voxel ("from each voxel in the brain"),
+    50 samples and one streamline per sample volume (P = S = 50, sample_mode 1,
+    Alg. 1), MaxStep = sum of the segmentation array = 1888."""
+    nx, ny, nz = (96, 96, 48) if which == 1 else (102, 102, 60)
+    semi = (0.453 * nx, 0.484 * ny, 0.471 * nz)
+    w = whole_brain(nx=nx, ny=ny, nz=nz, semi=semi, nsamples=50, nfibres=2, particles_per_seed=50,
+                    step=step, curv_thr=curv_thr, max_steps=1888, gen_seed=gen_seed, seeds="brain")
+    return w.replace(name=f"paper_d{which}_step{step}_thr{curv_thr}", sample_mode=1,
+                     recipe=w.recipe + f"; paper mode D{which}, step {step}, dot threshold {curv_thr}")
+
+
 # ----------------------------------------------------------------------------- configs
 
 CONFIGS = {
@@ -422,6 +438,13 @@ CONFIGS = {
     "c4": lambda: to_half(whole_brain()),
     "c5": lambda: to_half(whole_brain(nx=145, ny=174, nz=145, nfibres=3,
                                       semi=(66.0, 82.0, 66.0), particles_per_seed=10000)),
+    # NEXT-1: the paper's own mode on dataset-shaped phantoms (Table II parameters)
+    "d1": lambda: paper_dataset(1, 0.1, 0.9),
+    "d1_s02": lambda: paper_dataset(1, 0.2, 0.8),
+    "d1_s03": lambda: paper_dataset(1, 0.3, 0.85),
+    "d2": lambda: paper_dataset(2, 0.1, 0.9),
+    "d2_s02": lambda: paper_dataset(2, 0.2, 0.85),
+    "d2_s03": lambda: paper_dataset(2, 0.3, 0.8),
 }
 
 

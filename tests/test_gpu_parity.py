@@ -283,3 +283,30 @@ def test_lane_efficiency_and_gather_bench(pt, tracker):
     assert fa > 0.8 and fa > fb, (fa, fb)
     r = tracker.gather_bench(1 << 30, 32)
     assert r > 1e9
+
+
+# ----------------------------------------------------------------------------- NEXT-1 paper mode
+
+def test_paper_mode_closed_form(pt, tracker):
+    """NEXT-1 on the GPU: the alternating-sample tube of the oracle pin, bit-exact."""
+    from tests.test_oracle_pins import _alternating_tube
+    w = _alternating_tube(P=64)
+    g = gpu_run(tracker, w)
+    r = oracle.track(w)
+    assert_parity(g, r)
+
+
+@pytest.mark.parametrize("half", [False, True])
+def test_paper_mode_parity(pt, tracker, half):
+    """NEXT-1: one sample volume per streamline (P = S), every particle and the map, plus
+    paths, on a small paper-dataset-shaped volume."""
+    w = phantom.paper_dataset(1, 0.2, 0.8)
+    w = phantom.wm_seeds(w, every=max(1, w.nseeds // 1500))
+    if half:
+        w = phantom.to_half(w)
+    g = gpu_run(tracker, w, REC_ALL | pt.PT_REC_PATHS, path_stride=256)
+    r = oracle.track(w, path_stride=256, threads=_threads())
+    assert_parity(g, r)
+    assert paths_equal(g["paths"], r["paths"])
+    s = gpu_run(tracker, w, REC_ALL | pt.PT_KERNEL_SIMPLE)
+    assert_parity(s, r)
