@@ -364,6 +364,31 @@ def run_ours(args):
                "sample": f"every {every}th WM seed ({sub.nseeds} seeds) x particles j<{J}: "
                          f"{s} steps in {dt:.1f} s"}
 
+    emulated = None
+    if rank == 0 and world == 1 and args.emulate_ranks:
+        # Projected multi-GPU scaling on ONE GPU: the shard of each rank of an N-way split
+        # (seed i -> rank i mod N, global ids) is timed back to back; N GPUs would finish
+        # when the slowest shard does, plus one NCCL reduce of the map (not timed here).
+        emulated = {}
+        for N in args.emulate_ranks:
+            times, steps_r = [], []
+            for r in range(N):
+                sub = _shard(w, r, N)
+                sd = torch.as_tensor(sub.seeds, device=dev).contiguous()
+                si = torch.as_tensor(sub.ids().astype(np.int64), device=dev).contiguous()
+                for it in range(2):  # warm-up + timed
+                    flush_buf.fill_(1)
+                    tr.track(sd, si, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
+                             max_steps=w.max_steps, rng_seed=w.rng_seed,
+                             particles_per_seed=w.particles_per_seed, out_map=out_map, flags=base_flags)
+                    st_r = tr.stats()
+                times.append(st_r["track_ms"])
+                steps_r.append(st_r["total_steps"])
+            emulated[str(N)] = {"shard_ms": times, "shard_steps": steps_r,
+                                "projected_value": sum(steps_r) / (max(times) * 1e-3),
+                                "imbalance_max_over_mean": max(times) / (sum(times) / len(times))}
+        torch.cuda.synchronize()
+
     lengths = None
     if rank == 0 and (args.lengths or args.config in PAPER_TABLE2):
         # one more (untimed) pass with per-particle lengths: the Eq. 4 / Fig. 5 statistics
@@ -414,6 +439,7 @@ def run_ours(args):
             "seeds_per_s": total_seeds * args.steps / (ms * 1e-3),
             "active_lane_fraction": lane_frac,
             "lengths": lengths,
+            "emulated_scaling": emulated,
             "roofline": roof,
             "gather_roofline": gather,
             "cpu_baseline": cpu,
@@ -442,6 +468,9 @@ def main(argv=None):
     ap.add_argument("--no-gather-bench", action="store_true")
     ap.add_argument("--no-per-step-stats", dest="per_step_stats", action="store_false")
     ap.add_argument("--no-map", action="store_true", help="diagnostic: no visitation map")
+    ap.add_argument("--emulate-ranks", type=lambda x: [int(v) for v in x.split(",") if v], default=[],
+                    help="e.g. 2,4,8: time each rank's seed shard back to back on one GPU and "
+                         "report the projected N-GPU throughput (max shard time)")
     ap.add_argument("--lengths", action="store_true",
                     help="report streamline-length statistics (untimed extra pass with PT_REC_LEN)")
     ap.add_argument("--tag", default="", help="free-form label echoed by experiment scripts")
