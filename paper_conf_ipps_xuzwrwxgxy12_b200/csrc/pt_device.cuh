@@ -141,18 +141,6 @@ __device__ __forceinline__ void ldg_record_if<64>(bool p, const void* ptr, uint3
     ldg_record_if<32>(p, static_cast<const char*>(ptr) + 32, w + 8);
 }
 
-// The same with an L2 cache-eviction policy (createpolicy ... L2::evict_last): keeps the
-// visitation map resident in L2 while the record stream churns through it.
-__device__ __forceinline__ uint64_t l2_evict_last_policy() {
-    uint64_t pol;
-    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
-    return pol;
-}
-__device__ __forceinline__ void red_add_if_hint(bool p, uint32_t* addr, uint32_t v, uint64_t pol) {
-    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %3, 0;\n\t@q red.global.add.L2::cache_hint.u32 [%0], %1, %2;\n\t}"
-                 :: "l"(addr), "r"(v), "l"(pol), "r"((int)p) : "memory");
-}
-
 __device__ __forceinline__ void red_add_if(bool p, uint32_t* addr, uint32_t v) {
     asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q red.global.add.u32 [%0], %1;\n\t}"
                  :: "l"(addr), "r"(v), "r"((int)p) : "memory");

@@ -15,6 +15,10 @@ namespace pt {
 // tickets), so a seed's particles run on one SM (L1 locality) while the chip as a whole
 // works on a compact set of Morton-adjacent seeds (L2 locality).
 constexpr int kThreads = PT_CTA_THREADS;
+#ifndef PT_CTA_THREADS2
+#define PT_CTA_THREADS2 768
+#endif
+constexpr int kThreads2 = PT_CTA_THREADS2;  // CTA size of the 2-slot kernel (<= 85 registers)
 constexpr int kSimpleThreads = 256;  // no-refill ablation kernel
 constexpr uint32_t kSub = 32;
 constexpr uint32_t kMinCtaChunk = 1024;

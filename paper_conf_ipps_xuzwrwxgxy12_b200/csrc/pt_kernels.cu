@@ -24,47 +24,13 @@
 #include "pt_device.cuh"
 #include "pt_internal.h"
 
-#ifndef PT_MIN_BLOCKS
-#define PT_MIN_BLOCKS 1
-#endif
-#ifndef PT_MAP_HINT
-#define PT_MAP_HINT 0  // 1: REDs carry an L2 evict_last policy (measured: no effect)
-#endif
-#ifndef PT_MAP_PERSIST
-#define PT_MAP_PERSIST 0  // 1: persisting L2 access-policy window over the map (measured: no effect)
-#endif
-#ifndef PT_MAP_CACHE
-#define PT_MAP_CACHE 0      // entries of the per-CTA shared-memory count cache (power of 2; 0 = off)
+#ifndef PT_SLOTS
+#define PT_SLOTS 1  // particles per lane in the persistent kernel (1 or 2; 2 measured no faster)
 #endif
 
 namespace pt {
 
 enum { kEndMask = 0, kEndCurv = 1, kEndMaxlen = 2 };
-
-// Per-CTA shared-memory cache of visitation counts (REFILL kernel).  Entry = (voxel+1) << 32
-// | count; direct-mapped by a multiplicative hash.  A flush adds to the entry of its voxel
-// or replaces a different voxel's entry, whose count then goes to the global map with one
-// RED; the CTA drains the table at exit.  Integer sums commute, so the map is unchanged.
-constexpr uint32_t kMapCache = PT_MAP_CACHE;
-
-__device__ __forceinline__ void cache_add(unsigned long long* tab, uint32_t* map, uint32_t v, uint32_t c) {
-    constexpr uint32_t kBits = kMapCache > 1 ? 31 - __builtin_clz(kMapCache) : 0;
-    const uint32_t h = kBits ? (v * 0x9E3779B1u) >> (32 - kBits) : 0u;
-    unsigned long long* e = tab + h;
-    const uint32_t key = v + 1u;
-    unsigned long long old = *reinterpret_cast<volatile unsigned long long*>(e);
-    for (;;) {
-        const uint32_t ok = (uint32_t)(old >> 32), oc = (uint32_t)old;
-        const bool same = ok == key && oc < 0x80000000u;
-        const unsigned long long want = same ? old + c : (((unsigned long long)key << 32) | c);
-        const unsigned long long prev = atomicCAS(e, old, want);
-        if (prev == old) {
-            if (!same && ok != 0u) atomicAdd(map + (ok - 1u), oc);
-            return;
-        }
-        old = prev;
-    }
-}
 
 // CTA work distribution (REFILL kernel): s_work packs (CTA chunk index << 24 | tickets
 // taken).  A warp takes ticket t: t < subs(chunk) -> sub-chunk t of the CTA chunk;
@@ -126,154 +92,207 @@ __device__ __forceinline__ unsigned long long cta_take(unsigned long long* s_wor
     }
 }
 
-// OUT: per-particle outputs or polylines are recorded (compiled out of the bench path).
-template <int F, bool HALF, bool REFILL, bool OUT>
-__global__ void __launch_bounds__(REFILL ? kThreads : kSimpleThreads, PT_MIN_BLOCKS)
-track_kernel(const __grid_constant__ TrackArgs a) {
+// State of one particle slot of a lane.
+template <int F, bool HALF>
+struct Slot {
+    bool alive;        // holds a particle in flight
+    bool pend;         // the round's 3rd candidate step waits for the next round's gather
+    float qx, qy, qz;  // committed position, centred coordinates (R10)
+    float px, py, pz;  // direction of the last (candidate) step
+    uint32_t gvox;     // voxel read by the round-start gather (seed or pending candidate)
+    int n;             // committed steps
+    uint64_t pid;      // global particle id = seed_id * P + j (RNG key, R16)
+    uint32_t run_vox, run_cnt;  // run-length merge of consecutive visits
+    uint32_t sfix;     // paper mode (NEXT-1): the particle's sample volume, j mod S
+    int why;           // >= 0: ended with this reason, outputs pending (finish)
+    uint4 W;           // Philox block of the current round
+    Rec<F, HALF> rv;   // record of the current step
+};
+
+template <bool REFILL, int SLOTS>
+struct Cta {
+    static constexpr int kTPB = REFILL ? (SLOTS == 2 ? kThreads2 : kThreads) : kSimpleThreads;
+};
+
+// The tracking kernel.  OUT: per-particle outputs or polylines are recorded (compiled out of
+// the bench path).  REFILL: persistent CTAs with lane refill (false: one particle per thread,
+// the no-refill ablation).  SLOTS: particles per lane; with 2, a lane interleaves the steps
+// of two independent particles so that one particle's gather is in flight while the other
+// computes (more gathers in flight per SM without more threads, all from the same claim).
+template <int F, bool HALF, bool REFILL, bool OUT, int SLOTS>
+__global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(const __grid_constant__ TrackArgs a) {
     using R = Rec<F, HALF>;
     constexpr int RB = R::kBytes;
-    constexpr int TPB = REFILL ? kThreads : kSimpleThreads;
-    // rarely used state lives in shared memory to keep the hot loop's register count low
-    __shared__ unsigned long long s_li[TPB];     // particle index of this call (outputs)
-    __shared__ uint32_t s_q[TPB / 32][3];        // per-warp sub-chunk: seed, next j, end j
-    __shared__ unsigned long long s_work;        // CTA chunk + tickets (see cta_take)
-#if defined(PT_DIAG_RED) && PT_DIAG_RED == 1
-    __shared__ uint32_t s_diag[1024];
-#endif
+    constexpr int TPB = Cta<REFILL, SLOTS>::kTPB;
+    __shared__ unsigned long long s_li[OUT ? SLOTS * TPB : 1];  // particle index (outputs)
+    __shared__ uint32_t s_q[TPB / 32][3];                        // per-warp sub-chunk
+    __shared__ unsigned long long s_work;                        // CTA claim + tickets
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t wib = threadIdx.x >> 5;
     const uint32_t lt_mask = (1u << lane) - 1u;
-    extern __shared__ unsigned long long s_cache[];  // kMapCache entries when REFILL && map
-    constexpr bool kCache = REFILL && kMapCache > 0;
-    const bool use_cache = kCache && a.map != nullptr;
     const bool has_map = a.map != nullptr;
-    // privatised map: CTA b adds into copy b % map_copies (no cross-SM contention on the
-    // hot lines near the seeds; the copies are summed by map_combine_kernel)
-    uint32_t* const map = has_map ? a.map + (size_t)(blockIdx.x % a.map_copies) *
-                                                  ((size_t)a.nx * a.ny * a.nz)
+    // privatised map copies (PT_MAP_COPIES): CTA b adds into copy b % map_copies
+    uint32_t* const map = has_map ? a.map + (size_t)(blockIdx.x % a.map_copies) * ((size_t)a.nx * a.ny * a.nz)
                                   : nullptr;
-    const uint64_t map_pol = PT_MAP_HINT ? l2_evict_last_policy() : 0ull;
     if (threadIdx.x == 0) s_work = kNoChunk << 24;
-    if constexpr (kCache) {
-        if (use_cache)
-            for (uint32_t i = threadIdx.x; i < kMapCache; i += TPB) s_cache[i] = 0ull;
-    }
-    __syncthreads();
-
-    // ---- per-lane particle state
-    bool alive = false;   // lane holds a particle in flight
-    bool pend = false;    // the round's 3rd candidate step waits for the next round's gather
-    float qx = 0.f, qy = 0.f, qz = 0.f;   // committed position, centred coordinates (R10)
-    float px = 0.f, py = 0.f, pz = 0.f;   // direction of the last (candidate) step
-    uint32_t gvox = 0;    // voxel read by the round-start gather (seed or pending candidate)
-    int n = 0;            // committed steps
-    uint64_t pid = 0;     // global particle id = seed_id * P + j (RNG key, R16)
-    uint32_t run_vox = 0, run_cnt = 0;  // run-length merge of consecutive visits
-    uint32_t sfix = 0;    // paper mode (NEXT-1): the particle's sample volume, j mod S
-    R rv;                 // record of the current step
-    uint4 W = make_uint4(0u, 0u, 0u, 0u);
-
-    // ---- per-lane counters (a lane never sees 2^32 steps in one launch)
-    uint32_t my_steps = 0, my_particles = 0, my_active = 0, rounds = 0;
-    bool exhausted = false;  // warp-uniform
     if (lane == 0) {
         s_q[wib][0] = 0u;
         s_q[wib][1] = 0u;
         s_q[wib][2] = 0u;
     }
-    __syncwarp();
+    __syncthreads();
 
-    int why = -1;  // >= 0: the particle ended with this reason; outputs pending (finish())
+    Slot<F, HALF> P[SLOTS];
+#pragma unroll
+    for (int sl = 0; sl < SLOTS; ++sl) {
+        P[sl].alive = false;
+        P[sl].pend = false;
+        P[sl].qx = P[sl].qy = P[sl].qz = 0.f;
+        P[sl].px = P[sl].py = P[sl].pz = 0.f;
+        P[sl].gvox = 0u;
+        P[sl].n = 0;
+        P[sl].pid = 0ull;
+        P[sl].run_vox = 0u;
+        P[sl].run_cnt = 0u;
+        P[sl].sfix = 0u;
+        P[sl].why = -1;
+        P[sl].W = make_uint4(0u, 0u, 0u, 0u);
+#pragma unroll
+        for (int k = 0; k < R::kWords; ++k) P[sl].rv.w[k] = 0u;
+    }
+    // per-lane counters (a lane never sees 2^32 steps in one launch)
+    uint32_t my_steps = 0, my_particles = 0, my_active = 0, rounds = 0;
+    bool exhausted = false;  // warp-uniform
 
-    auto red = [&](uint32_t v, uint32_t c) {
-        if (kCache && use_cache) cache_add(s_cache, map, v, c);
-        else atomicAdd(map + v, c);  // no return value used -> RED
-    };
-    // a termination only records the reason; the outputs are written once per round for
-    // all ended lanes at the top of the loop (one divergent block instead of one per site)
-    auto end = [&](int w) {
-        why = w;
-        alive = false;
-        pend = false;
+    // a termination only records the reason; outputs and the count flush are written once
+    // per round for all ended particles at the top of the loop
+    auto end = [&](Slot<F, HALF>& x, int w) {
+        x.why = w;
+        x.alive = false;
+        x.pend = false;
     };
     // SetEndPoint()
-    auto finish = [&]() {
+    auto finish = [&](Slot<F, HALF>& x, int sl) {
         if (OUT && (a.o_nsteps || a.o_reason || a.o_end)) {
-            const uint64_t li = s_li[threadIdx.x];
-            if (a.o_nsteps) a.o_nsteps[li] = (uint16_t)n;
-            if (a.o_reason) a.o_reason[li] = (uint8_t)why;
+            const uint64_t li = s_li[sl * TPB + threadIdx.x];
+            if (a.o_nsteps) a.o_nsteps[li] = (uint16_t)x.n;
+            if (a.o_reason) a.o_reason[li] = (uint8_t)x.why;
             if (a.o_end) {
                 float* e = a.o_end + 3 * li;
-                e[0] = __fadd_rn(qx, a.fcx);
-                e[1] = __fadd_rn(qy, a.fcy);
-                e[2] = __fadd_rn(qz, a.fcz);
+                e[0] = __fadd_rn(x.qx, a.fcx);
+                e[1] = __fadd_rn(x.qy, a.fcy);
+                e[2] = __fadd_rn(x.qz, a.fcz);
             }
         }
-        if (has_map && run_cnt) red(run_vox, run_cnt);
-        run_cnt = 0;
-        my_steps += (uint32_t)n;
+        if (has_map && x.run_cnt) atomicAdd(map + x.run_vox, x.run_cnt);  // RED
+        x.run_cnt = 0;
+        my_steps += (uint32_t)x.n;
         my_particles += 1u;
-        why = -1;
+        x.why = -1;
     };
-    // commit a step (lanes with c): new position, one visit of the new voxel (R13);
+    // commit a step (if c): new position, one visit of the new voxel (R13);
     // consecutive visits of the same voxel are merged (run length) and flushed with a
     // predicated RED when the voxel changes.  Straight-line, no branch.
-    auto commit_if = [&](bool c, float x, float y, float z, uint32_t v) {
-        qx = c ? x : qx;
-        qy = c ? y : qy;
-        qz = c ? z : qz;
-        n += c ? 1 : 0;
+    auto commit_if = [&](Slot<F, HALF>& x, int sl, bool c, float nx_, float ny_, float nz_, uint32_t v) {
+        x.qx = c ? nx_ : x.qx;
+        x.qy = c ? ny_ : x.qy;
+        x.qz = c ? nz_ : x.qz;
+        x.n += c ? 1 : 0;
         if (has_map) {
-            const bool change = v != run_vox;
-            if (kCache && use_cache) {
-                if (c && change && run_cnt != 0u) red(run_vox, run_cnt);
-            } else {
-#if defined(PT_DIAG_RED) && PT_DIAG_RED == 1  // diagnostic builds only (wrong maps)
-                if (c && change && run_cnt != 0u) atomicAdd(&s_diag[run_vox & 1023u], run_cnt);
-#elif defined(PT_DIAG_RED) && PT_DIAG_RED == 2
-                red_add_if(c && change && run_cnt != 0u, a.map + ((run_vox & 4095u) + blockIdx.x * 4096u), run_cnt);
-#else
-                if (PT_MAP_HINT) red_add_if_hint(c && change && run_cnt != 0u, map + run_vox, run_cnt, map_pol);
-                else red_add_if(c && change && run_cnt != 0u, map + run_vox, run_cnt);
-#endif
-            }
-            run_cnt = c ? (change ? 1u : run_cnt + 1u) : run_cnt;
-            run_vox = c ? v : run_vox;
+            const bool change = v != x.run_vox;
+            red_add_if(c && change && x.run_cnt != 0u, map + x.run_vox, x.run_cnt);
+            x.run_cnt = c ? (change ? 1u : x.run_cnt + 1u) : x.run_cnt;
+            x.run_vox = c ? v : x.run_vox;
         }
-        if (OUT && a.o_paths && c && n < a.path_stride) {
-            float* pp = a.o_paths + (s_li[threadIdx.x] * (uint64_t)a.path_stride + (uint64_t)n) * 3u;
-            pp[0] = __fadd_rn(qx, a.fcx);
-            pp[1] = __fadd_rn(qy, a.fcy);
-            pp[2] = __fadd_rn(qz, a.fcz);
+        if (OUT && a.o_paths && c && x.n < a.path_stride) {
+            float* pp = a.o_paths + (s_li[sl * TPB + threadIdx.x] * (uint64_t)a.path_stride + (uint64_t)x.n) * 3u;
+            pp[0] = __fadd_rn(x.qx, a.fcx);
+            pp[1] = __fadd_rn(x.qy, a.fcy);
+            pp[2] = __fadd_rn(x.qz, a.fcz);
         }
     };
     // GetStartPoint(): centred seed position, seed voxel (R10, R12)
-    auto start = [&](uint64_t si, uint64_t j) {
+    auto start = [&](Slot<F, HALF>& x, int sl, uint64_t si, uint64_t j) {
         const uint64_t li = si * a.P + j;
-        if (OUT) s_li[threadIdx.x] = li;
+        if (OUT) s_li[sl * TPB + threadIdx.x] = li;
         const uint64_t sid = a.seed_ids ? a.seed_ids[si] : si;
-        pid = sid * a.P + j;
-        sfix = (uint32_t)(j % a.S);
-        qx = __fsub_rn(a.seeds[3 * si + 0], a.fcx);
-        qy = __fsub_rn(a.seeds[3 * si + 1], a.fcy);
-        qz = __fsub_rn(a.seeds[3 * si + 2], a.fcz);
-        n = 0;
-        pend = false;
-        run_cnt = 0;
-        alive = true;
+        x.pid = sid * a.P + j;
+        x.sfix = (uint32_t)(j % a.S);
+        x.qx = __fsub_rn(a.seeds[3 * si + 0], a.fcx);
+        x.qy = __fsub_rn(a.seeds[3 * si + 1], a.fcy);
+        x.qz = __fsub_rn(a.seeds[3 * si + 2], a.fcz);
+        x.n = 0;
+        x.pend = false;
+        x.run_cnt = 0;
+        x.alive = true;
         if (OUT && a.o_paths) {
             float* pp = a.o_paths + li * (uint64_t)a.path_stride * 3u;
-            pp[0] = __fadd_rn(qx, a.fcx);
-            pp[1] = __fadd_rn(qy, a.fcy);
-            pp[2] = __fadd_rn(qz, a.fcz);
+            pp[0] = __fadd_rn(x.qx, a.fcx);
+            pp[1] = __fadd_rn(x.qy, a.fcy);
+            pp[2] = __fadd_rn(x.qz, a.fcz);
         }
-        const int ix = axis_index(qx, a.cx), iy = axis_index(qy, a.cy), iz = axis_index(qz, a.cz);
-        if ((unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny &&
-            (unsigned)iz < (unsigned)a.nz) {
-            gvox = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
+        const int ix = axis_index(x.qx, a.cx), iy = axis_index(x.qy, a.cy), iz = axis_index(x.qz, a.cz);
+        if ((unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny && (unsigned)iz < (unsigned)a.nz) {
+            x.gvox = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
         } else {
-            end(kEndMask);  // seed outside the volume (R12): finished right away, so the
-            finish();       // refill loop may hand this lane another particle
+            end(x, kEndMask);  // seed outside the volume (R12): finished right away, so the
+            finish(x, sl);     // refill loop may hand this lane another particle
+        }
+    };
+    // one step of Alg. 1's inner loop for a slot; k = position in the round
+    auto step = [&](Slot<F, HALF>& x, int sl, int k) {
+        my_active += x.alive ? 1u : 0u;
+        const bool first = x.n == 0;
+        // choose the fibre closest to the previous direction: eligible iff
+        // f_j > fib_thr (R7), strict >, lowest j wins (R8); the first step takes fibre 0
+        // (R5).  "Interpolation()" of Alg. 1 = this sample's record at the voxel (R2).
+        float vx, vy, vz, f0;
+        x.rv.fibre(0, vx, vy, vz, f0);
+        float bc = __fadd_rn(__fadd_rn(__fmul_rn(vx, x.px), __fmul_rn(vy, x.py)), __fmul_rn(vz, x.pz));
+        float best = f0 > a.fib_thr ? fabsf(bc) : -1.f;
+#pragma unroll
+        for (int j = 1; j < F; ++j) {
+            float ux, uy, uz, fu;
+            x.rv.fibre(j, ux, uy, uz, fu);
+            const float cj = __fadd_rn(__fadd_rn(__fmul_rn(ux, x.px), __fmul_rn(uy, x.py)), __fmul_rn(uz, x.pz));
+            const bool pick = !first && fu > a.fib_thr && fabsf(cj) > best;
+            best = pick ? fabsf(cj) : best;
+            bc = pick ? cj : bc;
+            vx = pick ? ux : vx;
+            vy = pick ? uy : vy;
+            vz = pick ? uz : vz;
+        }
+        // maximum angle, measured by the dot product (R4); orientation
+        // kept (R9); first step: sign = top bit of word 3 of block 0 (R6, R16)
+        const bool curv_ok = first || fabsf(bc) > a.curv_thr;
+        const bool neg = first ? (x.W.w >> 31) != 0u : !(bc > 0.f);
+        // StepToNextPoint(): q' = q + h * (sign * v), no FMA
+        const float dx = neg ? -vx : vx, dy = neg ? -vy : vy, dz = neg ? -vz : vz;
+        const float nqx = __fadd_rn(x.qx, __fmul_rn(a.step, dx));
+        const float nqy = __fadd_rn(x.qy, __fmul_rn(a.step, dy));
+        const float nqz = __fadd_rn(x.qz, __fmul_rn(a.step, dz));
+        const int ix = axis_index(nqx, a.cx), iy = axis_index(nqy, a.cy), iz = axis_index(nqz, a.cz);
+        const bool inb = (unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny && (unsigned)iz < (unsigned)a.nz;
+        const uint32_t v = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
+        // stop criteria in order: maximum steps (R14), angle, volume (R11)
+        const bool maxed = x.n == a.max_steps;
+        const bool go = x.alive && !maxed && curv_ok && inb;
+        x.why = (x.alive && !go) ? (maxed ? kEndMaxlen : (!curv_ok ? kEndCurv : kEndMask)) : x.why;
+        x.alive = go;
+        x.px = go ? dx : x.px;
+        x.py = go ? dy : x.py;
+        x.pz = go ? dz : x.pz;
+        if (k < 2) {
+            const uint32_t w = (k == 0) ? x.W.y : x.W.z;
+            const uint32_t sk = a.sample_mode ? x.sfix : sample_of(w, a.S);
+            ldg_record_if<RB>(go, a.rec + ((uint64_t)v * a.S + sk) * RB, x.rv.w);
+            const bool outside = go && x.rv.outside();  // candidate outside the mask (R11)
+            x.why = outside ? kEndMask : x.why;
+            x.alive = go && !outside;
+            commit_if(x, sl, x.alive, nqx, nqy, nqz, v);
+        } else {
+            x.pend = go;  // next round's start gathers and tests it
+            x.gvox = go ? v : x.gvox;
         }
     };
 
@@ -281,39 +300,47 @@ track_kernel(const __grid_constant__ TrackArgs a) {
         const uint64_t g = (uint64_t)blockIdx.x * TPB + threadIdx.x;
         if (g < a.nparticles) {
             const uint64_t si = g / a.P;
-            start(si, g - si * a.P);
+            start(P[0], 0, si, g - si * a.P);
         }
     }
 
     for (;;) {
-        if (why >= 0) finish();  // particles that ended during the previous round
+#pragma unroll
+        for (int sl = 0; sl < SLOTS; ++sl)
+            if (P[sl].why >= 0) finish(P[sl], sl);  // particles that ended in the last round
 
         // ------------------------------------------------ lane refill (replaces the
         // paper's CPU Reduction()/segment relaunch)
         if (REFILL) {
-            uint32_t need = __ballot_sync(kFull, !alive);
-            if (need != 0u && !exhausted) {
+            bool any_need = false;
+#pragma unroll
+            for (int sl = 0; sl < SLOTS; ++sl) any_need |= !P[sl].alive;
+            if (__any_sync(kFull, any_need) && !exhausted) {
                 uint32_t cseed = s_q[wib][0], cnext = s_q[wib][1], cend = s_q[wib][2];
-                while (need != 0u) {
-                    if (cnext == cend) {
-                        unsigned long long r = 0;
-                        if (lane == 0) r = cta_take(&s_work, a);
-                        r = __shfl_sync(kFull, r, 0);
-                        if (r == kNoWork) {
-                            exhausted = true;
-                            break;
+#pragma unroll
+                for (int sl = 0; sl < SLOTS; ++sl) {
+                    uint32_t need = __ballot_sync(kFull, !P[sl].alive);
+                    while (need != 0u && !exhausted) {
+                        if (cnext == cend) {
+                            unsigned long long r = 0;
+                            if (lane == 0) r = cta_take(&s_work, a);
+                            r = __shfl_sync(kFull, r, 0);
+                            if (r == kNoWork) {
+                                exhausted = true;
+                                break;
+                            }
+                            cseed = (uint32_t)(r >> 32);
+                            cnext = (uint32_t)r;
+                            const uint64_t e = (uint64_t)cnext + kSub;
+                            cend = (uint32_t)(e < a.P ? e : a.P);
                         }
-                        cseed = (uint32_t)(r >> 32);
-                        cnext = (uint32_t)r;
-                        const uint64_t e = (uint64_t)cnext + kSub;
-                        cend = (uint32_t)(e < a.P ? e : a.P);
+                        const uint32_t avail = cend - cnext;
+                        const uint32_t rank = __popc(need & lt_mask);
+                        if (!P[sl].alive && rank < avail) start(P[sl], sl, cseed, (uint64_t)(cnext + rank));
+                        const uint32_t cnt = (uint32_t)__popc(need);
+                        cnext += cnt < avail ? cnt : avail;
+                        need = __ballot_sync(kFull, !P[sl].alive);
                     }
-                    const uint32_t avail = cend - cnext;
-                    const uint32_t rank = __popc(need & lt_mask);
-                    if (!alive && rank < avail) start(cseed, (uint64_t)(cnext + rank));
-                    const uint32_t cnt = (uint32_t)__popc(need);
-                    cnext += cnt < avail ? cnt : avail;
-                    need = __ballot_sync(kFull, !alive);
                 }
                 __syncwarp();
                 if (lane == 0) {
@@ -324,96 +351,41 @@ track_kernel(const __grid_constant__ TrackArgs a) {
                 __syncwarp();
             }
         }
-        if (!__any_sync(kFull, alive)) break;
+        bool any_alive = false;
+#pragma unroll
+        for (int sl = 0; sl < SLOTS; ++sl) any_alive |= P[sl].alive;
+        if (!__any_sync(kFull, any_alive)) break;
         rounds += 1u;
 
-        // ------------------------------------------------ round start: one Philox block,
-        // gather of (pending candidate | seed) voxel = mask test + first step's record.
-        // Straight-line code: every lane computes, only live lanes load / commit.
-        {
-            const uint32_t t0 = (uint32_t)n + (pend ? 1u : 0u);  // a multiple of 3
-            W = philox4x32_10(make_uint4(t0 / 3u, (uint32_t)pid, (uint32_t)(pid >> 32), 0u),
-                              a.key0, a.key1);
-            const uint32_t s0 = a.sample_mode ? sfix : sample_of(W.x, a.S);
-            ldg_record_if<RB>(alive, a.rec + ((uint64_t)gvox * a.S + s0) * RB, rv.w);
+        // ------------------------------------------------ round start: one Philox block per
+        // slot, gather of (pending candidate | seed) voxel = mask test + first step's record;
+        // the slots' gathers are issued back to back so they are in flight together
+#pragma unroll
+        for (int sl = 0; sl < SLOTS; ++sl) {
+            Slot<F, HALF>& x = P[sl];
+            const uint32_t t0 = (uint32_t)x.n + (x.pend ? 1u : 0u);  // a multiple of 3
+            x.W = philox4x32_10(make_uint4(t0 / 3u, (uint32_t)x.pid, (uint32_t)(x.pid >> 32), 0u), a.key0, a.key1);
+            const uint32_t s0 = a.sample_mode ? x.sfix : sample_of(x.W.x, a.S);
+            ldg_record_if<RB>(x.alive, a.rec + ((uint64_t)x.gvox * a.S + s0) * RB, x.rv.w);
+        }
+#pragma unroll
+        for (int sl = 0; sl < SLOTS; ++sl) {
+            Slot<F, HALF>& x = P[sl];
             // seed outside the mask (R12) or pending candidate rejected (R11)
-            const bool outside = alive && rv.outside();
-            why = outside ? kEndMask : why;
-            alive = alive && !outside;
+            const bool outside = x.alive && x.rv.outside();
+            x.why = outside ? kEndMask : x.why;
+            x.alive = x.alive && !outside;
             // accepted candidate: recomputed bit-identically from (q, d) instead of kept
-            commit_if(pend && !outside, __fadd_rn(qx, __fmul_rn(a.step, px)),
-                      __fadd_rn(qy, __fmul_rn(a.step, py)), __fadd_rn(qz, __fmul_rn(a.step, pz)), gvox);
-            pend = false;
+            commit_if(x, sl, x.pend && !outside, __fadd_rn(x.qx, __fmul_rn(a.step, x.px)),
+                      __fadd_rn(x.qy, __fmul_rn(a.step, x.py)), __fadd_rn(x.qz, __fmul_rn(a.step, x.pz)), x.gvox);
+            x.pend = false;
         }
 
-        // ------------------------------------------------ three steps
+        // ------------------------------------------------ three steps, slots interleaved
 #pragma unroll
         for (int k = 0; k < 3; ++k) {
-            my_active += alive ? 1u : 0u;
-            const bool first = n == 0;
-            // choose the fibre closest to the previous direction: eligible iff
-            // f_j > fib_thr (R7), strict >, lowest j wins (R8); the first step takes fibre 0
-            // (R5).  "Interpolation()" of Alg. 1 = this sample's record at the voxel (R2).
-            float vx, vy, vz, f0;
-            rv.fibre(0, vx, vy, vz, f0);
-            float bc = __fadd_rn(__fadd_rn(__fmul_rn(vx, px), __fmul_rn(vy, py)), __fmul_rn(vz, pz));
-            float best = f0 > a.fib_thr ? fabsf(bc) : -1.f;
 #pragma unroll
-            for (int j = 1; j < F; ++j) {
-                float ux, uy, uz, fu;
-                rv.fibre(j, ux, uy, uz, fu);
-                const float cj = __fadd_rn(__fadd_rn(__fmul_rn(ux, px), __fmul_rn(uy, py)), __fmul_rn(uz, pz));
-                const bool pick = !first && fu > a.fib_thr && fabsf(cj) > best;
-                best = pick ? fabsf(cj) : best;
-                bc = pick ? cj : bc;
-                vx = pick ? ux : vx;
-                vy = pick ? uy : vy;
-                vz = pick ? uz : vz;
-            }
-            // maximum angle, measured by the dot product (R4); orientation
-            // kept (R9); first step: sign = top bit of word 3 of block 0 (R6, R16)
-            const bool curv_ok = first || fabsf(bc) > a.curv_thr;
-            const bool neg = first ? (W.w >> 31) != 0u : !(bc > 0.f);
-            // StepToNextPoint(): q' = q + h * (sign * v), no FMA
-            const float dx = neg ? -vx : vx, dy = neg ? -vy : vy, dz = neg ? -vz : vz;
-            const float nqx = __fadd_rn(qx, __fmul_rn(a.step, dx));
-            const float nqy = __fadd_rn(qy, __fmul_rn(a.step, dy));
-            const float nqz = __fadd_rn(qz, __fmul_rn(a.step, dz));
-            const int ix = axis_index(nqx, a.cx), iy = axis_index(nqy, a.cy), iz = axis_index(nqz, a.cz);
-            const bool inb = (unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny &&
-                             (unsigned)iz < (unsigned)a.nz;
-            const uint32_t v = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
-            // stop criteria in order: maximum steps (R14), angle, volume (R11)
-            const bool maxed = n == a.max_steps;
-            const bool go = alive && !maxed && curv_ok && inb;
-            why = (alive && !go) ? (maxed ? kEndMaxlen : (!curv_ok ? kEndCurv : kEndMask)) : why;
-            alive = go;
-            px = go ? dx : px;
-            py = go ? dy : py;
-            pz = go ? dz : pz;
-            if (k < 2) {
-                const uint32_t w = (k == 0) ? W.y : W.z;
-                const uint32_t sk = a.sample_mode ? sfix : sample_of(w, a.S);
-                ldg_record_if<RB>(go, a.rec + ((uint64_t)v * a.S + sk) * RB, rv.w);
-                const bool outside = go && rv.outside();  // candidate outside the mask (R11)
-                why = outside ? kEndMask : why;
-                alive = go && !outside;
-                commit_if(alive, nqx, nqy, nqz, v);
-            } else {
-                pend = go;  // next round's start gathers and tests it
-                gvox = go ? v : gvox;
-            }
-        }
-    }
-
-    // ---- drain the count cache
-    if constexpr (kCache) {
-        if (use_cache) {
-            __syncthreads();
-            for (uint32_t i = threadIdx.x; i < kMapCache; i += TPB) {
-                const unsigned long long e = s_cache[i];
-                if (e >> 32) atomicAdd(map + ((uint32_t)(e >> 32) - 1u), (uint32_t)e);
-            }
+            for (int sl = 0; sl < SLOTS; ++sl) step(P[sl], sl, k);
         }
     }
 
@@ -428,7 +400,7 @@ track_kernel(const __grid_constant__ TrackArgs a) {
         atomicAdd(a.stats + kStatSteps, (unsigned long long)my_steps);
         atomicAdd(a.stats + kStatParticles, (unsigned long long)my_particles);
         atomicAdd(a.stats + kStatLaneActive, (unsigned long long)my_active);
-        atomicAdd(a.stats + kStatLaneSlots, (unsigned long long)rounds * 3ull * 32ull);
+        atomicAdd(a.stats + kStatLaneSlots, (unsigned long long)rounds * 3ull * 32ull * SLOTS);
     }
 }
 
@@ -587,50 +559,23 @@ __global__ void __launch_bounds__(256) gather_bench_kernel(const uint8_t* __rest
 // ------------------------------------------------------------------------- launchers
 template <int F, bool HALF, bool REFILL, bool OUT>
 static cudaError_t launch_t(const TrackArgs& a, int num_sms, cudaStream_t st) {
-    auto k = track_kernel<F, HALF, REFILL, OUT>;
-    constexpr int TPB = REFILL ? kThreads : kSimpleThreads;
+    constexpr int SL = REFILL ? PT_SLOTS : 1;
+    auto k = track_kernel<F, HALF, REFILL, OUT, SL>;
+    constexpr int TPB = Cta<REFILL, SL>::kTPB;
     if (a.nparticles == 0) return cudaSuccess;
-    const size_t dyn = (REFILL && kMapCache > 0 && a.map) ? kMapCache * sizeof(unsigned long long) : 0;
     unsigned grid;
     if (REFILL) {
         int per_sm = 0;
-        cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)(kMapCache * sizeof(unsigned long long)));
-        if (e == cudaSuccess)  // prefer L1 over shared memory: records are gathered through L1
-            e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, kMapCache ? -1 : 0);
-        if (e != cudaSuccess) return e;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, TPB, dyn);
+        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, TPB, 0);
         if (e != cudaSuccess) return e;
         if (per_sm < 1) return cudaErrorInvalidConfiguration;
-        const uint64_t need = (a.nparticles + TPB - 1) / TPB;
+        const uint64_t need = (a.nparticles + (uint64_t)TPB * SL - 1) / ((uint64_t)TPB * SL);
         const uint64_t full = (uint64_t)num_sms * (uint64_t)per_sm;
         grid = (unsigned)(need < full ? need : full);
     } else {
         grid = (unsigned)((a.nparticles + TPB - 1) / TPB);
     }
-    if (PT_MAP_PERSIST && REFILL && a.map) {
-        cudaLaunchConfig_t cfg = {};
-        cfg.gridDim = dim3(grid);
-        cfg.blockDim = dim3(TPB);
-        cfg.dynamicSmemBytes = dyn;
-        cfg.stream = st;
-        cudaLaunchAttribute at[1];
-        at[0].id = cudaLaunchAttributeAccessPolicyWindow;
-        at[0].val.accessPolicyWindow.base_ptr = a.map;
-        at[0].val.accessPolicyWindow.num_bytes = (size_t)a.nx * a.ny * a.nz * sizeof(uint32_t);
-        at[0].val.accessPolicyWindow.hitRatio = 1.0f;
-        at[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-        at[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-        cfg.attrs = at;
-        cfg.numAttrs = 1;
-        size_t lim = 0;
-        cudaDeviceGetLimit(&lim, cudaLimitPersistingL2CacheSize);
-        if (lim < at[0].val.accessPolicyWindow.num_bytes)
-            cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, at[0].val.accessPolicyWindow.num_bytes);
-        cudaGetLastError();
-        return cudaLaunchKernelEx(&cfg, k, a);
-    }
-    k<<<grid, TPB, dyn, st>>>(a);
+    k<<<grid, TPB, 0, st>>>(a);
     return cudaGetLastError();
 }
 
