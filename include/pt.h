@@ -48,7 +48,10 @@ typedef enum { PT_END_MASK = 0, PT_END_CURV = 1, PT_END_MAXLEN = 2 } pt_reason;
 #define PT_REC_REASON     (1u << 1)  /* record per-particle pt_reason (uint8)           */
 #define PT_REC_END        (1u << 2)  /* record per-particle end point (3 x float32)     */
 #define PT_REC_PATHS      (1u << 3)  /* record polylines, path_stride points/particle   */
-#define PT_MAP_ACCUMULATE (1u << 4)  /* add to the map instead of zeroing it first      */
+#define PT_MAP_ACCUMULATE (1u << 4)  /* add to the map (and the connectivity matrix)
+                                        instead of zeroing it first                     */
+#define PT_REC_CONN       (1u << 5)  /* record the seed x target connectivity matrix for
+                                        the targets of pt_load_targets (NEXT-2)          */
 #define PT_KERNEL_SIMPLE  (1u << 8)  /* ablation: one thread per particle, no lane
                                         refill (the paper's "Extreme case 1")   */
 #define PT_SEED_ORDER_INPUT (1u << 9) /* ablation: claim seeds in input order instead of
@@ -123,6 +126,23 @@ typedef struct {
  * PT_ERR_OOM; PT_ERR_CUDA.  Map overflow is reported by pt_get_stats/pt_get_paths. */
 pt_status pt_track(pt_ctx* ctx, const float* seeds_xyz, const uint64_t* seed_ids,
                    int64_t nseeds, const pt_params* params, uint32_t* map);
+
+/* Target regions for the seed x target connectivity matrix (NEXT-2; the connectivity
+ * estimate of P:L109, "counting the number of streamlines passing through B, and dividing
+ * it by the total number", with B a labelled region).
+ *   labels  : [nz][ny][nx] uint8 of the loaded volume's shape, 0 = no target, t in
+ *             1..ntargets = target t-1.  Host or device; copied.  NULL (or ntargets 0)
+ *             removes the targets.
+ *   ntargets: 0..64.
+ * Errors: PT_ERR_STATE before pt_load_samples; PT_ERR_ARG for ntargets > 64. */
+pt_status pt_load_targets(pt_ctx* ctx, const uint8_t* labels, int32_t ntargets);
+
+/* Seed x target matrix of the last pt_track with PT_REC_CONN: out[s][t] (uint32) = number
+ * of seed s's particles whose path (the voxels of its committed steps, R13/R21) enters
+ * target t at least once; s = seed index of that call.  capacity = elements out holds
+ * (>= nseeds * ntargets, else PT_ERR_ARG); *count receives nseeds * ntargets (query with
+ * out = NULL).  Host or device out; synchronises ctx's stream. */
+pt_status pt_get_connectivity(pt_ctx* ctx, uint32_t* out, int64_t capacity, int64_t* count);
 
 /* Per-particle outputs of the last pt_track, particle index = seed_index*P + j.
  * Set capacity = number of particles the buffers hold; NULL buffers are skipped;

@@ -71,7 +71,7 @@ def lib():
             L.oracle_sample_index.restype = ctypes.c_uint32
             L.oracle_track.argtypes = [ctypes.POINTER(_Volume), ctypes.POINTER(_Params), vp, vp,
                                        ctypes.c_int64, ctypes.c_int64, ctypes.c_int64,
-                                       vp, vp, vp, vp, vp, ctypes.c_int32]
+                                       vp, vp, vp, vp, vp, ctypes.c_int32, vp, ctypes.c_int32, vp]
             L.oracle_track.restype = ctypes.c_int
             _lib = L
     return _lib
@@ -117,12 +117,13 @@ def _structs(volume, step, curv_thr, fib_thr, max_steps, rng_seed, P, sample_mod
 
 
 def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = True,
-          want_particles: bool = True, path_stride: int = 0, threads: int = 1) -> dict:
+          want_particles: bool = True, path_stride: int = 0, threads: int = 1,
+          labels: Optional[np.ndarray] = None, ntargets: int = 0) -> dict:
     """Run the oracle on workload ``w`` (a phantom.Workload or duck-typed equivalent).
 
     Returns dict(map=uint64[Z][Y][X] or None, nsteps=int32[n], reason=uint8[n],
-    end=float32[n][3], paths=float32[n][path_stride][3] or None), particles ordered
-    (seed index, j).  ``threads`` > 1 runs independent single-threaded oracle calls on
+    end=float32[n][3], paths=float32[n][path_stride][3] or None, conn=uint64[nseeds][ntargets]
+    or None), particles ordered (seed index, j).  ``threads`` > 1 runs independent single-threaded oracle calls on
     disjoint seed shards (seed i -> worker i mod threads) and sums their maps.
     """
     v = w.volume
@@ -142,6 +143,9 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
     L = lib()
     threads = max(1, min(int(threads), ns)) if ns else 1
 
+    lab = None if labels is None else np.ascontiguousarray(labels, np.uint8)
+    T = int(ntargets) if lab is not None else 0
+
     def run(shard: np.ndarray, mp: Optional[np.ndarray]):
         sd = np.ascontiguousarray(seeds[shard])
         si = np.ascontiguousarray(ids[shard])
@@ -150,12 +154,13 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
         lr = np.zeros(m, np.uint8) if want_particles else None
         le = np.zeros((m, 3), np.float32) if want_particles else None
         lp = np.zeros((m, path_stride, 3), np.float32) if paths is not None else None
+        lc = np.zeros((len(shard), T), np.uint64) if T else None
         rc = L.oracle_track(ctypes.byref(vs), ctypes.byref(ps), sd.ctypes.data, si.ctypes.data,
                             len(shard), j_begin, j_end, _ptr(mp), _ptr(ln), _ptr(lr), _ptr(le),
-                            _ptr(lp), path_stride)
+                            _ptr(lp), path_stride, _ptr(lab), T, _ptr(lc))
         if rc != 0:
             raise ValueError(f"oracle_track rejected its arguments (rc={rc})")
-        return ln, lr, le, lp
+        return ln, lr, le, lp, lc
 
     maps = [np.zeros((v.nz, v.ny, v.nx), np.uint64) if want_map else None for _ in range(threads)]
     shards = [np.arange(t, ns, threads) for t in range(threads)]
@@ -172,8 +177,11 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
             t.join()
         if any(r is None for r in results):
             raise RuntimeError("oracle worker failed")
+    conn = np.zeros((ns, T), np.uint64) if T else None
     for t, shard in enumerate(shards):
-        ln, lr, le, lp = results[t]
+        ln, lr, le, lp, lc = results[t]
+        if conn is not None and len(shard):
+            conn[shard] = lc
         if len(shard) == 0:
             continue
         rows = (shard[:, None] * npp + np.arange(npp)[None, :]).ravel()
@@ -188,4 +196,4 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
         mp = maps[0]
         for m in maps[1:]:
             mp += m
-    return dict(map=mp, nsteps=nsteps, reason=reason, end=end, paths=paths)
+    return dict(map=mp, nsteps=nsteps, reason=reason, end=end, paths=paths, conn=conn)

@@ -15,6 +15,7 @@
 #include <float.h>
 #include <math.h>
 #include <stddef.h>
+#include <string.h>
 
 #if !defined(FLT_EVAL_METHOD) || FLT_EVAL_METHOD != 0
 #error "oracle needs FLT_EVAL_METHOD == 0 (binary32 evaluation)"
@@ -134,7 +135,8 @@ int oracle_track(const oracle_volume* vol, const oracle_params* prm,
                  const float* seeds_xyz, const uint64_t* seed_ids, int64_t nseeds,
                  int64_t j_begin, int64_t j_end,
                  uint64_t* map, int32_t* nsteps, uint8_t* reason, float* end_xyz,
-                 float* paths, int32_t path_stride) {
+                 float* paths, int32_t path_stride,
+                 const uint8_t* labels, int32_t ntargets, uint64_t* conn) {
     const int F = vol->nfibres;
     const uint32_t S = (uint32_t)vol->nsamples;
     const uint64_t P = (uint64_t)prm->particles_per_seed;
@@ -146,6 +148,7 @@ int oracle_track(const oracle_volume* vol, const oracle_params* prm,
     if (!valid_params(vol, prm)) return -1;
     if (nseeds < 0 || j_begin < 0 || j_end < j_begin || (uint64_t)j_end > P) return -2;
     if (paths && path_stride < 1) return -3;
+    if (conn && (!labels || ntargets < 1 || ntargets > 64)) return -5;
 
     for (si = 0; si < nseeds; ++si) {
         const uint64_t sid = seed_ids ? seed_ids[si] : (uint64_t)si;
@@ -155,11 +158,13 @@ int oracle_track(const oracle_volume* vol, const oracle_params* prm,
             const int64_t out = si * npp + (jj - j_begin);
             const uint32_t plo = (uint32_t)pid, phi = (uint32_t)(pid >> 32);
             float q[3], p[3] = {0.0f, 0.0f, 0.0f};
+            unsigned char entered[64];   /* NEXT-2: targets this streamline passed through */
             int64_t vox;
             int32_t n = 0;
             int why;
             int a;
 
+            memset(entered, 0, sizeof entered);
             /* GetStartPoint(): centred coordinates q = x - c (R10). */
             for (a = 0; a < 3; ++a) q[a] = seeds_xyz[si * 3 + a] - c[a];
             if (paths) {
@@ -237,6 +242,8 @@ int oracle_track(const oracle_volume* vol, const oracle_params* prm,
                     vox = vn;
                     n = n + 1;
                     if (map) map[vox] += 1u;
+                    if (conn && labels[vox] != 0 && labels[vox] <= ntargets)
+                        entered[labels[vox] - 1] = 1;     /* R21: committed steps only */
                     if (paths && n < path_stride) {
                         for (a = 0; a < 3; ++a) paths[(out * path_stride + n) * 3 + a] = q[a] + c[a];
                     }
@@ -246,6 +253,12 @@ int oracle_track(const oracle_volume* vol, const oracle_params* prm,
             if (nsteps) nsteps[out] = n;
             if (reason) reason[out] = (uint8_t)why;
             if (end_xyz) for (a = 0; a < 3; ++a) end_xyz[out * 3 + a] = q[a] + c[a];
+            /* count the streamlines passing through each target, once each */
+            if (conn) {
+                int t;
+                for (t = 0; t < ntargets; ++t)
+                    if (entered[t]) conn[si * ntargets + t] += 1u;
+            }
         }
     }
     return 0;

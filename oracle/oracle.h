@@ -66,12 +66,16 @@ uint32_t oracle_sample_index(uint32_t w, uint32_t nsamples);
  *                            each may be NULL
  *   paths     [particle][path_stride][3] corner-coordinate positions, point 0 = start,
  *             point k = after the k-th committed step, unused points = NaN; may be NULL
+ *   labels    [Z][Y][X] target labels (0 = none, t+1 = target t) or NULL; ntargets <= 64
+ *   conn      [nseeds][ntargets] uint64, accumulated: number of the seed's particles whose
+ *             committed steps enter target t at least once (NEXT-2; R21); may be NULL
  * Returns 0 on success, <0 on invalid arguments (nothing written). */
 int oracle_track(const oracle_volume* vol, const oracle_params* prm,
                  const float* seeds_xyz, const uint64_t* seed_ids, int64_t nseeds,
                  int64_t j_begin, int64_t j_end,
                  uint64_t* map, int32_t* nsteps, uint8_t* reason, float* end_xyz,
-                 float* paths, int32_t path_stride);
+                 float* paths, int32_t path_stride,
+                 const uint8_t* labels, int32_t ntargets, uint64_t* conn);
 
 #ifdef __cplusplus
 }

@@ -25,7 +25,7 @@ __all__ = [
     "pt_load_samples", "pt_track", "pt_get_paths", "pt_get_stats", "pt_gather_bench",
     "pt_record_bytes", "PT_F32", "PT_F16", "PT_REC_LEN", "PT_REC_REASON", "PT_REC_END",
     "PT_REC_PATHS", "PT_MAP_ACCUMULATE", "PT_KERNEL_SIMPLE", "PT_SEED_ORDER_INPUT",
-    "PT_SAMPLE_PER_STREAMLINE", "PT_END_MASK", "PT_END_CURV",
+    "PT_SAMPLE_PER_STREAMLINE", "PT_REC_CONN", "pt_load_targets", "pt_get_connectivity", "PT_END_MASK", "PT_END_CURV",
     "PT_END_MAXLEN", "EXPORTS",
 ]
 
@@ -37,13 +37,15 @@ PT_REC_REASON = 1 << 1
 PT_REC_END = 1 << 2
 PT_REC_PATHS = 1 << 3
 PT_MAP_ACCUMULATE = 1 << 4
+PT_REC_CONN = 1 << 5
 PT_KERNEL_SIMPLE = 1 << 8
 PT_SEED_ORDER_INPUT = 1 << 9
 PT_SAMPLE_PER_STREAMLINE = 1 << 10
 
 # every symbol include/pt.h declares
 EXPORTS = ["pt_create", "pt_destroy", "pt_last_error", "pt_set_stream", "pt_load_samples",
-           "pt_track", "pt_get_paths", "pt_get_stats", "pt_gather_bench", "pt_record_bytes"]
+           "pt_track", "pt_get_paths", "pt_get_stats", "pt_gather_bench", "pt_record_bytes",
+           "pt_load_targets", "pt_get_connectivity"]
 
 _STATUS = {1: "PT_ERR_ARG", 2: "PT_ERR_STATE", 3: "PT_ERR_OOM", 4: "PT_ERR_CUDA", 5: "PT_ERR_OVERFLOW"}
 
@@ -110,6 +112,10 @@ def lib() -> ctypes.CDLL:
     L.pt_get_stats.restype = ctypes.c_int
     L.pt_gather_bench.argtypes = [vp, ctypes.c_int64, ctypes.c_int32, P(ctypes.c_double)]
     L.pt_gather_bench.restype = ctypes.c_int
+    L.pt_load_targets.argtypes = [vp, vp, ctypes.c_int32]
+    L.pt_load_targets.restype = ctypes.c_int
+    L.pt_get_connectivity.argtypes = [vp, vp, ctypes.c_int64, P(ctypes.c_int64)]
+    L.pt_get_connectivity.restype = ctypes.c_int
     L.pt_record_bytes.argtypes = [ctypes.c_int32, ctypes.c_int32]
     L.pt_record_bytes.restype = ctypes.c_int32
     _lib = L
@@ -164,6 +170,16 @@ def pt_get_stats(ctx) -> pt_stats:
     s = pt_stats()
     _check(ctx, lib().pt_get_stats(ctx, ctypes.byref(s)))
     return s
+
+
+def pt_load_targets(ctx, labels_ptr, ntargets: int) -> None:
+    _check(ctx, lib().pt_load_targets(ctx, labels_ptr, ntargets))
+
+
+def pt_get_connectivity(ctx, out_ptr, capacity: int) -> int:
+    n = ctypes.c_int64()
+    _check(ctx, lib().pt_get_connectivity(ctx, out_ptr, capacity, ctypes.byref(n)))
+    return n.value
 
 
 def pt_gather_bench(ctx, buffer_bytes: int, record_bytes: int) -> float:
@@ -288,6 +304,19 @@ class Tracker:
         if paths:
             bufs.paths = alloc("paths", (n, stride, 3), np.float32, torch.float32)
         pt_get_paths(self.ctx, bufs)
+        return out
+
+    def load_targets(self, labels, ntargets: int) -> None:
+        """Target regions for the seed x target matrix (uint8 [Z][Y][X], 0 = none, t+1)."""
+        labels = _contig(labels)
+        self._stream()
+        pt_load_targets(self.ctx, _ptr(labels), ntargets)
+
+    def connectivity(self) -> np.ndarray:
+        """Seed x target matrix (uint32 [nseeds][ntargets]) of the last PT_REC_CONN track."""
+        n = pt_get_connectivity(self.ctx, None, 0)
+        out = np.empty(n, np.uint32)
+        pt_get_connectivity(self.ctx, out.ctypes.data, n)
         return out
 
     def gather_bench(self, buffer_bytes: int, record_bytes: int) -> float:

@@ -58,6 +58,12 @@ struct pt_ctx {
     float* d_paths = nullptr;
     size_t paths_cap = 0;
     unsigned long long* d_stats = nullptr;
+    uint8_t* d_labels = nullptr;   // NEXT-2 target labels [V]
+    size_t labels_cap = 0;
+    int32_t ntargets = 0;
+    uint32_t* d_conn = nullptr;    // NEXT-2 seed x target matrix of the last call
+    size_t conn_cap = 0;
+    uint64_t last_conn_count = 0;
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
     // last call
     bool tracked = false;
@@ -195,7 +201,7 @@ void pt_destroy(pt_ctx* c) {
     DeviceGuard g(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
     else cudaDeviceSynchronize();
-    void* bufs[] = {c->d_rec, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_copies, c->d_nsteps,
+    void* bufs[] = {c->d_rec, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_copies, c->d_labels, c->d_conn, c->d_nsteps,
                     c->d_reason, c->d_end, c->d_paths, c->d_stats};
     for (void* b : bufs)
         if (b) cudaFree(b);
@@ -293,6 +299,7 @@ pt_status pt_load_samples(pt_ctx* c, const pt_volume* v, const void* dyads, cons
     c->rec_bytes = rb;
     c->loaded = true;
     c->tracked = false;
+    c->ntargets = 0;  // targets belong to a volume shape
     return PT_OK;
 }
 
@@ -387,6 +394,14 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         d_order = c->d_order + 3 * N;
     }
 
+    const bool want_conn = (fl & PT_REC_CONN) != 0;
+    if (want_conn && (c->ntargets <= 0 || !c->d_labels))
+        return fail(c, PT_ERR_STATE, "pt_track: PT_REC_CONN needs targets (pt_load_targets)");
+    if (want_conn) {
+        CK(ensure(c->d_conn, c->conn_cap, N * (uint64_t)c->ntargets), "pt_track: connectivity buffer");
+        if (N) CK(cudaMemsetAsync(c->d_conn, 0, N * (uint64_t)c->ntargets * sizeof(uint32_t), st), "pt_track: connectivity zero");
+    }
+
     pt::TrackArgs a{};
     a.rec = c->d_rec;
     a.nx = nxv;
@@ -450,6 +465,9 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.o_paths = (fl & PT_REC_PATHS) ? c->d_paths : nullptr;
     a.path_stride = (fl & PT_REC_PATHS) ? p->path_stride : 0;
     a.stats = c->d_stats;
+    a.labels = want_conn ? c->d_labels : nullptr;
+    a.ntargets = want_conn ? (uint32_t)c->ntargets : 0u;
+    a.conn = want_conn ? c->d_conn : nullptr;
 
     CK(cudaEventRecord(c->ev[1], st), "pt_track: event");
     CK(pt::launch_track(a, c->vol.nfibres, c->vol.dtype == PT_F16, (fl & PT_KERNEL_SIMPLE) != 0, c->num_sms, st),
@@ -469,6 +487,42 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     c->last_flags = fl;
     c->last_stride = (fl & PT_REC_PATHS) ? p->path_stride : 0;
     c->last_map = d_map != nullptr;
+    c->last_conn_count = want_conn ? N * (uint64_t)c->ntargets : 0;
+    return PT_OK;
+}
+
+pt_status pt_load_targets(pt_ctx* c, const uint8_t* labels, int32_t ntargets) {
+    if (!c) return PT_ERR_ARG;
+    c->err.clear();
+    if (!c->loaded) return fail(c, PT_ERR_STATE, "pt_load_targets: load the sample volume first");
+    if (ntargets < 0 || ntargets > 64) return fail(c, PT_ERR_ARG, "pt_load_targets: ntargets must be in [0, 64]");
+    if (!labels || ntargets == 0) {
+        c->ntargets = 0;
+        return PT_OK;
+    }
+    DeviceGuard g(c->device);
+    const size_t V = (size_t)c->vol.nx * c->vol.ny * c->vol.nz;
+    CK(ensure(c->d_labels, c->labels_cap, V), "pt_load_targets: label buffer");
+    CK(cudaMemcpyAsync(c->d_labels, labels, V, cudaMemcpyDefault, c->stream), "pt_load_targets: copy");
+    CK(cudaStreamSynchronize(c->stream), "pt_load_targets: synchronise");
+    c->ntargets = ntargets;
+    return PT_OK;
+}
+
+pt_status pt_get_connectivity(pt_ctx* c, uint32_t* out, int64_t capacity, int64_t* count) {
+    if (!c) return PT_ERR_ARG;
+    c->err.clear();
+    if (!c->tracked || c->last_conn_count == 0)
+        return fail(c, PT_ERR_STATE, "pt_get_connectivity: the last pt_track did not record PT_REC_CONN");
+    if (count) *count = (int64_t)c->last_conn_count;
+    if (!out) return PT_OK;
+    if (capacity < (int64_t)c->last_conn_count)
+        return fail(c, PT_ERR_ARG, "pt_get_connectivity: capacity %lld < %llu", (long long)capacity,
+                    (unsigned long long)c->last_conn_count);
+    DeviceGuard g(c->device);
+    CK(cudaMemcpyAsync(out, c->d_conn, c->last_conn_count * sizeof(uint32_t), cudaMemcpyDefault, c->stream),
+       "pt_get_connectivity: copy");
+    CK(cudaStreamSynchronize(c->stream), "pt_get_connectivity: synchronise");
     return PT_OK;
 }
 

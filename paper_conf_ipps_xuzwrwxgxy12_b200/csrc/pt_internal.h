@@ -63,6 +63,9 @@ struct TrackArgs {
     uint8_t* o_reason;
     float* o_end;                // [nparticles][3]
     float* o_paths;              // [nparticles][path_stride][3]
+    const uint8_t* labels;       // [V] target labels (0 none, t+1) or nullptr
+    uint32_t ntargets;
+    uint32_t* conn;              // [nseeds][ntargets] seed x target matrix or nullptr
     int path_stride;
     unsigned long long* stats;   // [kNumStats]
 };

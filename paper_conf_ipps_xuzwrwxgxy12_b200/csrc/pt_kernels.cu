@@ -107,6 +107,8 @@ struct Slot {
     int why;           // >= 0: ended with this reason, outputs pending (finish)
     uint4 W;           // Philox block of the current round
     Rec<F, HALF> rv;   // record of the current step
+    uint64_t tmask;    // NEXT-2: targets entered by the path so far (bit t-1)
+    uint32_t sidx;     // NEXT-2: seed index of this call
 };
 
 template <bool REFILL, int SLOTS>
@@ -157,6 +159,8 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
         P[sl].sfix = 0u;
         P[sl].why = -1;
         P[sl].W = make_uint4(0u, 0u, 0u, 0u);
+        P[sl].tmask = 0ull;
+        P[sl].sidx = 0u;
 #pragma unroll
         for (int k = 0; k < R::kWords; ++k) P[sl].rv.w[k] = 0u;
     }
@@ -186,6 +190,15 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
         }
         if (has_map && x.run_cnt) atomicAdd(map + x.run_vox, x.run_cnt);  // RED
         x.run_cnt = 0;
+        if (OUT && a.conn) {  // NEXT-2: one count per target the streamline entered
+            uint64_t m = x.tmask;
+            while (m) {
+                const int t = __ffsll((long long)m) - 1;
+                atomicAdd(a.conn + (uint64_t)x.sidx * a.ntargets + (uint32_t)t, 1u);
+                m &= m - 1ull;
+            }
+            x.tmask = 0ull;
+        }
         my_steps += (uint32_t)x.n;
         my_particles += 1u;
         x.why = -1;
@@ -204,6 +217,10 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
             x.run_cnt = c ? (change ? 1u : x.run_cnt + 1u) : x.run_cnt;
             x.run_vox = c ? v : x.run_vox;
         }
+        if (OUT && a.conn && c) {  // NEXT-2: targets entered by committed steps (R21)
+            const uint32_t lbl = __ldg(a.labels + v);
+            x.tmask |= lbl ? (1ull << (lbl - 1u)) : 0ull;
+        }
         if (OUT && a.o_paths && c && x.n < a.path_stride) {
             float* pp = a.o_paths + (s_li[sl * TPB + threadIdx.x] * (uint64_t)a.path_stride + (uint64_t)x.n) * 3u;
             pp[0] = __fadd_rn(x.qx, a.fcx);
@@ -218,6 +235,8 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
         const uint64_t sid = a.seed_ids ? a.seed_ids[si] : si;
         x.pid = sid * a.P + j;
         x.sfix = (uint32_t)(j % a.S);
+        x.tmask = 0ull;
+        x.sidx = (uint32_t)si;
         x.qx = __fsub_rn(a.seeds[3 * si + 0], a.fcx);
         x.qy = __fsub_rn(a.seeds[3 * si + 1], a.fcy);
         x.qz = __fsub_rn(a.seeds[3 * si + 2], a.fcz);
@@ -581,7 +600,7 @@ static cudaError_t launch_t(const TrackArgs& a, int num_sms, cudaStream_t st) {
 
 template <int F, bool HALF>
 static cudaError_t launch_f(const TrackArgs& a, bool simple, int num_sms, cudaStream_t st) {
-    const bool out = a.o_nsteps || a.o_reason || a.o_end || a.o_paths;
+    const bool out = a.o_nsteps || a.o_reason || a.o_end || a.o_paths || a.conn;
     if (simple) return out ? launch_t<F, HALF, false, true>(a, num_sms, st) : launch_t<F, HALF, false, false>(a, num_sms, st);
     return out ? launch_t<F, HALF, true, true>(a, num_sms, st) : launch_t<F, HALF, true, false>(a, num_sms, st);
 }

@@ -310,3 +310,59 @@ def test_paper_mode_parity(pt, tracker, half):
     assert paths_equal(g["paths"], r["paths"])
     s = gpu_run(tracker, w, REC_ALL | pt.PT_KERNEL_SIMPLE)
     assert_parity(s, r)
+
+
+# ----------------------------------------------------------------------------- NEXT-2 connectivity
+
+def _targets(shape, n, seed):
+    """n roughly spherical target regions at random positions (labels 1..n)."""
+    rng = np.random.default_rng(seed)
+    Z, Y, X = shape
+    zz, yy, xx = np.meshgrid(np.arange(Z), np.arange(Y), np.arange(X), indexing="ij")
+    lab = np.zeros(shape, np.uint8)
+    for t in range(n):
+        c = rng.uniform([0, 0, 0], [Z, Y, X])
+        r = rng.uniform(2.0, 6.0)
+        lab[(zz - c[0]) ** 2 + (yy - c[1]) ** 2 + (xx - c[2]) ** 2 < r * r] = t + 1
+    return lab
+
+
+@pytest.mark.parametrize("simple", [False, True])
+@pytest.mark.parametrize("mode", [0, 1])
+def test_connectivity_parity(pt, tracker, simple, mode):
+    """NEXT-2: seed x target matrix bit-exact vs the oracle, both kernels, random
+    per-step sampling and paper mode."""
+    import torch
+    w = phantom.crossing(sigma=0.15, f_jitter=0.03, nseeds=200, particles_per_seed=300).replace(sample_mode=mode)
+    lab = _targets(w.volume.mask.shape, 64, seed=7)
+    tracker.load_volume(w.volume)
+    tracker.load_targets(lab, 64)
+    flags = REC_ALL | pt.PT_REC_CONN | (pt.PT_KERNEL_SIMPLE if simple else 0)
+    m = tracker.track_workload(w, flags=flags)
+    torch.cuda.synchronize()
+    g = tracker.get_paths()
+    g["map"] = m.cpu().numpy().view(np.uint32)
+    conn = tracker.connectivity().reshape(w.nseeds, 64)
+    r = oracle.track(w, labels=lab, ntargets=64, threads=_threads())
+    assert_parity(g, r)
+    assert np.array_equal(conn.astype(np.uint64), r["conn"])
+    assert conn.sum() > 1000
+
+
+def test_connectivity_brain_and_errors(pt, tracker):
+    w = phantom.whole_brain(nx=40, ny=36, nz=24, semi=(17.0, 15.0, 10.0), nsamples=16, nfibres=3,
+                            particles_per_seed=37)
+    w = phantom.wm_seeds(w, every=max(1, w.nseeds // 200))
+    lab = _targets(w.volume.mask.shape, 12, seed=3)
+    tracker.load_volume(w.volume)
+    with pytest.raises(pt.PtError) as e:
+        tracker.track_workload(w, flags=pt.PT_REC_CONN)
+    assert e.value.status == pt.PT_ERR_STATE
+    with pytest.raises(pt.PtError) as e:
+        tracker.load_targets(lab, 65)
+    assert e.value.status == pt.PT_ERR_ARG
+    tracker.load_targets(lab, 12)
+    tracker.track_workload(w, flags=pt.PT_REC_CONN)
+    conn = tracker.connectivity().reshape(w.nseeds, 12)
+    r = oracle.track(w, labels=lab, ntargets=12, want_particles=False)
+    assert np.array_equal(conn.astype(np.uint64), r["conn"])

@@ -496,3 +496,56 @@ def test_paper_mode_bruteforce(half):
         assert np.array_equal(r["paths"][i, :k].view(np.uint32), pos[:k].view(np.uint32)), i
     with pytest.raises(ValueError):
         oracle.track(w.replace(sample_mode=2))
+
+
+# ----------------------------------------------------------------------------- NEXT-2 connectivity
+
+def test_connectivity_tube_closed_form():
+    """NEXT-2 (count the streamlines passing through B): tube with two target slabs.
+    A particle counts once for a target iff its exact rational path (committed steps, R21)
+    enters a voxel of the slab, however many steps it spends there."""
+    w = phantom.tube(particles_per_seed=50, seed_x=16)
+    nx = w.volume.nx
+    lab = np.zeros_like(w.volume.mask)
+    lab[:, :, 24:26] = 1      # ahead in +x
+    lab[:, :, 3:5] = 2        # behind
+    lab[:, :, 16] = 3         # the seed voxel column
+    r = oracle.track(w, labels=lab, ntargets=3)
+    sg = _signs(w)
+    expect = np.zeros((w.nseeds, 3), np.uint64)
+    for i in range(w.nparticles):
+        s = i // w.particles_per_seed
+        path = _exact_path(nx, 16, int(sg[i]), int(r["nsteps"][i]))
+        hit = {1: any(24 <= v <= 25 for v in path), 2: any(3 <= v <= 4 for v in path),
+               3: any(v == 16 for v in path)}
+        for t in (1, 2, 3):
+            expect[s, t - 1] += hit[t]
+    assert np.array_equal(r["conn"], expect)
+    # every forward particle passes target 1, every backward one target 2; target 3 (the
+    # seed voxel) is entered again only by backward particles (q = +0 lands in voxel c)
+    fwd = (sg > 0).reshape(w.nseeds, -1).sum(1)
+    assert np.array_equal(r["conn"][:, 0], fwd) and np.array_equal(r["conn"][:, 1], 50 - fwd)
+    assert np.array_equal(r["conn"][:, 2], 50 - fwd)
+
+
+def test_connectivity_matches_bruteforce_paths():
+    """NEXT-2 on a dispersed brain: the oracle's matrix equals one computed from the numpy
+    brute-force tracker's positions and the label volume."""
+    w = phantom.whole_brain(nx=16, ny=14, nz=10, semi=(7.0, 6.0, 4.0), nsamples=6, nfibres=2,
+                            particles_per_seed=8, seeds="brain")
+    w = phantom.wm_seeds(w, every=max(1, w.nseeds // 10)).replace(curv_thr=0.3)
+    rng = np.random.default_rng(4)
+    lab = (rng.integers(0, 5, w.volume.mask.shape) * (rng.random(w.volume.mask.shape) < 0.3)).astype(np.uint8)
+    r = oracle.track(w, labels=lab, ntargets=4)
+    expect = np.zeros((w.nseeds, 4), np.uint64)
+    for i in range(w.nparticles):
+        n, why, pos = bruteforce.track(w, i // w.particles_per_seed, i % w.particles_per_seed)
+        got = set()
+        for x, y, z in pos[1:]:  # committed positions (R21)
+            vx = int(np.floor(x)); vy = int(np.floor(y)); vz = int(np.floor(z))
+            if lab[vz, vy, vx]:
+                got.add(int(lab[vz, vy, vx]))
+        for t in got:
+            expect[i // w.particles_per_seed, t - 1] += 1
+    assert np.array_equal(r["conn"], expect)
+    assert r["conn"].sum() > 0
