@@ -224,9 +224,17 @@ def run_ours(args):
     world = _env_int("WORLD_SIZE", 1)
     rank = _env_int("RANK", 0)
     local = _env_int("LOCAL_RANK", 0)
+    # BENCH_DIST_BACKEND=gloo + BENCH_SINGLE_DEVICE=1: test hook that runs the multi-rank
+    # path with every rank on cuda:0 (NCCL cannot put two ranks on one GPU)
+    backend = os.environ.get("BENCH_DIST_BACKEND", "nccl")
+    if os.environ.get("BENCH_SINGLE_DEVICE") == "1":
+        local = 0
     if world > 1:
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
 
@@ -289,10 +297,19 @@ def run_ours(args):
     my_steps = st["total_steps"]  # identical every step (deterministic)
     t = torch.tensor([ms, float(my_steps), float(mine.nseeds), float(st["lane_active"]),
                       float(st["lane_slots"])], dtype=torch.float64, device=dev)
+    def allreduce(x, op):
+        # gloo (test hook) reduces host tensors
+        if backend == "gloo" and x.is_cuda:
+            h = x.cpu()
+            dist.all_reduce(h, op=op)
+            x.copy_(h)
+        else:
+            dist.all_reduce(x, op=op)
+
     if world > 1:
         tmax = t.clone()
-        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
-        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        allreduce(tmax, dist.ReduceOp.MAX)
+        allreduce(t, dist.ReduceOp.SUM)
         ms = float(tmax[0])
     total_steps = float(t[1]) if world > 1 else float(my_steps)
     total_seeds = float(t[2]) if world > 1 else float(mine.nseeds)
@@ -325,7 +342,7 @@ def run_ours(args):
     e2e_s = time.perf_counter() - t0
     te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
     if world > 1:
-        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        allreduce(te, dist.ReduceOp.MAX)
     e2e_value = total_steps * e2e_steps / float(te[0])
 
     # ---- roofline (dominant kernel = the tracking kernel)

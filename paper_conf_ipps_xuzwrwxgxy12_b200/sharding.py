@@ -37,8 +37,14 @@ def reduce_map(map_i32, dst: int = 0, group=None, all_ranks: bool = False):
         raise TypeError("the map must be an int32 view of the uint32 counts")
     if not dist.is_available() or not dist.is_initialized() or dist.get_world_size(group) == 1:
         return map_i32
+    t = map_i32
+    staged = map_i32.is_cuda and dist.get_backend(group) == "gloo"  # gloo: host tensors only
+    if staged:
+        t = map_i32.cpu()
     if all_ranks:
-        dist.all_reduce(map_i32, op=dist.ReduceOp.SUM, group=group)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
     else:
-        dist.reduce(map_i32, dst=dst, op=dist.ReduceOp.SUM, group=group)
+        dist.reduce(t, dst=dst, op=dist.ReduceOp.SUM, group=group)
+    if staged:
+        map_i32.copy_(t)
     return map_i32
