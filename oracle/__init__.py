@@ -48,7 +48,8 @@ class _Params(ctypes.Structure):
     _fields_ = [("step", ctypes.c_float), ("curv_thr", ctypes.c_float),
                 ("fib_thr", ctypes.c_float), ("max_steps", ctypes.c_int32),
                 ("rng_seed", ctypes.c_uint64), ("particles_per_seed", ctypes.c_int64),
-                ("sample_mode", ctypes.c_int32)]
+                ("sample_mode", ctypes.c_int32), ("bidir", ctypes.c_int32),
+                ("interp", ctypes.c_int32), ("init_fibre", ctypes.c_int32)]
 
 
 _lib = None
@@ -108,11 +109,13 @@ def sample_index(w: int, nsamples: int) -> int:
 
 # ----------------------------------------------------------------------------- tracking
 
-def _structs(volume, step, curv_thr, fib_thr, max_steps, rng_seed, P, sample_mode=0):
+def _structs(volume, step, curv_thr, fib_thr, max_steps, rng_seed, P, sample_mode=0, bidir=0,
+             interp=0, init_fibre=0):
     v = volume
     vs = _Volume(v.nx, v.ny, v.nz, v.nsamples, v.nfibres, 1 if v.dyads.dtype == np.float16 else 0,
                  v.dyads.ctypes.data, v.f.ctypes.data, v.mask.ctypes.data)
-    ps = _Params(step, curv_thr, fib_thr, max_steps, rng_seed, P, sample_mode)
+    ps = _Params(step, curv_thr, fib_thr, max_steps, rng_seed, P, sample_mode, bidir, interp,
+                 init_fibre)
     return vs, ps
 
 
@@ -123,7 +126,8 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
 
     Returns dict(map=uint64[Z][Y][X] or None, nsteps=int32[n], reason=uint8[n],
     end=float32[n][3], paths=float32[n][path_stride][3] or None, conn=uint64[nseeds][ntargets]
-    or None), particles ordered (seed index, j).  ``threads`` > 1 runs independent single-threaded oracle calls on
+    or None), particles ordered (seed index, j) -- with ``w.bidir`` two entries per particle
+    (seed index, j, half), n = 2 * nseeds * npp.  ``threads`` > 1 runs independent single-threaded oracle calls on
     disjoint seed shards (seed i -> worker i mod threads) and sums their maps.
     """
     v = w.volume
@@ -133,9 +137,12 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
     seeds = np.ascontiguousarray(w.seeds, np.float32)
     ids = np.ascontiguousarray(w.ids(), np.uint64)
     ns = seeds.shape[0]
-    n = ns * npp
+    bidir = int(getattr(w, "bidir", 0))
+    H = 2 if bidir else 1                          # entries per particle
+    n = ns * npp * H
     vs, ps = _structs(v, w.step, w.curv_thr, w.fib_thr, w.max_steps, w.rng_seed, P,
-                      int(getattr(w, "sample_mode", 0)))
+                      int(getattr(w, "sample_mode", 0)), bidir, int(getattr(w, "interp", 0)),
+                      int(getattr(w, "init_fibre", 0)))
     nsteps = np.zeros(n, np.int32) if want_particles else None
     reason = np.zeros(n, np.uint8) if want_particles else None
     end = np.zeros((n, 3), np.float32) if want_particles else None
@@ -149,7 +156,7 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
     def run(shard: np.ndarray, mp: Optional[np.ndarray]):
         sd = np.ascontiguousarray(seeds[shard])
         si = np.ascontiguousarray(ids[shard])
-        m = len(shard) * npp
+        m = len(shard) * npp * H
         ln = np.zeros(m, np.int32) if want_particles else None
         lr = np.zeros(m, np.uint8) if want_particles else None
         le = np.zeros((m, 3), np.float32) if want_particles else None
@@ -184,7 +191,7 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
             conn[shard] = lc
         if len(shard) == 0:
             continue
-        rows = (shard[:, None] * npp + np.arange(npp)[None, :]).ravel()
+        rows = (shard[:, None] * (npp * H) + np.arange(npp * H)[None, :]).ravel()
         if want_particles:
             nsteps[rows] = ln
             reason[rows] = lr

@@ -44,6 +44,17 @@ typedef struct {
      * 1: paper mode (NEXT-1): particle j of a seed follows sample volume j mod S for its
      *    whole path (Alg. 1: one sample volume per streamline). */
     int32_t sample_mode;
+    /* NEXT-3 FSL-fidelity variants (R22-R24); all 0 = the north star's contract.
+     * bidir: 1 = bidirectional streamlines (R22): half 0 is the one-directional particle,
+     *        half 1 restarts at the seed with previous direction -d0 (d0 = half 0's first
+     *        step direction) and draws from RNG stream 1.
+     * interp: 1 = probabilistic (trilinear) interpolation of the sampled voxel (R23,
+     *        "Interpolation()" P:L175), uniforms from RNG stream 2 + half.
+     * init_fibre: first-step fibre of half 0 (R24): 0 = fibre 0 (R5), 1 = uniform among
+     *        the eligible fibres, 2 = f-weighted among the eligible fibres. */
+    int32_t bidir;
+    int32_t interp;
+    int32_t init_fibre;
 } oracle_params;
 
 enum { ORACLE_END_MASK = 0, ORACLE_END_CURV = 1, ORACLE_END_MAXLEN = 2 };
@@ -63,12 +74,14 @@ uint32_t oracle_sample_index(uint32_t w, uint32_t nsamples);
  *   seeds_xyz [nseeds][3] corner coordinates; seed_ids [nseeds] (NULL => 0..nseeds-1)
  *   map       [Z][Y][X] uint64, accumulated (+=) ; may be NULL
  *   nsteps, reason, end_xyz: per particle, index (seed_index*(j_end-j_begin) + j-j_begin);
- *                            each may be NULL
+ *                            each may be NULL.  With bidir, per half: index 2*that + half.
  *   paths     [particle][path_stride][3] corner-coordinate positions, point 0 = start,
  *             point k = after the k-th committed step, unused points = NaN; may be NULL
+ *             (with bidir: [particle][2][path_stride][3], one polyline per half)
  *   labels    [Z][Y][X] target labels (0 = none, t+1 = target t) or NULL; ntargets <= 64
  *   conn      [nseeds][ntargets] uint64, accumulated: number of the seed's particles whose
  *             committed steps enter target t at least once (NEXT-2; R21); may be NULL
+ *             (with bidir a streamline is the union of its two halves)
  * Returns 0 on success, <0 on invalid arguments (nothing written). */
 int oracle_track(const oracle_volume* vol, const oracle_params* prm,
                  const float* seeds_xyz, const uint64_t* seed_ids, int64_t nseeds,

@@ -81,6 +81,10 @@ class Workload:
     particles_per_seed: int = 1000
     recipe: str = ""
     sample_mode: int = 0  # 0: random sample per step (R1); 1: paper mode, s = j mod S (NEXT-1)
+    # NEXT-3 FSL-fidelity variants (R22-R24)
+    bidir: int = 0        # 1: bidirectional streamlines (two halves per particle)
+    interp: int = 0       # 1: probabilistic interpolation of the sampled voxel
+    init_fibre: int = 0   # first-step fibre: 0 fibre 0, 1 uniform eligible, 2 f-weighted
 
     @property
     def nseeds(self) -> int:
