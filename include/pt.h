@@ -61,6 +61,22 @@ typedef enum { PT_END_MASK = 0, PT_END_CURV = 1, PT_END_MAXLEN = 2 } pt_reason;
                                         follows sample volume j mod S for its whole path
                                         (Alg. 1) instead of a fresh
                                         random sample every step (R1)                    */
+/* NEXT-3 FSL-fidelity variants (R22-R24; run by the variant kernel).        */
+#define PT_BIDIR          (1u << 11) /* bidirectional streamlines (R22): each particle runs
+                                        two halves from its seed; half 0 is the one-
+                                        directional particle, half 1 starts against half
+                                        0's first direction (RNG stream 1).  Per-particle
+                                        outputs hold 2 entries per particle (index 2*i+h);
+                                        the map counts both halves; a connectivity
+                                        streamline is the union of the halves            */
+#define PT_INTERP         (1u << 12) /* probabilistic (trilinear) interpolation of the
+                                        sampled voxel, "Interpolation()" P:L175 (R23)    */
+#define PT_INIT_RANDOM    (1u << 13) /* first fibre uniform over the eligible fibres (R24) */
+#define PT_INIT_FWEIGHT   (1u << 14) /* first fibre drawn with probability f_j / sum f over
+                                        the eligible fibres (R24); exclusive with
+                                        PT_INIT_RANDOM                                   */
+#define PT_KERNEL_VARIANT (1u << 15) /* run the variant kernel even with no variant flag
+                                        (same results as the main kernel; ablation/tests) */
 
 /* Create a context on CUDA device `cuda_device` (the caller's current device is left
  * unchanged).  *out receives the context or NULL.  The stream defaults to the legacy
@@ -106,7 +122,8 @@ typedef struct {
     uint64_t rng_seed;          /* Philox-4x32-10 key (R16)                               */
     int64_t particles_per_seed; /* P >= 1; particle j of seed id k has pid = k*P + j      */
     uint32_t flags;             /* PT_REC_* | PT_MAP_ACCUMULATE | PT_KERNEL_SIMPLE |
-                                   PT_SEED_ORDER_INPUT | PT_SAMPLE_PER_STREAMLINE         */
+                                   PT_SEED_ORDER_INPUT | PT_SAMPLE_PER_STREAMLINE |
+                                   PT_BIDIR | PT_INTERP | PT_INIT_* | PT_KERNEL_VARIANT   */
     int32_t path_stride;        /* points stored per particle with PT_REC_PATHS (>= 1)    */
 } pt_params;
 
@@ -123,7 +140,9 @@ typedef struct {
  * synchronous (device map, then a device-to-host copy).  Per-particle outputs selected
  * by flags stay on the device until pt_get_paths.  Errors: PT_ERR_STATE before
  * pt_load_samples; PT_ERR_ARG for parameter ranges, nseeds < 0 or pid overflow;
- * PT_ERR_OOM; PT_ERR_CUDA.  Map overflow is reported by pt_get_stats/pt_get_paths. */
+ * PT_ERR_OOM; PT_ERR_CUDA; PT_ERR_ARG for PT_KERNEL_SIMPLE combined with a NEXT-3
+ * variant flag or for PT_INIT_RANDOM | PT_INIT_FWEIGHT.  Map overflow is reported by
+ * pt_get_stats/pt_get_paths. */
 pt_status pt_track(pt_ctx* ctx, const float* seeds_xyz, const uint64_t* seed_ids,
                    int64_t nseeds, const pt_params* params, uint32_t* map);
 
@@ -144,7 +163,8 @@ pt_status pt_load_targets(pt_ctx* ctx, const uint8_t* labels, int32_t ntargets);
  * out = NULL).  Host or device out; synchronises ctx's stream. */
 pt_status pt_get_connectivity(pt_ctx* ctx, uint32_t* out, int64_t capacity, int64_t* count);
 
-/* Per-particle outputs of the last pt_track, particle index = seed_index*P + j.
+/* Per-particle outputs of the last pt_track, particle index = seed_index*P + j
+ * (with PT_BIDIR: entry 2*(seed_index*P + j) + half, count = 2 * nseeds * P).
  * Set capacity = number of particles the buffers hold; NULL buffers are skipped;
  * count receives the number of particles of the last pt_track (query with all buffers
  * NULL).  nsteps [count] uint16; reason [count] uint8; end_xyz [count][3] float32

@@ -25,7 +25,8 @@ __all__ = [
     "pt_load_samples", "pt_track", "pt_get_paths", "pt_get_stats", "pt_gather_bench",
     "pt_record_bytes", "PT_F32", "PT_F16", "PT_REC_LEN", "PT_REC_REASON", "PT_REC_END",
     "PT_REC_PATHS", "PT_MAP_ACCUMULATE", "PT_KERNEL_SIMPLE", "PT_SEED_ORDER_INPUT",
-    "PT_SAMPLE_PER_STREAMLINE", "PT_REC_CONN", "pt_load_targets", "pt_get_connectivity", "PT_END_MASK", "PT_END_CURV",
+    "PT_SAMPLE_PER_STREAMLINE", "PT_REC_CONN", "PT_BIDIR", "PT_INTERP", "PT_INIT_RANDOM",
+    "PT_INIT_FWEIGHT", "PT_KERNEL_VARIANT", "variant_flags", "pt_load_targets", "pt_get_connectivity", "PT_END_MASK", "PT_END_CURV",
     "PT_END_MAXLEN", "EXPORTS",
 ]
 
@@ -41,6 +42,17 @@ PT_REC_CONN = 1 << 5
 PT_KERNEL_SIMPLE = 1 << 8
 PT_SEED_ORDER_INPUT = 1 << 9
 PT_SAMPLE_PER_STREAMLINE = 1 << 10
+PT_BIDIR = 1 << 11
+PT_INTERP = 1 << 12
+PT_INIT_RANDOM = 1 << 13
+PT_INIT_FWEIGHT = 1 << 14
+PT_KERNEL_VARIANT = 1 << 15
+
+
+def variant_flags(bidir: int = 0, interp: int = 0, init_fibre: int = 0) -> int:
+    """pt_params.flags bits of the NEXT-3 variants (R22-R24)."""
+    return ((PT_BIDIR if bidir else 0) | (PT_INTERP if interp else 0) |
+            {0: 0, 1: PT_INIT_RANDOM, 2: PT_INIT_FWEIGHT}[int(init_fibre)])
 
 # every symbol include/pt.h declares
 EXPORTS = ["pt_create", "pt_destroy", "pt_last_error", "pt_set_stream", "pt_load_samples",
@@ -269,6 +281,8 @@ class Tracker:
                        out_map=None, want_map: bool = True):
         if getattr(w, "sample_mode", 0) == 1:
             flags |= PT_SAMPLE_PER_STREAMLINE
+        flags |= variant_flags(getattr(w, "bidir", 0), getattr(w, "interp", 0),
+                               getattr(w, "init_fibre", 0))
         seeds = w.seeds if seeds is None else seeds
         if seed_ids is None and w.seed_ids is not None:
             seed_ids = w.seed_ids

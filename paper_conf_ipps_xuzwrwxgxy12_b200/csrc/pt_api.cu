@@ -36,6 +36,8 @@ struct pt_ctx {
     int rec_bytes = 0;
     uint8_t* d_rec = nullptr;
     size_t rec_size = 0;
+    uint8_t* d_mask = nullptr;    // tracking mask copy (the variant kernel's interpolation)
+    size_t mask_cap = 0;
     // per-call buffers
     float* d_seeds = nullptr;
     size_t seeds_cap = 0;
@@ -201,7 +203,7 @@ void pt_destroy(pt_ctx* c) {
     DeviceGuard g(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
     else cudaDeviceSynchronize();
-    void* bufs[] = {c->d_rec, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_copies, c->d_labels, c->d_conn, c->d_nsteps,
+    void* bufs[] = {c->d_rec, c->d_mask, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_copies, c->d_labels, c->d_conn, c->d_nsteps,
                     c->d_reason, c->d_end, c->d_paths, c->d_stats};
     for (void* b : bufs)
         if (b) cudaFree(b);
@@ -284,7 +286,9 @@ pt_status pt_load_samples(pt_ctx* c, const pt_volume* v, const void* dyads, cons
         c->rec_size = rec_size;
     }
     c->loaded = false;
-    cudaError_t e = cudaMemsetAsync(c->d_stats + pt::kStatBadInput, 0, sizeof(unsigned long long), c->stream);
+    cudaError_t e = ensure(c->d_mask, c->mask_cap, (size_t)V);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(c->d_mask, d_m, (size_t)V, cudaMemcpyDeviceToDevice, c->stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(c->d_stats + pt::kStatBadInput, 0, sizeof(unsigned long long), c->stream);
     if (e == cudaSuccess)
         e = pt::launch_repack(d_dy, d_f, d_m, c->d_rec, (int64_t)V, v->nsamples, v->nfibres,
                               v->dtype == PT_F16, rb, c->d_stats + pt::kStatBadInput, c->stream);
@@ -324,6 +328,15 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     const uint64_t N = (uint64_t)nseeds;
     if (N && P > UINT64_MAX / N) return fail(c, PT_ERR_ARG, "pt_track: nseeds * P overflows");
     const uint64_t npart = N * P;
+    const uint32_t kVariantFlags = PT_BIDIR | PT_INTERP | PT_INIT_RANDOM | PT_INIT_FWEIGHT | PT_KERNEL_VARIANT;
+    const bool variant = (p->flags & kVariantFlags) != 0;
+    if (variant && (p->flags & PT_KERNEL_SIMPLE))
+        return fail(c, PT_ERR_ARG, "pt_track: PT_KERNEL_SIMPLE cannot run the NEXT-3 variants");
+    if ((p->flags & PT_INIT_RANDOM) && (p->flags & PT_INIT_FWEIGHT))
+        return fail(c, PT_ERR_ARG, "pt_track: PT_INIT_RANDOM and PT_INIT_FWEIGHT are exclusive");
+    const uint64_t H = (p->flags & PT_BIDIR) ? 2 : 1;   // output entries per particle
+    if (npart > UINT64_MAX / 2) return fail(c, PT_ERR_ARG, "pt_track: too many particles");
+    const uint64_t nout = npart * H;
     DeviceGuard g(c->device);
     if (!g.ok) return fail(c, PT_ERR_CUDA, "pt_track: cannot select device %d", c->device);
     cudaStream_t st = c->stream;
@@ -365,12 +378,12 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
 
     // outputs
     const uint32_t fl = p->flags;
-    if (fl & PT_REC_LEN) CK(ensure(c->d_nsteps, c->nsteps_cap, npart), "pt_track: nsteps buffer");
-    if (fl & PT_REC_REASON) CK(ensure(c->d_reason, c->reason_cap, npart), "pt_track: reason buffer");
-    if (fl & PT_REC_END) CK(ensure(c->d_end, c->end_cap, 3 * npart), "pt_track: end buffer");
+    if (fl & PT_REC_LEN) CK(ensure(c->d_nsteps, c->nsteps_cap, nout), "pt_track: nsteps buffer");
+    if (fl & PT_REC_REASON) CK(ensure(c->d_reason, c->reason_cap, nout), "pt_track: reason buffer");
+    if (fl & PT_REC_END) CK(ensure(c->d_end, c->end_cap, 3 * nout), "pt_track: end buffer");
     if (fl & PT_REC_PATHS) {
-        CK(ensure(c->d_paths, c->paths_cap, 3 * npart * (uint64_t)p->path_stride), "pt_track: path buffer");
-        CK(cudaMemsetAsync(c->d_paths, 0xFF, 3 * npart * (uint64_t)p->path_stride * sizeof(float), st), "pt_track: path fill");
+        CK(ensure(c->d_paths, c->paths_cap, 3 * nout * (uint64_t)p->path_stride), "pt_track: path buffer");
+        CK(cudaMemsetAsync(c->d_paths, 0xFF, 3 * nout * (uint64_t)p->path_stride * sizeof(float), st), "pt_track: path fill");
     }
 
     CK(cudaEventRecord(c->ev[0], st), "pt_track: event");
@@ -451,7 +464,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.map = d_map;
     a.map_copies = 1;
     const bool simple = (fl & PT_KERNEL_SIMPLE) != 0;
-    uint32_t copies = (d_map && !simple && npart > 0) ? (uint32_t)PT_MAP_COPIES : 1u;
+    uint32_t copies = (d_map && !simple && !variant && npart > 0) ? (uint32_t)PT_MAP_COPIES : 1u;
     if (copies > (uint32_t)c->num_sms) copies = (uint32_t)c->num_sms;
     if (copies > 1) {
         CK(ensure(c->d_copies, c->copies_cap, (size_t)copies * V), "pt_track: map copies");
@@ -468,10 +481,18 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.labels = want_conn ? c->d_labels : nullptr;
     a.ntargets = want_conn ? (uint32_t)c->ntargets : 0u;
     a.conn = want_conn ? c->d_conn : nullptr;
+    a.bidir = (fl & PT_BIDIR) ? 1u : 0u;
+    a.interp = (fl & PT_INTERP) ? 1u : 0u;
+    a.init_mode = (fl & PT_INIT_RANDOM) ? 1u : ((fl & PT_INIT_FWEIGHT) ? 2u : 0u);
+    a.mask = c->d_mask;
 
     CK(cudaEventRecord(c->ev[1], st), "pt_track: event");
-    CK(pt::launch_track(a, c->vol.nfibres, c->vol.dtype == PT_F16, (fl & PT_KERNEL_SIMPLE) != 0, c->num_sms, st),
-       "pt_track: tracking kernel launch");
+    if (variant)
+        CK(pt::launch_track_var(a, c->vol.nfibres, c->vol.dtype == PT_F16, c->num_sms, st),
+           "pt_track: variant tracking kernel launch");
+    else
+        CK(pt::launch_track(a, c->vol.nfibres, c->vol.dtype == PT_F16, (fl & PT_KERNEL_SIMPLE) != 0, c->num_sms, st),
+           "pt_track: tracking kernel launch");
     CK(cudaEventRecord(c->ev[2], st), "pt_track: event");
     if (a.map_copies > 1)
         CK(pt::launch_map_combine(a.map, a.map_copies, (int64_t)V, d_map, true, st), "pt_track: map combine");
@@ -483,7 +504,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     if (host_map) CK(cudaStreamSynchronize(st), "pt_track: synchronise");
 
     c->tracked = true;
-    c->last_count = npart;
+    c->last_count = nout;
     c->last_flags = fl;
     c->last_stride = (fl & PT_REC_PATHS) ? p->path_stride : 0;
     c->last_map = d_map != nullptr;

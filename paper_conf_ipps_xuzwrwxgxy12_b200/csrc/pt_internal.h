@@ -20,6 +20,10 @@ constexpr int kThreads = PT_CTA_THREADS;
 #endif
 constexpr int kThreads2 = PT_CTA_THREADS2;  // CTA size of the 2-slot kernel (<= 85 registers)
 constexpr int kSimpleThreads = 256;  // no-refill ablation kernel
+#ifndef PT_VAR_THREADS
+#define PT_VAR_THREADS 768
+#endif
+constexpr int kVarThreads = PT_VAR_THREADS;  // NEXT-3 variant kernel (one CTA per SM)
 constexpr uint32_t kSub = 32;
 constexpr uint32_t kMinCtaChunk = 1024;
 
@@ -68,11 +72,19 @@ struct TrackArgs {
     uint32_t* conn;              // [nseeds][ntargets] seed x target matrix or nullptr
     int path_stride;
     unsigned long long* stats;   // [kNumStats]
+    // NEXT-3 variants (track_var_kernel only; R22-R24)
+    uint32_t bidir;              // 1: two halves per particle, outputs at 2*i + half
+    uint32_t interp;             // 1: probabilistic interpolation of the sampled voxel
+    uint32_t init_mode;          // first fibre: 0 fibre 0, 1 uniform eligible, 2 f-weighted
+    const uint8_t* mask;         // [V] tracking mask (interp: candidate test) or nullptr
 };
 
 // Launchers (return the launch error, if any).
 cudaError_t launch_track(const TrackArgs& a, int nfibres, bool half, bool simple, int num_sms,
                          cudaStream_t st);
+// NEXT-3 variant kernel (bidirectional / interpolation / first-fibre modes; also runs the
+// default semantics when forced with PT_KERNEL_VARIANT).
+cudaError_t launch_track_var(const TrackArgs& a, int nfibres, bool half, int num_sms, cudaStream_t st);
 cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask, uint8_t* rec,
                           int64_t V, int S, int F, bool half, int rec_bytes,
                           unsigned long long* bad, cudaStream_t st);
