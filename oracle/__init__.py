@@ -18,6 +18,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "oracle.c")
+_SRC_MCMC = os.path.join(_HERE, "oracle_mcmc.c")
 _HDR = os.path.join(_HERE, "oracle.h")
 _LIB = os.path.join(_HERE, "liboracle.so")
 CFLAGS = ["-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared",
@@ -28,11 +29,12 @@ END_MASK, END_CURV, END_MAXLEN = 0, 1, 2
 
 def build(force: bool = False) -> str:
     """Compile liboracle.so with gcc (no FMA contraction, no fast-math)."""
+    srcs = [_SRC, _SRC_MCMC]
     stale = (not os.path.exists(_LIB) or
-             os.path.getmtime(_LIB) < max(os.path.getmtime(_SRC), os.path.getmtime(_HDR)))
+             os.path.getmtime(_LIB) < max(os.path.getmtime(f) for f in srcs + [_HDR]))
     if force or stale:
         tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, _SRC, "-lm"])
+        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, *srcs, "-lm"])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -50,6 +52,19 @@ class _Params(ctypes.Structure):
                 ("rng_seed", ctypes.c_uint64), ("particles_per_seed", ctypes.c_int64),
                 ("sample_mode", ctypes.c_int32), ("bidir", ctypes.c_int32),
                 ("interp", ctypes.c_int32), ("init_fibre", ctypes.c_int32)]
+
+
+class _Dwi(ctypes.Structure):
+    _fields_ = [("nx", ctypes.c_int32), ("ny", ctypes.c_int32), ("nz", ctypes.c_int32),
+                ("nmeas", ctypes.c_int32), ("dwi", ctypes.c_void_p), ("bvals", ctypes.c_void_p),
+                ("bvecs", ctypes.c_void_p), ("mask", ctypes.c_void_p)]
+
+
+class _McmcParams(ctypes.Structure):
+    _fields_ = [("nfibres", ctypes.c_int32), ("burnin", ctypes.c_int32),
+                ("nsamples", ctypes.c_int32), ("interval", ctypes.c_int32),
+                ("adapt_every", ctypes.c_int32), ("rng_seed", ctypes.c_uint64),
+                ("fixed", ctypes.c_uint32)]
 
 
 _lib = None
@@ -74,6 +89,14 @@ def lib():
                                        ctypes.c_int64, ctypes.c_int64, ctypes.c_int64,
                                        vp, vp, vp, vp, vp, ctypes.c_int32, vp, ctypes.c_int32, vp]
             L.oracle_track.restype = ctypes.c_int
+            L.oracle_mcmc_signal.argtypes = [ctypes.c_int, vp, ctypes.c_int, vp, vp, vp]
+            L.oracle_mcmc_signal.restype = None
+            L.oracle_mcmc_draw.argtypes = [ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
+                                           ctypes.c_uint32, vp, vp]
+            L.oracle_mcmc_draw.restype = None
+            L.oracle_mcmc.argtypes = [ctypes.POINTER(_Dwi), ctypes.POINTER(_McmcParams), vp,
+                                      ctypes.c_int64, ctypes.c_int64, vp, vp]
+            L.oracle_mcmc.restype = ctypes.c_int
             _lib = L
     return _lib
 
@@ -204,3 +227,76 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
         for m in maps[1:]:
             mp += m
     return dict(map=mp, nsteps=nsteps, reason=reason, end=end, paths=paths, conn=conn)
+
+
+# ----------------------------------------------------------------------------- NEXT-4 MCMC
+
+def mcmc_signal(nfibres: int, omega, bvals, bvecs) -> np.ndarray:
+    """Eq. 1 for one parameter vector (S0, d, sigma, f1, th1, ph1, ...)."""
+    om = np.ascontiguousarray(omega, np.float64)
+    b = np.ascontiguousarray(bvals, np.float32)
+    r = np.ascontiguousarray(bvecs, np.float32)
+    mu = np.zeros(b.size, np.float64)
+    lib().oracle_mcmc_signal(int(nfibres), om.ctypes.data, b.size, b.ctypes.data, r.ctypes.data,
+                             mu.ctypes.data)
+    return mu
+
+
+def mcmc_draw(seed: int, loop: int, voxel: int, k: int):
+    """(z, log u) of MH step (loop, voxel, k) (M6)."""
+    z = np.zeros(1, np.float64)
+    lu = np.zeros(1, np.float64)
+    lib().oracle_mcmc_draw(seed, loop, voxel, k, z.ctypes.data, lu.ctypes.data)
+    return float(z[0]), float(lu[0])
+
+
+def mcmc(d, *, init: Optional[np.ndarray] = None, fixed: int = 0, threads: int = 1,
+         voxels: Optional[np.ndarray] = None) -> dict:
+    """Run the MCMC oracle on a phantom.DwiWorkload ``d``.
+
+    Returns dict(samples=float64 [NP][S][Z][Y][X] (0 outside the sampled voxels),
+    accepted=uint32 [NP][Z][Y][X]).  ``voxels`` (sorted linear indices) restricts the run to
+    a subset of the mask; ``threads`` > 1 runs independent single-threaded oracle calls on
+    disjoint voxel ranges.
+    """
+    NP = 3 + 3 * int(d.nfibres)
+    V = d.nx * d.ny * d.nz
+    dwi = np.ascontiguousarray(d.dwi, np.float32)
+    bv = np.ascontiguousarray(d.bvals, np.float32)
+    bc = np.ascontiguousarray(d.bvecs, np.float32)
+    mask = np.ascontiguousarray(d.mask, np.uint8)
+    if voxels is not None:
+        sub = np.zeros(V, np.uint8)
+        sub[np.asarray(voxels, np.int64)] = 1
+        mask = (sub.reshape(mask.shape) & (mask != 0)).astype(np.uint8)
+    ds = _Dwi(d.nx, d.ny, d.nz, bv.size, dwi.ctypes.data, bv.ctypes.data, bc.ctypes.data,
+              mask.ctypes.data)
+    ps = _McmcParams(int(d.nfibres), int(d.burnin), int(d.nsamples), int(d.interval),
+                     int(d.adapt_every), int(d.rng_seed), int(fixed))
+    ini = None if init is None else np.ascontiguousarray(init, np.float64).reshape(NP, V)
+    samples = np.zeros((NP, int(d.nsamples), V), np.float64)
+    acc = np.zeros((NP, V), np.uint32)
+    L = lib()
+    flat = np.flatnonzero(mask.ravel())
+    threads = max(1, min(int(threads), max(1, flat.size)))
+    cuts = [0] + [int(flat[(flat.size * t) // threads]) for t in range(1, threads)] + [V]
+    errs = []
+
+    def run(t):
+        rc = L.oracle_mcmc(ctypes.byref(ds), ctypes.byref(ps), _ptr(ini), cuts[t], cuts[t + 1],
+                           samples.ctypes.data, acc.ctypes.data)
+        if rc != 0:
+            errs.append(rc)
+
+    if threads == 1:
+        run(0)
+    else:
+        th = [threading.Thread(target=run, args=(t,)) for t in range(threads)]
+        for t in th:
+            t.start()
+        for t in th:
+            t.join()
+    if errs:
+        raise ValueError(f"oracle_mcmc rejected its arguments (rc={errs[0]})")
+    return dict(samples=samples.reshape(NP, int(d.nsamples), d.nz, d.ny, d.nx),
+                accepted=acc.reshape(NP, d.nz, d.ny, d.nx))

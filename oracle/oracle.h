@@ -90,6 +90,45 @@ int oracle_track(const oracle_volume* vol, const oracle_params* prm,
                  float* paths, int32_t path_stride,
                  const uint8_t* labels, int32_t ntargets, uint64_t* conn);
 
+
+/* ---------------------------------------------------------------- NEXT-4: MCMC sampler
+ * (oracle_mcmc.c) Metropolis-Hastings sampling of Eq. 1, readings
+ * M1-M9 of DESIGN.md §12.  Parameters per voxel, in MH order:
+ *   omega = (S0, d, sigma, f_1, theta_1, phi_1, ..., f_N, theta_N, phi_N),  NP = 3 + 3N. */
+#define ORACLE_MCMC_MAX_MEAS 256
+
+typedef struct {
+    int32_t nx, ny, nz, nmeas;
+    const float* dwi;     /* [nmeas][nz][ny][nx] (x fastest, measurement slowest; Fig. 1) */
+    const float* bvals;   /* [nmeas] b-values (ms/um^2 units: b d ~ 1)                     */
+    const float* bvecs;   /* [nmeas][3] unit gradient directions                          */
+    const uint8_t* mask;  /* [nz][ny][nx] voxels to sample (!= 0)                          */
+} oracle_dwi;
+
+typedef struct {
+    int32_t nfibres;      /* N of Eq. 1, 1..3 (the paper: 2)                        */
+    int32_t burnin;       /* NumBurnIn (500 in the paper's example)                */
+    int32_t nsamples;     /* NumSamples (50)                                        */
+    int32_t interval;     /* L, the sample interval (2)                             */
+    int32_t adapt_every;  /* K loops between proposal updates (Fig. 2; M8)                 */
+    uint64_t rng_seed;    /* Philox key (M6)                                                */
+    uint32_t fixed;       /* bit k: parameter k keeps its initial value (M9)                */
+} oracle_mcmc_params;
+
+/* Eq. 1 for one parameter vector: mu[i], i < n. */
+void oracle_mcmc_signal(int nfibres, const double* omega, int n, const float* bvals,
+                        const float* bvecs, double* mu);
+/* The Gaussian and log-uniform of MH step (loop, voxel, k) (M6). */
+void oracle_mcmc_draw(uint64_t seed, uint32_t loop, uint32_t voxel, uint32_t k, double* z,
+                      double* logu);
+/* Sample the voxels v in [v_begin, v_end) with mask != 0.
+ *   init     [NP][V] initial states or NULL (automatic, M7)
+ *   samples  [NP][nsamples][V] (written for sampled voxels only)
+ *   accepted [NP][V] accepted proposals per parameter, or NULL
+ * Returns 0, or < 0 for invalid arguments. */
+int oracle_mcmc(const oracle_dwi* dw, const oracle_mcmc_params* p, const double* init,
+                int64_t v_begin, int64_t v_end, double* samples, uint32_t* accepted);
+
 #ifdef __cplusplus
 }
 #endif

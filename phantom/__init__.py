@@ -30,6 +30,7 @@ import numpy as np
 __all__ = [
     "Volume", "Workload", "tube", "crossing", "whole_brain", "isotropic", "bent_tube",
     "t_junction", "fork", "paper_dataset", "mirror_x", "to_half", "config", "CONFIGS", "wm_seeds",
+    "DwiWorkload", "gradient_scheme", "dwi_brain", "dwi_uniform", "MCMC_CONFIGS", "mcmc_config",
 ]
 
 
@@ -429,6 +430,165 @@ def paper_dataset(which: int = 1, step: float = 0.1, curv_thr: float = 0.9, gen_
                     step=step, curv_thr=curv_thr, max_steps=1888, gen_seed=gen_seed, seeds="brain")
     return w.replace(name=f"paper_d{which}_step{step}_thr{curv_thr}", sample_mode=1,
                      recipe=w.recipe + f"; paper mode D{which}, step {step}, dot threshold {curv_thr}")
+
+
+# ----------------------------------------------------------------------------- NEXT-4 DWI
+
+@dataclasses.dataclass
+class DwiWorkload:
+    """Synthetic diffusion-weighted data for the MCMC sampler (NEXT-4, Fig. 1: a 4-D
+    volume of n measurements, b-values and gradient directions) plus the sampler settings."""
+    name: str
+    nx: int
+    ny: int
+    nz: int
+    dwi: np.ndarray       # [n][Z][Y][X] float32
+    bvals: np.ndarray     # [n] float32 (ms/um^2: b = 1 is 1000 s/mm^2)
+    bvecs: np.ndarray     # [n][3] float32 unit vectors
+    mask: np.ndarray      # [Z][Y][X] uint8: voxels to sample ("valid (white matter)", P:L301)
+    truth: Optional[np.ndarray] = None  # [NP][Z][Y][X] float64 generating parameters
+    nfibres: int = 2      # N = 2 (P:L69)
+    burnin: int = 500     # NumBurnIn (P:L147)
+    nsamples: int = 50    # P:L301
+    interval: int = 2     # L (P:L301)
+    adapt_every: int = 50  # K (Fig. 2; reading M8)
+    rng_seed: int = 0x4D434D43_2012
+    recipe: str = ""
+
+    @property
+    def nmeas(self) -> int:
+        return int(self.bvals.size)
+
+    @property
+    def nvoxels(self) -> int:
+        return int((self.mask != 0).sum())
+
+    @property
+    def nparams(self) -> int:
+        return 3 + 3 * self.nfibres
+
+    @property
+    def loops(self) -> int:
+        return self.burnin + self.nsamples * self.interval
+
+    def replace(self, **kw) -> "DwiWorkload":
+        return dataclasses.replace(self, **kw)
+
+
+def gradient_scheme(ndirs: int = 60, nb0: int = 4, b: float = 1.0):
+    """nb0 b = 0 measurements followed by ndirs directions on the upper hemisphere
+    (Fibonacci lattice), all at b.  Returns (bvals [n] float32, bvecs [n][3] float32)."""
+    k = np.arange(ndirs, dtype=np.float64) + 0.5
+    z = 1.0 - k / ndirs                       # (0, 1]: upper hemisphere
+    phi = k * math.pi * (3.0 - math.sqrt(5.0))
+    rr = np.sqrt(1.0 - z * z)
+    dirs = np.stack([rr * np.cos(phi), rr * np.sin(phi), z], 1)
+    bvecs = np.concatenate([np.tile([[1.0, 0.0, 0.0]], (nb0, 1)), dirs], 0).astype(np.float32)
+    bvals = np.concatenate([np.zeros(nb0), np.full(ndirs, b)]).astype(np.float32)
+    return bvals, bvecs
+
+
+def _forward(S0, d, f, v, bvals, bvecs):
+    """Synthetic scanner: the multiple partial volume model of Eq. 1, numpy
+    float64 over voxels.  S0, d: [m]; f: [N][m]; v: [N][m][3]; returns [n][m]."""
+    b = bvals.astype(np.float64)[:, None]
+    r = bvecs.astype(np.float64)
+    att = (1.0 - f.sum(0))[None, :] * np.exp(-b * d[None, :])
+    for j in range(f.shape[0]):
+        dot = r @ v[j].T                      # [n][m]
+        att = att + f[j][None, :] * np.exp(-b * d[None, :] * dot * dot)
+    return S0[None, :] * att
+
+
+def dwi_brain(nx=102, ny=102, nz=60, nfibres=2, scale=1.0803, snr=25.0, ndirs=60, nb0=4, b=1.0,
+              gen_seed=41, **kw) -> DwiWorkload:
+    """NEXT-4 workload: brain-shaped DWI (the c3 fibre families, ``_brain_fields``).  Mask
+    = an ellipsoid of semi-axes scale x half the box (clipped to the box), sized so the
+    valid-voxel count matches Table III: 102x102x60 -> ~402k (dataset 2),
+    96x96x48 -> ~205k (dataset 1).  Ground truth per voxel: the N strongest families with
+    f_total 0.6 (as c3), S0 = 1000 (1 + 0.05 g), d = 1.0 (1 + 0.1 g) um^2/ms; Gaussian noise
+    sigma = S0 / snr.  Gradient scheme: ``gradient_scheme(ndirs, nb0, b)``."""
+    rng = np.random.Generator(np.random.PCG64(gen_seed))
+    semi = (scale * nx / 2.0, scale * ny / 2.0, scale * nz / 2.0)
+    r2, dirs, weights, _ = _brain_fields(nx, ny, nz, semi)
+    mask = (r2 <= 1.0).astype(np.uint8)
+    V = nx * ny * nz
+    idx = np.flatnonzero(mask.ravel())
+    m = idx.size
+    N = nfibres
+    order = np.argsort(-weights, axis=0).reshape(3, -1)[:, idx]
+    wsort = np.take_along_axis(weights.reshape(3, -1)[:, idx], order, 0)
+    keep = np.zeros_like(wsort, bool)
+    keep[0] = True
+    for k in range(1, min(N, 3)):
+        keep[k] = wsort[k] >= (0.62 if k == 1 else 0.40) * wsort[0]
+    wk = np.where(keep[:N], wsort[:N], 0.0)
+    f = 0.6 * wk / wk.sum(0, keepdims=True)
+    fam = np.stack([dd.reshape(-1, 3)[idx] for dd in dirs], 0).astype(np.float64)   # [3][m][3]
+    v = np.stack([np.take_along_axis(fam, order[k][None, :, None].repeat(3, -1), 0)[0] for k in range(N)], 0)
+    S0 = 1000.0 * (1.0 + 0.05 * rng.standard_normal(m))
+    d = 1.0 * (1.0 + 0.1 * rng.standard_normal(m))
+    bvals, bvecs = gradient_scheme(ndirs, nb0, b)
+    mu = _forward(S0, d, f, v, bvals, bvecs)
+    y = mu + (S0 / snr)[None, :] * rng.standard_normal(mu.shape)
+    dwi = np.zeros((bvals.size, V), np.float32)
+    dwi[:, idx] = y.astype(np.float32)
+    NP = 3 + 3 * N
+    truth = np.zeros((NP, V), np.float64)
+    truth[0, idx] = S0
+    truth[1, idx] = d
+    truth[2, idx] = S0 / snr
+    for j in range(N):
+        vj = v[j] * np.where(v[j][:, 2:3] < 0, -1.0, 1.0)      # theta in [0, pi/2]
+        truth[3 + 3 * j, idx] = f[j]
+        truth[4 + 3 * j, idx] = np.arccos(np.clip(vj[:, 2], -1, 1))
+        truth[5 + 3 * j, idx] = np.arctan2(vj[:, 1], vj[:, 0])
+    return DwiWorkload(f"dwi_brain_{nx}x{ny}x{nz}_N{N}", nx, ny, nz,
+                       np.ascontiguousarray(dwi.reshape(bvals.size, nz, ny, nx)), bvals, bvecs,
+                       np.ascontiguousarray(mask), truth.reshape(NP, nz, ny, nx), nfibres=N,
+                       recipe=f"brain ellipsoid scale {scale}, {m} voxels, SNR {snr}, "
+                              f"{nb0} b0 + {ndirs} dirs at b={b}, gen_seed={gen_seed}", **kw)
+
+
+def dwi_uniform(nvox=64, S0=1000.0, d=1.0, f=(0.4, 0.2), v=((1.0, 0.0, 0.0), (0.0, 1.0, 0.0)),
+                snr=25.0, ndirs=60, nb0=4, b=1.0, gen_seed=5, nx=None, **kw) -> DwiWorkload:
+    """nvox voxels (a 1-row volume, all in the mask) with the same generating parameters and
+    independent noise: the pins' workload (posterior statistics across voxels)."""
+    rng = np.random.Generator(np.random.PCG64(gen_seed))
+    N = len(f)
+    bvals, bvecs = gradient_scheme(ndirs, nb0, b)
+    vv = np.array([np.asarray(x, np.float64) / np.linalg.norm(x) for x in v])[:, None, :].repeat(nvox, 1)
+    S0a = np.full(nvox, float(S0))
+    da = np.full(nvox, float(d))
+    fa = np.array([np.full(nvox, float(x)) for x in f])
+    mu = _forward(S0a, da, fa, vv, bvals, bvecs)
+    y = mu + (S0 / snr) * rng.standard_normal(mu.shape) if snr else mu
+    nx = nvox if nx is None else nx
+    NP = 3 + 3 * N
+    truth = np.zeros((NP, nvox))
+    truth[0] = S0
+    truth[1] = d
+    truth[2] = S0 / snr if snr else 0.0
+    for j in range(N):
+        truth[3 + 3 * j] = f[j]
+        truth[4 + 3 * j] = math.acos(max(-1.0, min(1.0, vv[j, 0, 2])))
+        truth[5 + 3 * j] = math.atan2(vv[j, 0, 1], vv[j, 0, 0])
+    return DwiWorkload(f"dwi_uniform_{nvox}", nx, 1, 1,
+                       np.ascontiguousarray(y.astype(np.float32).reshape(bvals.size, 1, 1, nx)), bvals, bvecs,
+                       np.ones((1, 1, nx), np.uint8), truth.reshape(NP, 1, 1, nx), nfibres=N,
+                       recipe=f"uniform voxels S0={S0} d={d} f={f} snr={snr}", **kw)
+
+
+MCMC_CONFIGS = {
+    # Table III shapes (P:L301-308): valid-voxel counts ~205k / ~402k
+    "m1": lambda: dwi_brain(96, 96, 48, scale=0.96, gen_seed=43),
+    "m2": lambda: dwi_brain(102, 102, 60, scale=1.0803, gen_seed=41),
+    "m_small": lambda: dwi_brain(24, 24, 16, scale=1.0, gen_seed=47, burnin=100, nsamples=10),
+}
+
+
+def mcmc_config(name: str) -> DwiWorkload:
+    return MCMC_CONFIGS[name]()
 
 
 # ----------------------------------------------------------------------------- configs
