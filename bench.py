@@ -40,6 +40,21 @@ CONFIG_TEXT = {
           "dot threshold 0.9, MaxStep 1888 (Table II row 4 parameters)",
 }
 
+MCMC_METRIC = "MCMC voxels/sec (Table III workload: 50 samples, L = 2, burn-in 500)"
+MCMC_TEXT = {
+    "m1": "NEXT-4 MCMC: dataset-1-shaped DWI 96x96x48, 205k valid voxels, 4 b0 + 60 dirs, N = 2, "
+          "burn-in 500 + 50 samples x interval 2 (Table III row 1)",
+    "m2": "NEXT-4 MCMC: dataset-2-shaped DWI 102x102x60, 402k valid voxels, 4 b0 + 60 dirs, N = 2, "
+          "burn-in 500 + 50 samples x interval 2 (Table III row 2)",
+    "m_small": "NEXT-4 MCMC: 24x24x16 brain, burn-in 100 + 10 samples x 2",
+}
+# Table III: valid voxels, CPU time, GPU time (HD 5870), context only
+PAPER_TABLE3 = {"m1": {"voxels": 205082, "cpu_s": 1383, "gpu_s": 41.3, "speedup": 33.6},
+                "m2": {"voxels": 402194, "cpu_s": 2724, "gpu_s": 80.1, "speedup": 34.0}}
+# executed fp64 lane-instructions per voxel-loop of the MCMC kernel (ncu SASS count,
+# profiles/r01f_mcmc_ncu.md); None until measured
+MCMC_FP64_OPS_PER_VOXEL_LOOP = None
+
 # Table II of the paper, for context beside the NEXT-1 paper-mode workloads:
 # (total fibre length = total steps, longest fibre) on the real CABI datasets, HD 5870.
 PAPER_TABLE2 = {"d1": {"total_steps": 113822762, "longest": 453, "kernel_s": 3.02, "gpu_total_s": 6.74},
@@ -208,6 +223,185 @@ def run_reference(args):
         "e2e": {"value": v, "unit": "steps/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
+    return 0
+
+
+# ----------------------------------------------------------------------------- NEXT-4 MCMC arm
+
+def _fp64_peak():
+    """FP64 FMA lane-instructions/s derived from the unit counts: 148 SMs x 64 FP64 lanes
+    per SM per clock x the measured max SM clock (MEASURED_PEAKS.json, else 1965 MHz)."""
+    p = _peaks()
+    mhz = (p or {}).get("sm_max_mhz", 1965.0)
+    return 148 * 64 * mhz * 1e6
+
+
+def _mcmc_shard(d, rank, world):
+    """Voxel v -> rank v mod N (results are keyed by the voxel index, so exact)."""
+    import numpy as np
+    if world == 1:
+        return d
+    m = d.mask.copy().ravel()
+    idx = np.arange(m.size)
+    m[idx % world != rank] = 0
+    return d.replace(mask=m.reshape(d.mask.shape))
+
+
+def run_mcmc(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_xuzwrwxgxy12_b200 as pt
+    import phantom
+
+    world = _env_int("WORLD_SIZE", 1)
+    rank = _env_int("RANK", 0)
+    local = _env_int("LOCAL_RANK", 0)
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    d = _mcmc_shard(phantom.mcmc_config(args.config), rank, world)
+    tr = pt.Tracker(local)
+    dd = d.replace(dwi=torch.as_tensor(d.dwi, device=dev), bvals=torch.as_tensor(d.bvals, device=dev),
+                   bvecs=torch.as_tensor(d.bvecs, device=dev), mask=torch.as_tensor(d.mask, device=dev))
+    NP = d.nparams
+    out = torch.empty((NP, d.nsamples, d.nz, d.ny, d.nx), dtype=torch.float64, device=dev)
+    for _ in range(args.warmup):
+        tr.mcmc(dd, samples=out)
+    torch.cuda.synchronize()
+    clocks = ClockSampler(local)
+    clocks.start()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    kms = []
+    e0.record()
+    for _ in range(args.steps):
+        tr.mcmc(dd, samples=out)
+        kms.append(tr.mcmc_stats()["kernel_ms"])
+    e1.record()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ck = clocks.stop()
+    ms = e0.elapsed_time(e1)
+    st = tr.mcmc_stats()
+    t = torch.tensor([ms, float(st["voxels"]), float(st["mh_steps"]), float(st["accepted"])],
+                     dtype=torch.float64, device=dev)
+    if world > 1:
+        tm = t.clone()
+        dist.all_reduce(tm, op=dist.ReduceOp.MAX)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        ms = float(tm[0])
+    voxels, steps = float(t[1]), float(t[2])
+
+    # e2e: host DWI in (pinned), host samples out (pinned), through the same C ABI call
+    h = d.replace(dwi=torch.as_tensor(d.dwi).pin_memory(), bvals=torch.as_tensor(d.bvals),
+                  bvecs=torch.as_tensor(d.bvecs), mask=torch.as_tensor(d.mask).pin_memory())
+    out_h = torch.empty((NP, d.nsamples, d.nz, d.ny, d.nx), dtype=torch.float64).pin_memory()
+    tr.mcmc(h, samples=out_h)
+    if world > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    e2e_n = max(1, min(args.steps, 2))
+    for _ in range(e2e_n):
+        tr.mcmc(h, samples=out_h)
+    e2e_s = (time.perf_counter() - t0) / e2e_n
+    te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+
+    kmean = sum(kms) / len(kms)
+    roof = None
+    peak = _fp64_peak()
+    if MCMC_FP64_OPS_PER_VOXEL_LOOP:
+        ach = st["voxels"] * d.loops * MCMC_FP64_OPS_PER_VOXEL_LOOP / (kmean * 1e-3)
+        roof = {"bound": "alu", "achieved": ach / 1e12, "peak": peak / 1e12, "unit": "T fp64 lane-ops/s",
+                "frac": ach / peak, "traffic": None, "kernel_ms": kmean,
+                "ops_per_voxel_loop": MCMC_FP64_OPS_PER_VOXEL_LOOP,
+                "peak_source": "derived: 148 SMs x 64 FP64 lanes x sm_max_mhz"}
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+        oracle.build()
+        threads = len(os.sched_getaffinity(0))
+        idx = np.flatnonzero(d.mask.ravel())
+        cal = idx[:: max(1, idx.size // 16)][:16]
+        t1 = time.perf_counter()
+        oracle.mcmc(d, voxels=cal)
+        per_vox = (time.perf_counter() - t1) / max(1, cal.size)
+        nv = int(min(idx.size, max(threads, args.cpu_seconds * threads / max(per_vox, 1e-6))))
+        pick = idx[:: max(1, idx.size // nv)]
+        t1 = time.perf_counter()
+        oracle.mcmc(d, voxels=pick, threads=threads)
+        dt = time.perf_counter() - t1
+        cpu = {"value": pick.size / dt, "unit": "voxels/s", "cores": threads, "kind": "oracle",
+               "sample": f"every {max(1, idx.size // nv)}th valid voxel ({pick.size} voxels) in {dt:.1f} s"}
+    if rank == 0:
+        line = {
+            "metric": MCMC_METRIC, "value": voxels * args.steps / (ms * 1e-3), "unit": "voxels/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": MCMC_TEXT.get(args.config, args.config), "voxels": int(voxels),
+                       "measurements": int(d.nmeas), "loops": d.loops, "parameters": NP,
+                       "parallelism": f"voxel-sharded x{world}", "l2": "compute-bound (inputs read once per voxel)"},
+            "mh_steps_per_s": steps * args.steps / (ms * 1e-3),
+            "acceptance": float(t[3]) / max(1.0, steps),
+            "paper_table3_context": PAPER_TABLE3.get(args.config),
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "e2e": {"value": voxels / float(te[0]), "unit": "voxels/s",
+                    "h2d_bytes_per_step": int(d.dwi.nbytes + d.mask.nbytes + d.bvals.nbytes + d.bvecs.nbytes),
+                    "d2h_bytes_per_step": int(out_h.numel() * 8)},
+            "gpu_launches": 3 * args.steps,
+            "clocks": ck,
+        }
+        print(json.dumps(line), flush=True)
+    tr.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def run_mcmc_reference(args):
+    """Reference arm of the MCMC workload: the oracle on a bounded voxel sample."""
+    import numpy as np
+    import oracle
+    import phantom
+    if _env_int("RANK", 0) != 0:
+        return 0
+    oracle.build()
+    d = phantom.mcmc_config(args.config)
+    threads = len(os.sched_getaffinity(0))
+    idx = np.flatnonzero(d.mask.ravel())
+    cal = idx[:: max(1, idx.size // 16)][:16]
+    t1 = time.perf_counter()
+    oracle.mcmc(d, voxels=cal)
+    per_vox = (time.perf_counter() - t1) / max(1, cal.size)
+    nv = int(min(idx.size, max(threads, args.cpu_seconds / max(1, args.steps) * threads / max(per_vox, 1e-6))))
+    pick = idx[:: max(1, idx.size // nv)]
+    for _ in range(args.warmup):
+        oracle.mcmc(d, voxels=pick[:threads], threads=threads)
+    secs = 0.0
+    for _ in range(args.steps):
+        t1 = time.perf_counter()
+        oracle.mcmc(d, voxels=pick, threads=threads)
+        secs += time.perf_counter() - t1
+    v = pick.size * args.steps / secs
+    desc = f"{args.config}: every {max(1, idx.size // nv)}th valid voxel ({pick.size}); {threads} worker threads"
+    print(json.dumps({
+        "impl": "reference", "metric": MCMC_METRIC, "value": v, "unit": "voxels/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / args.steps,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic", "config": {"workload": MCMC_TEXT.get(args.config, args.config), "sample": desc},
+        "cpu_baseline": {"value": v, "unit": "voxels/s", "cores": threads, "kind": "oracle", "sample": desc},
+        "e2e": {"value": v, "unit": "voxels/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}), flush=True)
     return 0
 
 
@@ -499,6 +693,10 @@ def main(argv=None):
     args = ap.parse_args(argv)
     if args.warmup < 3 and args.impl == "ours" and not os.environ.get("BENCH_ALLOW_FEW_WARMUP"):
         args.warmup = 3
+    if args.config.startswith("m"):
+        if args.impl == "reference":
+            return run_mcmc_reference(args)
+        return run_mcmc(args)
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)

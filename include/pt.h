@@ -215,6 +215,67 @@ pt_status pt_gather_bench(pt_ctx* ctx, int64_t buffer_bytes, int32_t record_byte
  * (f16).  Returns 0 for invalid arguments. */
 int32_t pt_record_bytes(int32_t nfibres, int32_t dtype);
 
+
+/* ===================================================================================
+ * NEXT-4: MCMC sampling of the local fibre model (the paper's first GPU step, Sec. III-A
+ * P:L61-90, Sec. IV-A and Fig. 2; contract C-MCMC and readings M1-M9 of
+ * DESIGN.md §12).  Per valid voxel, Metropolis-Hastings on Eq. 1 (the multiple partial
+ * volume model) with parameters, in MH order,
+ *     omega = (S0, d, sigma, f_1, theta_1, phi_1, ..., f_N, theta_N, phi_N),  NP = 3 + 3N.
+ * Arithmetic is binary64.  The sample volumes (f_j, theta_j, phi_j) feed pt_load_samples
+ * through pt_mcmc_to_volume (Fig. 1).
+ * =================================================================================== */
+typedef struct {
+    int32_t nx, ny, nz;   /* volume                                                        */
+    int32_t nmeas;        /* n: measurements per voxel, 1..128                               */
+} pt_dwi_shape;
+
+typedef struct {
+    int32_t nfibres;      /* N of Eq. 1, 1..3 (the paper: 2)                          */
+    int32_t burnin;       /* NumBurnIn >= 0 (500)                                     */
+    int32_t nsamples;     /* NumSamples >= 1 (50)                                     */
+    int32_t interval;     /* L >= 1, the sample interval (2)                          */
+    int32_t adapt_every;  /* K >= 1: loops between proposal updates (Fig. 2; M8: 50)          */
+    uint64_t rng_seed;    /* Philox key (M6)                                                  */
+    uint32_t fixed;       /* bit k: parameter k keeps its initial value (M9); bits >= NP = 0  */
+} pt_mcmc_params;
+
+/* Run the sampler on every voxel with mask != 0.
+ *   dwi     : [nmeas][nz][ny][nx] float32 (the 4-D volume of Fig. 1, measurement slowest)
+ *   bvals   : [nmeas] float32 b-values;  bvecs: [nmeas][3] float32 unit gradient directions
+ *   mask    : [nz][ny][nx] uint8, the voxels to sample ("valid (white matter)" voxels)
+ *   init    : [NP][nz][ny][nx] float64 initial states, or NULL for the automatic initial
+ *             state (M7)
+ *   samples : [NP][nsamples][nz][ny][nx] float64 out (host or device; voxels outside the
+ *             mask are set to 0)
+ *   accepted: [NP][nz][ny][nx] uint32 out: accepted proposals per parameter, or NULL
+ * Inputs host or device (copied / read in place); synchronous.  Errors: PT_ERR_ARG for
+ * shapes, nmeas > 128, nfibres outside 1..3, burnin + nsamples*interval >= 2^32, NULL
+ * pointers; PT_ERR_OOM; PT_ERR_CUDA. */
+pt_status pt_mcmc(pt_ctx* ctx, const pt_dwi_shape* shape, const float* dwi, const float* bvals,
+                  const float* bvecs, const uint8_t* mask, const pt_mcmc_params* params,
+                  const double* init, double* samples, uint32_t* accepted);
+
+/* Counters of the last pt_mcmc (synchronises): voxels sampled, MH steps attempted
+ * (voxels x loops x free parameters), proposals accepted, kernel time (CUDA events). */
+typedef struct {
+    uint64_t voxels;
+    uint64_t mh_steps;
+    uint64_t accepted;
+    float kernel_ms;
+} pt_mcmc_stats;
+pt_status pt_get_mcmc_stats(pt_ctx* ctx, pt_mcmc_stats* out);
+
+/* Convert pt_mcmc samples into the tracker's canonical sample volumes (R20: the (theta,
+ * phi) -> unit vector conversion happens here, outside both trackers):
+ *   samples: [3+3N][S][nz][ny][nx] float64 (device or host)
+ *   dyads  : [N][S][nz][ny][nx][3] float32 out = (sin th cos ph, sin th sin ph, cos th)
+ *   f      : [N][S][nz][ny][nx] float32 out
+ * Voxels with mask == 0 get zeros.  Output device or host; synchronous. */
+pt_status pt_mcmc_to_volume(pt_ctx* ctx, const pt_dwi_shape* shape, int32_t nfibres,
+                            int32_t nsamples, const double* samples, const uint8_t* mask,
+                            float* dyads, float* f);
+
 #ifdef __cplusplus
 }
 #endif

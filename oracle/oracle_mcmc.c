@@ -118,7 +118,9 @@ static void initial_state(int nfibres, int n, const double* y, const float* bval
             int k, ok = bvals[i] != 0.0f;
             for (k = 0; k < j && ok; ++k) {
                 const int m = best[k];
-                const double dot = ((double)bvecs[3 * i] * (double)bvecs[3 * m] +
+                double dot;
+                if (m < 0) continue;              /* no earlier pick: no constraint (M7) */
+                dot = ((double)bvecs[3 * i] * (double)bvecs[3 * m] +
                                     (double)bvecs[3 * i + 1] * (double)bvecs[3 * m + 1]) +
                                    (double)bvecs[3 * i + 2] * (double)bvecs[3 * m + 2];
                 if (!(fabs(dot) < 0.5)) ok = 0;

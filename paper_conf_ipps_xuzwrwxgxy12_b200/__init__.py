@@ -26,7 +26,8 @@ __all__ = [
     "pt_record_bytes", "PT_F32", "PT_F16", "PT_REC_LEN", "PT_REC_REASON", "PT_REC_END",
     "PT_REC_PATHS", "PT_MAP_ACCUMULATE", "PT_KERNEL_SIMPLE", "PT_SEED_ORDER_INPUT",
     "PT_SAMPLE_PER_STREAMLINE", "PT_REC_CONN", "PT_BIDIR", "PT_INTERP", "PT_INIT_RANDOM",
-    "PT_INIT_FWEIGHT", "PT_KERNEL_VARIANT", "variant_flags", "pt_load_targets", "pt_get_connectivity", "PT_END_MASK", "PT_END_CURV",
+    "PT_INIT_FWEIGHT", "PT_KERNEL_VARIANT", "variant_flags", "pt_mcmc", "pt_get_mcmc_stats",
+    "pt_mcmc_to_volume", "pt_dwi_shape", "pt_mcmc_params", "pt_load_targets", "pt_get_connectivity", "PT_END_MASK", "PT_END_CURV",
     "PT_END_MAXLEN", "EXPORTS",
 ]
 
@@ -57,7 +58,8 @@ def variant_flags(bidir: int = 0, interp: int = 0, init_fibre: int = 0) -> int:
 # every symbol include/pt.h declares
 EXPORTS = ["pt_create", "pt_destroy", "pt_last_error", "pt_set_stream", "pt_load_samples",
            "pt_track", "pt_get_paths", "pt_get_stats", "pt_gather_bench", "pt_record_bytes",
-           "pt_load_targets", "pt_get_connectivity"]
+           "pt_load_targets", "pt_get_connectivity", "pt_mcmc", "pt_get_mcmc_stats",
+           "pt_mcmc_to_volume"]
 
 _STATUS = {1: "PT_ERR_ARG", 2: "PT_ERR_STATE", 3: "PT_ERR_OOM", 4: "PT_ERR_CUDA", 5: "PT_ERR_OVERFLOW"}
 
@@ -91,6 +93,22 @@ class pt_stats(ctypes.Structure):
                 ("lane_active", ctypes.c_uint64), ("lane_slots", ctypes.c_uint64),
                 ("map_sum", ctypes.c_uint64), ("overflow", ctypes.c_int32),
                 ("kernel_ms", ctypes.c_float), ("track_ms", ctypes.c_float)]
+
+
+class pt_dwi_shape(ctypes.Structure):
+    _fields_ = [("nx", ctypes.c_int32), ("ny", ctypes.c_int32), ("nz", ctypes.c_int32),
+                ("nmeas", ctypes.c_int32)]
+
+
+class pt_mcmc_params(ctypes.Structure):
+    _fields_ = [("nfibres", ctypes.c_int32), ("burnin", ctypes.c_int32), ("nsamples", ctypes.c_int32),
+                ("interval", ctypes.c_int32), ("adapt_every", ctypes.c_int32),
+                ("rng_seed", ctypes.c_uint64), ("fixed", ctypes.c_uint32)]
+
+
+class pt_mcmc_stats(ctypes.Structure):
+    _fields_ = [("voxels", ctypes.c_uint64), ("mh_steps", ctypes.c_uint64), ("accepted", ctypes.c_uint64),
+                ("kernel_ms", ctypes.c_float)]
 
 
 _lib = None
@@ -128,6 +146,12 @@ def lib() -> ctypes.CDLL:
     L.pt_load_targets.restype = ctypes.c_int
     L.pt_get_connectivity.argtypes = [vp, vp, ctypes.c_int64, P(ctypes.c_int64)]
     L.pt_get_connectivity.restype = ctypes.c_int
+    L.pt_mcmc.argtypes = [vp, P(pt_dwi_shape), vp, vp, vp, vp, P(pt_mcmc_params), vp, vp, vp]
+    L.pt_mcmc.restype = ctypes.c_int
+    L.pt_get_mcmc_stats.argtypes = [vp, P(pt_mcmc_stats)]
+    L.pt_get_mcmc_stats.restype = ctypes.c_int
+    L.pt_mcmc_to_volume.argtypes = [vp, P(pt_dwi_shape), ctypes.c_int32, ctypes.c_int32, vp, vp, vp, vp]
+    L.pt_mcmc_to_volume.restype = ctypes.c_int
     L.pt_record_bytes.argtypes = [ctypes.c_int32, ctypes.c_int32]
     L.pt_record_bytes.restype = ctypes.c_int32
     _lib = L
@@ -192,6 +216,24 @@ def pt_get_connectivity(ctx, out_ptr, capacity: int) -> int:
     n = ctypes.c_int64()
     _check(ctx, lib().pt_get_connectivity(ctx, out_ptr, capacity, ctypes.byref(n)))
     return n.value
+
+
+def pt_mcmc(ctx, shape: pt_dwi_shape, dwi_ptr, bvals_ptr, bvecs_ptr, mask_ptr, params: pt_mcmc_params,
+            init_ptr, samples_ptr, accepted_ptr) -> None:
+    _check(ctx, lib().pt_mcmc(ctx, ctypes.byref(shape), dwi_ptr, bvals_ptr, bvecs_ptr, mask_ptr,
+                              ctypes.byref(params), init_ptr, samples_ptr, accepted_ptr))
+
+
+def pt_get_mcmc_stats(ctx) -> pt_mcmc_stats:
+    s = pt_mcmc_stats()
+    _check(ctx, lib().pt_get_mcmc_stats(ctx, ctypes.byref(s)))
+    return s
+
+
+def pt_mcmc_to_volume(ctx, shape: pt_dwi_shape, nfibres: int, nsamples: int, samples_ptr, mask_ptr,
+                      dyads_ptr, f_ptr) -> None:
+    _check(ctx, lib().pt_mcmc_to_volume(ctx, ctypes.byref(shape), nfibres, nsamples, samples_ptr,
+                                        mask_ptr, dyads_ptr, f_ptr))
 
 
 def pt_gather_bench(ctx, buffer_bytes: int, record_bytes: int) -> float:
@@ -336,3 +378,46 @@ class Tracker:
     def gather_bench(self, buffer_bytes: int, record_bytes: int) -> float:
         self._stream()
         return pt_gather_bench(self.ctx, buffer_bytes, record_bytes)
+
+    # ------------------------------------------------------------------ NEXT-4 MCMC
+
+    def mcmc(self, d, *, init=None, fixed: int = 0, accepted: bool = False, samples=None):
+        """pt_mcmc on a phantom.DwiWorkload-like ``d`` (dwi [n][Z][Y][X] float32, bvals,
+        bvecs, mask, nfibres, burnin, nsamples, interval, adapt_every, rng_seed).  Inputs
+        may be numpy (host) or torch tensors; returns (samples, accepted): a cuda float64
+        tensor [NP][S][Z][Y][X] (or the given ``samples`` buffer) and a cuda int32 tensor
+        [NP][Z][Y][X] holding the uint32 counts, or None."""
+        torch = self.torch
+        NP = 3 + 3 * int(d.nfibres)
+        nz, ny, nx = d.mask.shape
+        shape = pt_dwi_shape(nx, ny, nz, int(np.asarray(d.bvals).size if isinstance(d.bvals, np.ndarray)
+                                                else d.bvals.numel()))
+        prm = pt_mcmc_params(int(d.nfibres), int(d.burnin), int(d.nsamples), int(d.interval),
+                             int(d.adapt_every), int(d.rng_seed), int(fixed))
+        if samples is None:
+            samples = torch.empty((NP, int(d.nsamples), nz, ny, nx), dtype=torch.float64, device=self.device)
+        acc = torch.empty((NP, nz, ny, nx), dtype=torch.int32, device=self.device) if accepted else None
+        dwi, bv, bc, mask = (_contig(x) for x in (d.dwi, d.bvals, d.bvecs, d.mask))
+        ini = _contig(init)
+        self._stream()
+        pt_mcmc(self.ctx, shape, _ptr(dwi), _ptr(bv), _ptr(bc), _ptr(mask), prm, _ptr(ini),
+                _ptr(samples), _ptr(acc))
+        return samples, acc
+
+    def mcmc_stats(self) -> dict:
+        s = pt_get_mcmc_stats(self.ctx)
+        return {k: getattr(s, k) for k, _ in pt_mcmc_stats._fields_}
+
+    def mcmc_to_volume(self, samples, mask, nfibres: int):
+        """Sample volumes for load_samples from pt_mcmc samples (R20 conversion on the GPU):
+        returns (dyads [N][S][Z][Y][X][3], f [N][S][Z][Y][X]) float32 cuda tensors."""
+        torch = self.torch
+        S = int(samples.shape[1])
+        nz, ny, nx = mask.shape
+        dy = torch.empty((nfibres, S, nz, ny, nx, 3), dtype=torch.float32, device=self.device)
+        f = torch.empty((nfibres, S, nz, ny, nx), dtype=torch.float32, device=self.device)
+        mask = _contig(mask)
+        self._stream()
+        pt_mcmc_to_volume(self.ctx, pt_dwi_shape(nx, ny, nz, 1), nfibres, S, _ptr(samples), _ptr(mask),
+                          _ptr(dy), _ptr(f))
+        return dy, f

@@ -67,6 +67,18 @@ struct pt_ctx {
     size_t conn_cap = 0;
     uint64_t last_conn_count = 0;
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+    // NEXT-4 MCMC
+    cudaEvent_t mev[2] = {nullptr, nullptr};
+    unsigned long long* d_mstats = nullptr;
+    uint32_t* d_mvox = nullptr;     // compacted mask voxel list
+    size_t mvox_cap = 0;
+    uint8_t* d_mflags = nullptr;
+    size_t mflags_cap = 0;
+    uint8_t* d_mtemp = nullptr;     // DeviceSelect temp storage
+    size_t mtemp_cap = 0;
+    uint32_t* d_mcount = nullptr;   // [0] = selected voxels, [1] = work queue
+    bool mcmc_done = false;
+    uint64_t m_voxels = 0, m_steps = 0;
     // last call
     bool tracked = false;
     uint64_t last_count = 0;
@@ -181,6 +193,13 @@ pt_status pt_create(int cuda_device, pt_ctx** out) {
         return fail(nullptr, PT_ERR_CUDA, "pt_create: %s", cudaGetErrorString(e));
     }
     c->num_sms = prop.multiProcessorCount;
+    for (auto& ev : c->mev) {
+        if (cudaEventCreate(&ev) != cudaSuccess) {
+            cudaGetLastError();
+            pt_destroy(c);
+            return fail(nullptr, PT_ERR_CUDA, "pt_create: cudaEventCreate failed");
+        }
+    }
     for (auto& ev : c->ev) {
         if (cudaEventCreate(&ev) != cudaSuccess) {
             cudaGetLastError();
@@ -204,10 +223,13 @@ void pt_destroy(pt_ctx* c) {
     if (c->stream) cudaStreamSynchronize(c->stream);
     else cudaDeviceSynchronize();
     void* bufs[] = {c->d_rec, c->d_mask, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_copies, c->d_labels, c->d_conn, c->d_nsteps,
-                    c->d_reason, c->d_end, c->d_paths, c->d_stats};
+                    c->d_reason, c->d_end, c->d_paths, c->d_stats, c->d_mstats, c->d_mvox, c->d_mflags,
+                    c->d_mtemp, c->d_mcount};
     for (void* b : bufs)
         if (b) cudaFree(b);
     for (auto& ev : c->ev)
+        if (ev) cudaEventDestroy(ev);
+    for (auto& ev : c->mev)
         if (ev) cudaEventDestroy(ev);
     cudaGetLastError();
     delete c;
@@ -651,6 +673,179 @@ pt_status pt_gather_bench(pt_ctx* c, int64_t buffer_bytes, int32_t record_bytes,
     }
     cleanup();
     *sectors_per_s = best;
+    return PT_OK;
+}
+
+}  // extern "C"
+
+// ------------------------------------------------------------------------- NEXT-4 MCMC
+
+namespace {
+
+// Device view of a caller buffer: device pointers are used in place; host inputs are
+// copied into a temporary device buffer; host outputs get a temporary device buffer that
+// is copied back by finish().
+struct Staged {
+    void* dev = nullptr;
+    void* tmp = nullptr;
+    void* host_out = nullptr;
+    size_t bytes = 0;
+    ~Staged() {
+        if (tmp) cudaFree(tmp);
+    }
+    cudaError_t in(const void* p, size_t n, cudaStream_t st) {
+        bytes = n;
+        if (!p || is_device_ptr(p)) {
+            dev = const_cast<void*>(p);
+            return cudaSuccess;
+        }
+        cudaError_t e = cudaMalloc(&tmp, n ? n : 1);
+        if (e != cudaSuccess) return e;
+        dev = tmp;
+        return cudaMemcpyAsync(tmp, p, n, cudaMemcpyHostToDevice, st);
+    }
+    cudaError_t out(void* p, size_t n) {
+        bytes = n;
+        if (!p || is_device_ptr(p)) {
+            dev = p;
+            return cudaSuccess;
+        }
+        cudaError_t e = cudaMalloc(&tmp, n ? n : 1);
+        if (e != cudaSuccess) return e;
+        dev = tmp;
+        host_out = p;
+        return cudaSuccess;
+    }
+    cudaError_t finish(cudaStream_t st) {
+        if (!host_out) return cudaSuccess;
+        return cudaMemcpyAsync(host_out, dev, bytes, cudaMemcpyDeviceToHost, st);
+    }
+};
+
+}  // namespace
+
+extern "C" {
+
+pt_status pt_mcmc(pt_ctx* c, const pt_dwi_shape* sh, const float* dwi, const float* bvals, const float* bvecs,
+                  const uint8_t* mask, const pt_mcmc_params* p, const double* init, double* samples,
+                  uint32_t* accepted) {
+    if (!c) return PT_ERR_ARG;
+    c->err.clear();
+    if (!sh || !p || !dwi || !bvals || !bvecs || !mask || !samples)
+        return fail(c, PT_ERR_ARG, "pt_mcmc: NULL argument");
+    if (sh->nx <= 0 || sh->ny <= 0 || sh->nz <= 0) return fail(c, PT_ERR_ARG, "pt_mcmc: dims must be > 0");
+    if (sh->nmeas < 1 || sh->nmeas > 128) return fail(c, PT_ERR_ARG, "pt_mcmc: nmeas must be in [1, 128]");
+    if (p->nfibres < 1 || p->nfibres > 3) return fail(c, PT_ERR_ARG, "pt_mcmc: nfibres must be in [1, 3]");
+    if (p->burnin < 0 || p->nsamples < 1 || p->interval < 1 || p->adapt_every < 1)
+        return fail(c, PT_ERR_ARG, "pt_mcmc: burnin >= 0, nsamples >= 1, interval >= 1, adapt_every >= 1");
+    const uint64_t loops = (uint64_t)p->burnin + (uint64_t)p->nsamples * (uint64_t)p->interval;
+    if (loops >= 0xFFFFFFFFull) return fail(c, PT_ERR_ARG, "pt_mcmc: burnin + nsamples * interval >= 2^32");
+    const uint64_t V = (uint64_t)sh->nx * sh->ny * sh->nz;
+    if (V > 0xFFFFFFFFull) return fail(c, PT_ERR_ARG, "pt_mcmc: more than 2^32-1 voxels");
+    const int N = p->nfibres, NP = 3 + 3 * N;
+    const uint32_t fixed = p->fixed & ((1u << NP) - 1u);
+    DeviceGuard g(c->device);
+    if (!g.ok) return fail(c, PT_ERR_CUDA, "pt_mcmc: cannot select device %d", c->device);
+    cudaStream_t st = c->stream;
+    const size_t n = (size_t)sh->nmeas;
+    Staged sd, sb, sv, sm, si, ss, sa;
+    CK(sd.in(dwi, n * V * sizeof(float), st), "pt_mcmc: dwi");
+    CK(sb.in(bvals, n * sizeof(float), st), "pt_mcmc: bvals");
+    CK(sv.in(bvecs, 3 * n * sizeof(float), st), "pt_mcmc: bvecs");
+    CK(sm.in(mask, V, st), "pt_mcmc: mask");
+    CK(si.in(init, init ? (size_t)NP * V * sizeof(double) : 0, st), "pt_mcmc: init");
+    CK(ss.out(samples, (size_t)NP * (size_t)p->nsamples * V * sizeof(double)), "pt_mcmc: samples buffer");
+    CK(sa.out(accepted, accepted ? (size_t)NP * V * sizeof(uint32_t) : 0), "pt_mcmc: accepted buffer");
+    if (!c->d_mstats) CK(cudaMalloc(&c->d_mstats, sizeof(unsigned long long) * pt::kMcmcNumStats), "pt_mcmc: stats");
+    if (!c->d_mcount) CK(cudaMalloc(&c->d_mcount, 2 * sizeof(uint32_t)), "pt_mcmc: counters");
+    CK(ensure(c->d_mvox, c->mvox_cap, V), "pt_mcmc: voxel list");
+    CK(ensure(c->d_mflags, c->mflags_cap, V), "pt_mcmc: flags");
+    CK(ensure(c->d_mtemp, c->mtemp_cap, pt::mcmc_select_temp_bytes(V)), "pt_mcmc: select temp");
+    CK(cudaMemsetAsync(c->d_mcount, 0, 2 * sizeof(uint32_t), st), "pt_mcmc: counters zero");
+    CK(cudaMemsetAsync(c->d_mstats, 0, sizeof(unsigned long long) * pt::kMcmcNumStats, st), "pt_mcmc: stats zero");
+    CK(cudaMemsetAsync(ss.dev, 0, ss.bytes, st), "pt_mcmc: samples zero");
+    if (sa.dev) CK(cudaMemsetAsync(sa.dev, 0, sa.bytes, st), "pt_mcmc: accepted zero");
+    CK(pt::launch_mcmc_voxel_list(static_cast<const uint8_t*>(sm.dev), V, c->d_mflags, c->d_mvox, c->d_mcount,
+                                  c->d_mtemp, c->mtemp_cap, st),
+       "pt_mcmc: voxel list");
+    uint32_t nvox = 0;
+    CK(cudaMemcpyAsync(&nvox, c->d_mcount, sizeof nvox, cudaMemcpyDeviceToHost, st), "pt_mcmc: count");
+    CK(cudaStreamSynchronize(st), "pt_mcmc: synchronise");
+
+    pt::McmcArgs a{};
+    a.dwi = static_cast<const float*>(sd.dev);
+    a.bvals = static_cast<const float*>(sb.dev);
+    a.bvecs = static_cast<const float*>(sv.dev);
+    a.vox = c->d_mvox;
+    a.nvox = nvox;
+    a.queue = c->d_mcount + 1;
+    a.V = V;
+    a.nmeas = sh->nmeas;
+    a.nfibres = N;
+    a.burnin = (uint32_t)p->burnin;
+    a.nsamples = (uint32_t)p->nsamples;
+    a.interval = (uint32_t)p->interval;
+    a.adapt_every = (uint32_t)p->adapt_every;
+    a.loops = (uint32_t)loops;
+    a.key0 = (uint32_t)p->rng_seed;
+    a.key1 = (uint32_t)(p->rng_seed >> 32);
+    a.fixed = fixed;
+    a.init = static_cast<const double*>(si.dev);
+    a.samples = static_cast<double*>(ss.dev);
+    a.accepted = static_cast<uint32_t*>(sa.dev);
+    a.stats = c->d_mstats;
+    CK(cudaEventRecord(c->mev[0], st), "pt_mcmc: event");
+    if (nvox) CK(pt::launch_mcmc(a, c->num_sms, st), "pt_mcmc: kernel launch");
+    CK(cudaEventRecord(c->mev[1], st), "pt_mcmc: event");
+    CK(ss.finish(st), "pt_mcmc: samples D2H");
+    CK(sa.finish(st), "pt_mcmc: accepted D2H");
+    CK(cudaStreamSynchronize(st), "pt_mcmc: synchronise");
+    c->mcmc_done = true;
+    c->m_voxels = nvox;
+    c->m_steps = (uint64_t)nvox * loops * (uint64_t)(NP - __builtin_popcount(fixed));
+    return PT_OK;
+}
+
+pt_status pt_get_mcmc_stats(pt_ctx* c, pt_mcmc_stats* out) {
+    if (!c || !out) return PT_ERR_ARG;
+    c->err.clear();
+    if (!c->mcmc_done) return fail(c, PT_ERR_STATE, "pt_get_mcmc_stats: no pt_mcmc yet");
+    DeviceGuard g(c->device);
+    unsigned long long s[pt::kMcmcNumStats];
+    CK(cudaStreamSynchronize(c->stream), "pt_get_mcmc_stats: synchronise");
+    CK(cudaMemcpy(s, c->d_mstats, sizeof s, cudaMemcpyDeviceToHost), "pt_get_mcmc_stats: copy");
+    out->voxels = c->m_voxels;
+    out->mh_steps = c->m_steps;
+    out->accepted = s[pt::kMcmcStatAccepted];
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, c->mev[0], c->mev[1]), "pt_get_mcmc_stats: kernel time");
+    out->kernel_ms = ms;
+    return PT_OK;
+}
+
+pt_status pt_mcmc_to_volume(pt_ctx* c, const pt_dwi_shape* sh, int32_t nfibres, int32_t nsamples,
+                            const double* samples, const uint8_t* mask, float* dyads, float* f) {
+    if (!c) return PT_ERR_ARG;
+    c->err.clear();
+    if (!sh || !samples || !mask || !dyads || !f) return fail(c, PT_ERR_ARG, "pt_mcmc_to_volume: NULL argument");
+    if (sh->nx <= 0 || sh->ny <= 0 || sh->nz <= 0) return fail(c, PT_ERR_ARG, "pt_mcmc_to_volume: dims must be > 0");
+    if (nfibres < 1 || nfibres > 3 || nsamples < 1)
+        return fail(c, PT_ERR_ARG, "pt_mcmc_to_volume: nfibres in [1, 3], nsamples >= 1");
+    const uint64_t V = (uint64_t)sh->nx * sh->ny * sh->nz;
+    DeviceGuard g(c->device);
+    cudaStream_t st = c->stream;
+    const size_t NP = 3 + 3 * (size_t)nfibres;
+    Staged ss, sm, sd, sf;
+    CK(ss.in(samples, NP * (size_t)nsamples * V * sizeof(double), st), "pt_mcmc_to_volume: samples");
+    CK(sm.in(mask, V, st), "pt_mcmc_to_volume: mask");
+    CK(sd.out(dyads, (size_t)nfibres * nsamples * V * 3 * sizeof(float)), "pt_mcmc_to_volume: dyads");
+    CK(sf.out(f, (size_t)nfibres * nsamples * V * sizeof(float)), "pt_mcmc_to_volume: f");
+    CK(pt::launch_samples_to_volume(static_cast<const double*>(ss.dev), static_cast<const uint8_t*>(sm.dev), V,
+                                    nfibres, nsamples, static_cast<float*>(sd.dev), static_cast<float*>(sf.dev), st),
+       "pt_mcmc_to_volume: kernel");
+    CK(sd.finish(st), "pt_mcmc_to_volume: dyads D2H");
+    CK(sf.finish(st), "pt_mcmc_to_volume: f D2H");
+    CK(cudaStreamSynchronize(st), "pt_mcmc_to_volume: synchronise");
     return PT_OK;
 }
 

@@ -79,6 +79,32 @@ struct TrackArgs {
     const uint8_t* mask;         // [V] tracking mask (interp: candidate test) or nullptr
 };
 
+// NEXT-4 MCMC sampler (pt_mcmc.cu): one warp per voxel of the compacted mask list.
+enum McmcStatIdx { kMcmcStatAccepted = 0, kMcmcNumStats = 2 };
+struct McmcArgs {
+    const float* dwi;            // [nmeas][V]
+    const float* bvals;          // [nmeas]
+    const float* bvecs;          // [nmeas][3]
+    const uint32_t* vox;         // [nvox] linear indices of the mask voxels
+    uint32_t nvox;
+    uint32_t* queue;             // voxel work counter (zeroed per call)
+    uint64_t V;
+    int nmeas, nfibres;
+    uint32_t burnin, nsamples, interval, adapt_every, loops;
+    uint32_t key0, key1;
+    uint32_t fixed;              // bit k: parameter k held at its initial value (M9)
+    const double* init;          // [NP][V] or nullptr (automatic initial state, M7)
+    double* samples;             // [NP][nsamples][V]
+    uint32_t* accepted;          // [NP][V] or nullptr
+    unsigned long long* stats;   // [kMcmcNumStats]
+};
+size_t mcmc_select_temp_bytes(uint64_t V);
+cudaError_t launch_mcmc_voxel_list(const uint8_t* mask, uint64_t V, uint8_t* flags, uint32_t* out, uint32_t* nsel,
+                                   void* temp, size_t temp_bytes, cudaStream_t st);
+cudaError_t launch_mcmc(const McmcArgs& a, int num_sms, cudaStream_t st);
+cudaError_t launch_samples_to_volume(const double* samples, const uint8_t* mask, uint64_t V, int N, int S,
+                                     float* dyads, float* f, cudaStream_t st);
+
 // Launchers (return the launch error, if any).
 cudaError_t launch_track(const TrackArgs& a, int nfibres, bool half, bool simple, int num_sms,
                          cudaStream_t st);

@@ -1,0 +1,510 @@
+// pt_mcmc.cu -- NEXT-4: Metropolis-Hastings sampling of the multiple partial volume model
+// (Eq. 1; Sec. IV-A and Fig. 2) on sm_100a, binary64 (reading M4).
+//
+// The paper runs one thread per voxel.  Here one WARP owns a voxel and its lanes
+// own the voxel's measurements (lane l holds i = l, l+32, ...): the per-measurement terms
+// of Eq. 1 stay in registers for the whole chain (e^{-b d}, e^{-b d (r.v_j)^2}, r.v_j,
+// the mixture A_i), so a proposal of S0, sigma or f_j costs no exponential at all, a
+// proposal of an angle costs one per measurement and a proposal of d costs N+1; the sum of
+// squared residuals is a warp reduction.  The NP draws of a loop do not depend on the state
+// (counter-based Philox, M6), and omega'_k only depends on omega_k, which no other MH step
+// of the loop changes: lane k computes draw k, the candidate and its transcendental
+// by-products (ln sigma', sincos, ln|sin theta'|) for all NP steps of the loop in parallel
+// at the loop's start; step k then only broadcasts them from lane k.
+//
+// Results follow contract C-MCMC of DESIGN.md §12 in the oracle's operation order; the
+// oracle uses glibc's exp/log/sin/cos, this file CUDA's (both within an ulp or two), and
+// the residual sum is a warp tree instead of a sequential loop, so samples agree to
+// ~1e-13 relative rather than bit for bit (the parity bar of DESIGN.md §12).
+#include <cuda_runtime.h>
+#include <cub/device/device_select.cuh>
+#include <thrust/iterator/counting_iterator.h>
+
+#include <cstdint>
+
+#include "pt_device.cuh"
+#include "pt_internal.h"
+
+namespace pt {
+
+namespace {
+
+constexpr uint32_t kTag = 0x4D434D43u;  // "MCMC": Philox counter word 3 (M6)
+constexpr double kTwoPi = 6.283185307179586;
+constexpr int kMcmcThreads = 128;         // 4 voxels (warps) per CTA
+
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+    return __shfl_sync(kFull, v, 0);  // one value for every lane (the butterfly's lanes may differ)
+}
+
+template <int N, int MPL>
+__global__ void __launch_bounds__(kMcmcThreads) mcmc_kernel(const __grid_constant__ McmcArgs a) {
+    constexpr int NP = 3 + 3 * N;
+    const uint32_t lane = threadIdx.x & 31u;
+    const int n = a.nmeas;
+    const double np1 = (double)(n + 1);
+
+    // per-measurement data (registers): i = lane + 32 m
+    bool valid[MPL];
+    float yf[MPL], bf[MPL], rx[MPL], ry[MPL], rz[MPL];
+#pragma unroll
+    for (int m = 0; m < MPL; ++m) {
+        const int i = (int)lane + 32 * m;
+        valid[m] = i < n;
+        bf[m] = valid[m] ? a.bvals[i] : 0.f;
+        rx[m] = valid[m] ? a.bvecs[3 * i] : 0.f;
+        ry[m] = valid[m] ? a.bvecs[3 * i + 1] : 0.f;
+        rz[m] = valid[m] ? a.bvecs[3 * i + 2] : 0.f;
+    }
+    unsigned long long acc_tot = 0ull;
+
+    for (;;) {
+        uint32_t slot = 0;
+        if (lane == 0) slot = atomicAdd(a.queue, 1u);
+        slot = __shfl_sync(kFull, slot, 0);
+        if (slot >= a.nvox) break;
+        const uint32_t v = a.vox[slot];
+        const uint64_t V = a.V;
+#pragma unroll
+        for (int m = 0; m < MPL; ++m) yf[m] = valid[m] ? a.dwi[(uint64_t)(lane + 32 * m) * V + v] : 0.f;
+
+        double w[NP];
+        double sth[N], cth[N], sph[N], cph[N], lsin[N];
+        // ------------------------------------------------ initial state (M7 or given)
+        if (a.init) {
+#pragma unroll
+            for (int k = 0; k < NP; ++k) w[k] = a.init[(uint64_t)k * V + v];
+        } else {
+            double s0 = 0.0, sd = 0.0, bsum = 0.0, ymax = -__longlong_as_double(0x7FF0000000000000ll);
+            int c0 = 0, cd = 0;
+#pragma unroll
+            for (int m = 0; m < MPL; ++m) {
+                if (!valid[m]) continue;
+                const double y = (double)yf[m];
+                ymax = y > ymax ? y : ymax;
+                if (bf[m] == 0.f) {
+                    s0 += y;
+                    c0 += 1;
+                } else {
+                    sd += y;
+                    bsum += (double)bf[m];
+                    cd += 1;
+                }
+            }
+            s0 = warp_sum(s0);
+            sd = warp_sum(sd);
+            bsum = warp_sum(bsum);
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                c0 += __shfl_xor_sync(kFull, c0, o);
+                cd += __shfl_xor_sync(kFull, cd, o);
+                ymax = fmax(ymax, __shfl_xor_sync(kFull, ymax, o));
+            }
+            double S0 = c0 ? s0 / (double)c0 : ymax;
+            if (!(S0 > 0.0)) S0 = 1.0;
+            double d = 0.0;
+            if (cd) d = -log((sd / (double)cd) / S0) / (bsum / (double)cd);
+            if (!(d > 0.0) || !isfinite(d)) d = cd ? 1.0 / (bsum / (double)cd) : 1.0;
+            w[0] = S0;
+            w[1] = d;
+            // fibre j: DW direction of the smallest signal with |r.v_k| < 1/2 for earlier fibres
+            float px[N], py[N], pz[N];
+            bool have[N];
+#pragma unroll
+            for (int j = 0; j < N; ++j) {
+                float by = __int_as_float(0x7F800000);
+                int bi = 0x7FFFFFFF;
+#pragma unroll
+                for (int m = 0; m < MPL; ++m) {
+                    bool ok = valid[m] && bf[m] != 0.f;
+#pragma unroll
+                    for (int k = 0; k < j; ++k) {
+                        const double dot = ((double)rx[m] * (double)px[k] + (double)ry[m] * (double)py[k]) +
+                                           (double)rz[m] * (double)pz[k];
+                        if (have[k]) ok = ok && fabs(dot) < 0.5;  // a missing pick constrains nothing
+                    }
+                    const int i = (int)lane + 32 * m;
+                    if (ok && (yf[m] < by || (yf[m] == by && i < bi))) {
+                        by = yf[m];
+                        bi = i;
+                    }
+                }
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) {
+                    const float oy = __shfl_xor_sync(kFull, by, o);
+                    const int oi = __shfl_xor_sync(kFull, bi, o);
+                    if (oy < by || (oy == by && oi < bi)) {
+                        by = oy;
+                        bi = oi;
+                    }
+                }
+                have[j] = bi != 0x7FFFFFFF;
+                px[j] = py[j] = pz[j] = 0.f;
+                if (have[j]) {
+                    px[j] = a.bvecs[3 * bi];
+                    py[j] = a.bvecs[3 * bi + 1];
+                    pz[j] = a.bvecs[3 * bi + 2];
+                }
+                w[3 + 3 * j] = j == 0 ? 0.3 : 0.1;
+                if (have[j]) {
+                    const double z = (double)pz[j];
+                    w[4 + 3 * j] = acos(z < -1.0 ? -1.0 : (z > 1.0 ? 1.0 : z));
+                    w[5 + 3 * j] = atan2((double)py[j], (double)px[j]);
+                } else if (j == 0) {
+                    w[4] = 1.0;
+                    w[5] = 0.0;
+                } else {
+                    w[4 + 3 * j] = w[4] + (j == 1 ? 1.5707963267948966 : 0.0);
+                    w[5 + 3 * j] = w[5] + (j == 2 ? 1.5707963267948966 : 0.0);
+                }
+            }
+            w[2] = 1.0;  // sigma: set below from the initial model's residual
+        }
+#pragma unroll
+        for (int j = 0; j < N; ++j) {
+            sincos(w[4 + 3 * j], &sth[j], &cth[j]);
+            sincos(w[5 + 3 * j], &sph[j], &cph[j]);
+            lsin[j] = log(fabs(sth[j]));
+        }
+
+        // ------------------------------------------------ per-measurement caches (Eq. 1)
+        double e0[MPL], ej[N][MPL], dj[N][MPL], A[MPL];
+        double sumf = 0.0;
+#pragma unroll
+        for (int j = 0; j < N; ++j) sumf = sumf + w[3 + 3 * j];
+        double sse = 0.0;
+#pragma unroll
+        for (int m = 0; m < MPL; ++m) {
+            const double b = (double)bf[m];
+            const double bd = b * w[1];
+            e0[m] = exp(-bd);
+            double acc = (1.0 - sumf) * e0[m];
+#pragma unroll
+            for (int j = 0; j < N; ++j) {
+                const double vx = sth[j] * cph[j], vy = sth[j] * sph[j], vz = cth[j];
+                dj[j][m] = ((double)rx[m] * vx + (double)ry[m] * vy) + (double)rz[m] * vz;
+                ej[j][m] = exp(-(bd * (dj[j][m] * dj[j][m])));
+                acc = acc + w[3 + 3 * j] * ej[j][m];
+            }
+            A[m] = acc;
+            const double r = (double)yf[m] - w[0] * acc;
+            sse += valid[m] ? r * r : 0.0;
+        }
+        sse = warp_sum(sse);
+        if (!a.init) {
+            double sig = sqrt(sse / (double)n);
+            if (!(sig >= 1e-3 * w[0])) sig = 1e-3 * w[0];
+            w[2] = sig;
+        }
+        double lsig = log(w[2]);
+        double lp = -np1 * lsig - sse / (2.0 * w[2] * w[2]);
+#pragma unroll
+        for (int j = 0; j < N; ++j) lp = lp + lsin[j];
+
+        // ------------------------------------------------ proposals (M8)
+        double prop[NP];
+        prop[0] = 0.01 * w[0];
+        prop[1] = 0.1 * w[1];
+        prop[2] = 0.1 * w[2];
+#pragma unroll
+        for (int j = 0; j < N; ++j) {
+            prop[3 + 3 * j] = 0.05;
+            prop[4 + 3 * j] = 0.1;
+            prop[5 + 3 * j] = 0.1;
+        }
+        uint32_t acc[NP], rej[NP], tot[NP];
+#pragma unroll
+        for (int k = 0; k < NP; ++k) acc[k] = rej[k] = tot[k] = 0u;
+
+        const uint32_t loops = a.loops;
+        for (uint32_t t = 0; t < loops; ++t) {
+            // lane k < NP: draw k of this loop (M6), candidate omega'_k and its by-products
+            double cz = 0.0, clu = 0.0, ca = 0.0, cb = 0.0, cc = 0.0;
+            if (lane < (uint32_t)NP) {
+                const uint4 R = philox4x32_10(make_uint4(t, v, lane, kTag), a.key0, a.key1);
+                const double u1 = ((double)R.x + 0.5) * 0x1p-32;
+                const double u2 = (double)R.y * 0x1p-32;
+                const double u3 = ((double)R.z + 0.5) * 0x1p-32;
+                const double z = sqrt(-2.0 * log(u1)) * cos(kTwoPi * u2);
+                clu = log(u3);
+                double wk = w[0], pk = prop[0];
+#pragma unroll
+                for (int k = 1; k < NP; ++k) {
+                    wk = lane == (uint32_t)k ? w[k] : wk;
+                    pk = lane == (uint32_t)k ? prop[k] : pk;
+                }
+                cz = wk + pk * z;
+                if (lane == 2u) {
+                    ca = log(cz);
+                } else if (lane >= 3u) {
+                    const uint32_t r3 = (lane - 3u) % 3u;
+                    if (r3 == 1u) {  // theta: sin, cos, ln|sin|
+                        sincos(cz, &ca, &cb);
+                        cc = log(fabs(ca));
+                    } else if (r3 == 2u) {  // phi: sin, cos
+                        sincos(cz, &ca, &cb);
+                    }
+                }
+            }
+            // Fig. 2: the MH step, repeated NumParameters times
+#pragma unroll
+            for (int k = 0; k < NP; ++k) {
+                if (a.fixed & (1u << k)) continue;
+                const double cand = __shfl_sync(kFull, cz, k);
+                const double lu = __shfl_sync(kFull, clu, k);
+                const double xa = __shfl_sync(kFull, ca, k);
+                const double xb = __shfl_sync(kFull, cb, k);
+                const double xc = __shfl_sync(kFull, cc, k);
+                // support (M3)
+                bool ok;
+                double nsumf = sumf;
+                if (k == 0 || k == 1 || k == 2) {
+                    ok = cand > 0.0;
+                } else if ((k - 3) % 3 == 0) {
+                    nsumf = 0.0;
+#pragma unroll
+                    for (int j = 0; j < N; ++j) nsumf = nsumf + (3 + 3 * j == k ? cand : w[3 + 3 * j]);
+                    ok = cand >= 0.0 && nsumf <= 1.0;
+                } else {
+                    ok = true;
+                }
+                if (!ok) {
+                    rej[k] += 1u;
+                    continue;
+                }
+                const int jf = k >= 3 ? (k - 3) / 3 : 0;  // fibre of an f/theta/phi step
+                double nvx = 0.0, nvy = 0.0, nvz = 0.0;
+                if (k >= 3 && (k - 3) % 3 == 1) {  // theta' with the current phi
+                    nvx = xa * cph[jf];
+                    nvy = xa * sph[jf];
+                    nvz = xb;
+                } else if (k >= 3 && (k - 3) % 3 == 2) {  // phi' with the current theta
+                    nvx = sth[jf] * xb;
+                    nvy = sth[jf] * xa;
+                    nvz = cth[jf];
+                }
+                double nsse = 0.0, nlp;
+                double ne[MPL], nd[MPL], nA[MPL], nej[N][MPL];
+                if (k == 2) {
+                    nlp = -np1 * xa - sse / (2.0 * cand * cand);
+#pragma unroll
+                    for (int j = 0; j < N; ++j) nlp = nlp + lsin[j];
+                } else {
+#pragma unroll
+                    for (int m = 0; m < MPL; ++m) {
+                        double mu;
+                        if (k == 0) {
+                            mu = cand * A[m];
+                        } else if (k == 1) {
+                            const double bd = (double)bf[m] * cand;
+                            ne[m] = exp(-bd);
+                            double accm = (1.0 - sumf) * ne[m];
+#pragma unroll
+                            for (int j = 0; j < N; ++j) {
+                                nej[j][m] = exp(-(bd * (dj[j][m] * dj[j][m])));
+                                accm = accm + w[3 + 3 * j] * nej[j][m];
+                            }
+                            nA[m] = accm;
+                            mu = w[0] * accm;
+                        } else if ((k - 3) % 3 == 0) {
+                            double accm = (1.0 - nsumf) * e0[m];
+#pragma unroll
+                            for (int j = 0; j < N; ++j) accm = accm + (j == jf ? cand : w[3 + 3 * j]) * ej[j][m];
+                            nA[m] = accm;
+                            mu = w[0] * accm;
+                        } else {
+                            const double bd = (double)bf[m] * w[1];
+                            nd[m] = ((double)rx[m] * nvx + (double)ry[m] * nvy) + (double)rz[m] * nvz;
+                            ne[m] = exp(-(bd * (nd[m] * nd[m])));
+                            double accm = (1.0 - sumf) * e0[m];
+#pragma unroll
+                            for (int j = 0; j < N; ++j) accm = accm + w[3 + 3 * j] * (j == jf ? ne[m] : ej[j][m]);
+                            nA[m] = accm;
+                            mu = w[0] * accm;
+                        }
+                        const double r = (double)yf[m] - mu;
+                        nsse += valid[m] ? r * r : 0.0;
+                    }
+                    nsse = warp_sum(nsse);
+                    nlp = -np1 * lsig - nsse / (2.0 * w[2] * w[2]);
+#pragma unroll
+                    for (int j = 0; j < N; ++j) nlp = nlp + ((k >= 3 && (k - 3) % 3 == 1 && j == jf) ? xc : lsin[j]);
+                }
+                // accept with probability min(r, 1): ln u < lp' - lp
+                if (lu < nlp - lp) {
+                    acc[k] += 1u;
+                    tot[k] += 1u;
+                    w[k] = cand;
+                    lp = nlp;
+                    if (k == 2) {
+                        lsig = xa;
+                    } else {
+                        sse = nsse;
+                        if (k == 1) {
+#pragma unroll
+                            for (int m = 0; m < MPL; ++m) {
+                                e0[m] = ne[m];
+#pragma unroll
+                                for (int j = 0; j < N; ++j) ej[j][m] = nej[j][m];
+                                A[m] = nA[m];
+                            }
+                        } else if (k >= 3) {
+                            const int r3 = (k - 3) % 3;
+                            if (r3 == 0) {
+                                sumf = nsumf;
+                            } else if (r3 == 1) {
+                                sth[jf] = xa;
+                                cth[jf] = xb;
+                                lsin[jf] = xc;
+                            } else {
+                                sph[jf] = xa;
+                                cph[jf] = xb;
+                            }
+#pragma unroll
+                            for (int m = 0; m < MPL; ++m) {
+                                A[m] = nA[m];
+                                if (r3 != 0) {
+                                    dj[jf][m] = nd[m];
+                                    ej[jf][m] = ne[m];
+                                }
+                            }
+                        } else {
+                            // S0: A unchanged
+                        }
+                    }
+                } else {
+                    rej[k] += 1u;
+                }
+            }
+            // Fig. 2: every K loops the acceptance rates update the proposals (M8)
+            if ((t + 1u) % a.adapt_every == 0u) {
+#pragma unroll
+                for (int k = 0; k < NP; ++k) {
+                    prop[k] = prop[k] * sqrt((5.0 * (double)(acc[k] + 1u)) / (3.0 * (double)(rej[k] + 1u)));
+                    acc[k] = rej[k] = 0u;
+                }
+            }
+            // samples after the burn-in, every L loops; lane k writes omega_k
+            if (t >= a.burnin && (t - a.burnin + 1u) % a.interval == 0u) {
+                const uint32_t s = (t - a.burnin + 1u) / a.interval - 1u;
+                double wk = w[0];
+#pragma unroll
+                for (int k = 1; k < NP; ++k) wk = lane == (uint32_t)k ? w[k] : wk;
+                if (lane < (uint32_t)NP) a.samples[((uint64_t)lane * a.nsamples + s) * V + v] = wk;
+            }
+        }
+        if (a.accepted) {
+            uint32_t tk = tot[0];
+#pragma unroll
+            for (int k = 1; k < NP; ++k) tk = lane == (uint32_t)k ? tot[k] : tk;
+            if (lane < (uint32_t)NP) a.accepted[(uint64_t)lane * V + v] = tk;
+        }
+        if (lane == 0) {
+#pragma unroll
+            for (int k = 0; k < NP; ++k) acc_tot += tot[k];
+        }
+    }
+    if (lane == 0 && acc_tot) atomicAdd(a.stats + kMcmcStatAccepted, acc_tot);
+}
+
+template <int N, int MPL>
+cudaError_t launch_m(const McmcArgs& a, int num_sms, cudaStream_t st) {
+    auto k = mcmc_kernel<N, MPL>;
+    int per_sm = 0;
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kMcmcThreads, 0);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) return cudaErrorInvalidConfiguration;
+    const uint64_t need = ((uint64_t)a.nvox + kMcmcThreads / 32 - 1) / (kMcmcThreads / 32);
+    const uint64_t full = (uint64_t)num_sms * (uint64_t)per_sm;
+    const uint64_t grid = need < full ? need : full;
+    if (grid == 0) return cudaSuccess;
+    k<<<(unsigned)grid, kMcmcThreads, 0, st>>>(a);
+    return cudaGetLastError();
+}
+
+template <int N>
+cudaError_t launch_mn(const McmcArgs& a, int num_sms, cudaStream_t st) {
+    switch ((a.nmeas + 31) / 32) {
+        case 1: return launch_m<N, 1>(a, num_sms, st);
+        case 2: return launch_m<N, 2>(a, num_sms, st);
+        case 3: return launch_m<N, 3>(a, num_sms, st);
+        case 4: return launch_m<N, 4>(a, num_sms, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+__global__ void mask_flags_kernel(const uint8_t* __restrict__ mask, uint64_t V, uint8_t* __restrict__ flags) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < V; i += (uint64_t)gridDim.x * blockDim.x)
+        flags[i] = mask[i] != 0 ? 1 : 0;
+}
+
+// (theta, phi) -> unit vector, f -> float (R20: the conversion is outside the trackers)
+__global__ void samples_to_volume_kernel(const double* __restrict__ smp, const uint8_t* __restrict__ mask,
+                                         uint64_t V, int N, int S, float* __restrict__ dyads, float* __restrict__ f) {
+    const uint64_t total = (uint64_t)N * S * V;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t v = i % V;
+        const uint64_t js = i / V;          // j * S + s
+        const uint64_t j = js / S, s = js - j * S;
+        float x = 0.f, y = 0.f, z = 0.f, ff = 0.f;
+        if (mask[v]) {
+            const double fj = smp[((3 + 3 * j) * S + s) * V + v];
+            const double th = smp[((4 + 3 * j) * S + s) * V + v];
+            const double ph = smp[((5 + 3 * j) * S + s) * V + v];
+            double st, ct, sp, cp;
+            sincos(th, &st, &ct);
+            sincos(ph, &sp, &cp);
+            x = (float)(st * cp);
+            y = (float)(st * sp);
+            z = (float)ct;
+            ff = (float)fj;
+        }
+        dyads[3 * i] = x;
+        dyads[3 * i + 1] = y;
+        dyads[3 * i + 2] = z;
+        f[i] = ff;
+    }
+}
+
+}  // namespace
+
+size_t mcmc_select_temp_bytes(uint64_t V) {
+    size_t bytes = 0;
+    cub::DeviceSelect::Flagged(nullptr, bytes, thrust::counting_iterator<uint32_t>(0), (const uint8_t*)nullptr,
+                               (uint32_t*)nullptr, (uint32_t*)nullptr, (int64_t)V);
+    return bytes;
+}
+
+cudaError_t launch_mcmc_voxel_list(const uint8_t* mask, uint64_t V, uint8_t* flags, uint32_t* out, uint32_t* nsel,
+                                   void* temp, size_t temp_bytes, cudaStream_t st) {
+    uint64_t blocks = (V + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    if (blocks < 1) blocks = 1;
+    mask_flags_kernel<<<(unsigned)blocks, 256, 0, st>>>(mask, V, flags);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+    return cub::DeviceSelect::Flagged(temp, temp_bytes, thrust::counting_iterator<uint32_t>(0), flags, out, nsel,
+                                      (int64_t)V, st);
+}
+
+cudaError_t launch_mcmc(const McmcArgs& a, int num_sms, cudaStream_t st) {
+    switch (a.nfibres) {
+        case 1: return launch_mn<1>(a, num_sms, st);
+        case 2: return launch_mn<2>(a, num_sms, st);
+        case 3: return launch_mn<3>(a, num_sms, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+cudaError_t launch_samples_to_volume(const double* samples, const uint8_t* mask, uint64_t V, int N, int S,
+                                     float* dyads, float* f, cudaStream_t st) {
+    uint64_t blocks = ((uint64_t)N * S * V + 255) / 256;
+    if (blocks > 148 * 32) blocks = 148 * 32;
+    if (blocks < 1) blocks = 1;
+    samples_to_volume_kernel<<<(unsigned)blocks, 256, 0, st>>>(samples, mask, V, N, S, dyads, f);
+    return cudaGetLastError();
+}
+
+}  // namespace pt
