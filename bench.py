@@ -439,6 +439,9 @@ def run_ours(args):
     mine = _shard(w, rank, world)
     tr = pt.Tracker(local)
     tr.load_volume(w.volume)
+    if args.segments:
+        tr.set_segments({"B": pt.SEGMENTS_B, "C": pt.SEGMENTS_C}.get(args.segments) or
+                        [int(x) for x in args.segments.split(",")])
     base_flags = args.track_flags | (pt.PT_SAMPLE_PER_STREAMLINE if getattr(w, "sample_mode", 0) else 0)
     V = w.volume.nx * w.volume.ny * w.volume.nz
     rb = pt.pt_record_bytes(w.volume.nfibres, pt.PT_F16 if w.volume.is_half else pt.PT_F32)
@@ -690,6 +693,9 @@ def main(argv=None):
     ap.add_argument("--track-flags", type=int, default=0,
                     help="extra pt_params.flags for ablations (e.g. 256 = PT_KERNEL_SIMPLE, "
                          "512 = PT_SEED_ORDER_INPUT)")
+    ap.add_argument("--segments", default="",
+                    help="schedule of the PT_KERNEL_SEGMENTED ablation (--track-flags 65536): "
+                         "B, C or a comma list of intervals (the paper's NumIteration[])")
     args = ap.parse_args(argv)
     if args.warmup < 3 and args.impl == "ours" and not os.environ.get("BENCH_ALLOW_FEW_WARMUP"):
         args.warmup = 3

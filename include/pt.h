@@ -77,6 +77,12 @@ typedef enum { PT_END_MASK = 0, PT_END_CURV = 1, PT_END_MAXLEN = 2 } pt_reason;
                                         PT_INIT_RANDOM                                   */
 #define PT_KERNEL_VARIANT (1u << 15) /* run the variant kernel even with no variant flag
                                         (same results as the main kernel; ablation/tests) */
+#define PT_KERNEL_SEGMENTED (1u << 16) /* ablation (ii): the paper's segmented relaunch
+                                        (Table IV): one thread per live particle
+                                        per segment of k steps, device stream compaction
+                                        between segments, schedule of pt_set_segments.
+                                        Same results; synchronous; not combinable with
+                                        PT_REC_PATHS, PT_REC_CONN or the NEXT-3 variants */
 
 /* Create a context on CUDA device `cuda_device` (the caller's current device is left
  * unchanged).  *out receives the context or NULL.  The stream defaults to the legacy
@@ -145,6 +151,12 @@ typedef struct {
  * pt_get_stats/pt_get_paths. */
 pt_status pt_track(pt_ctx* ctx, const float* seeds_xyz, const uint64_t* seed_ids,
                    int64_t nseeds, const pt_params* params, uint32_t* map);
+
+/* Segment schedule of PT_KERNEL_SEGMENTED: NumIteration[] of the paper,
+ * intervals[0..n-1] steps per segment, the last one repeating until no particle is alive.
+ * Default: strategy B = {1, 2, 5, 10, 20, 50, 100, 200, 500}.  Errors: PT_ERR_ARG for
+ * n < 1, n > 64 or an interval < 1. */
+pt_status pt_set_segments(pt_ctx* ctx, const int32_t* intervals, int32_t n);
 
 /* Target regions for the seed x target connectivity matrix (NEXT-2; the connectivity
  * estimate of P:L109, "counting the number of streamlines passing through B, and dividing

@@ -27,7 +27,8 @@ __all__ = [
     "PT_REC_PATHS", "PT_MAP_ACCUMULATE", "PT_KERNEL_SIMPLE", "PT_SEED_ORDER_INPUT",
     "PT_SAMPLE_PER_STREAMLINE", "PT_REC_CONN", "PT_BIDIR", "PT_INTERP", "PT_INIT_RANDOM",
     "PT_INIT_FWEIGHT", "PT_KERNEL_VARIANT", "variant_flags", "pt_mcmc", "pt_get_mcmc_stats",
-    "pt_mcmc_to_volume", "pt_dwi_shape", "pt_mcmc_params", "pt_load_targets", "pt_get_connectivity", "PT_END_MASK", "PT_END_CURV",
+    "pt_mcmc_to_volume", "pt_dwi_shape", "pt_mcmc_params", "PT_KERNEL_SEGMENTED", "pt_set_segments",
+    "SEGMENTS_B", "SEGMENTS_C", "pt_load_targets", "pt_get_connectivity", "PT_END_MASK", "PT_END_CURV",
     "PT_END_MAXLEN", "EXPORTS",
 ]
 
@@ -48,6 +49,10 @@ PT_INTERP = 1 << 12
 PT_INIT_RANDOM = 1 << 13
 PT_INIT_FWEIGHT = 1 << 14
 PT_KERNEL_VARIANT = 1 << 15
+PT_KERNEL_SEGMENTED = 1 << 16
+# the paper's increasing-interval segmentation strategies
+SEGMENTS_B = (1, 2, 5, 10, 20, 50, 100, 200, 500)
+SEGMENTS_C = (1, 1, 2, 2, 5, 5, 10, 10, 20, 20, 50, 50, 100, 100, 200, 200)
 
 
 def variant_flags(bidir: int = 0, interp: int = 0, init_fibre: int = 0) -> int:
@@ -59,7 +64,7 @@ def variant_flags(bidir: int = 0, interp: int = 0, init_fibre: int = 0) -> int:
 EXPORTS = ["pt_create", "pt_destroy", "pt_last_error", "pt_set_stream", "pt_load_samples",
            "pt_track", "pt_get_paths", "pt_get_stats", "pt_gather_bench", "pt_record_bytes",
            "pt_load_targets", "pt_get_connectivity", "pt_mcmc", "pt_get_mcmc_stats",
-           "pt_mcmc_to_volume"]
+           "pt_mcmc_to_volume", "pt_set_segments"]
 
 _STATUS = {1: "PT_ERR_ARG", 2: "PT_ERR_STATE", 3: "PT_ERR_OOM", 4: "PT_ERR_CUDA", 5: "PT_ERR_OVERFLOW"}
 
@@ -152,6 +157,8 @@ def lib() -> ctypes.CDLL:
     L.pt_get_mcmc_stats.restype = ctypes.c_int
     L.pt_mcmc_to_volume.argtypes = [vp, P(pt_dwi_shape), ctypes.c_int32, ctypes.c_int32, vp, vp, vp, vp]
     L.pt_mcmc_to_volume.restype = ctypes.c_int
+    L.pt_set_segments.argtypes = [vp, vp, ctypes.c_int32]
+    L.pt_set_segments.restype = ctypes.c_int
     L.pt_record_bytes.argtypes = [ctypes.c_int32, ctypes.c_int32]
     L.pt_record_bytes.restype = ctypes.c_int32
     _lib = L
@@ -234,6 +241,11 @@ def pt_mcmc_to_volume(ctx, shape: pt_dwi_shape, nfibres: int, nsamples: int, sam
                       dyads_ptr, f_ptr) -> None:
     _check(ctx, lib().pt_mcmc_to_volume(ctx, ctypes.byref(shape), nfibres, nsamples, samples_ptr,
                                         mask_ptr, dyads_ptr, f_ptr))
+
+
+def pt_set_segments(ctx, intervals) -> None:
+    arr = (ctypes.c_int32 * len(intervals))(*[int(x) for x in intervals])
+    _check(ctx, lib().pt_set_segments(ctx, arr, len(intervals)))
 
 
 def pt_gather_bench(ctx, buffer_bytes: int, record_bytes: int) -> float:
@@ -374,6 +386,10 @@ class Tracker:
         out = np.empty(n, np.uint32)
         pt_get_connectivity(self.ctx, out.ctypes.data, n)
         return out
+
+    def set_segments(self, intervals) -> None:
+        """Schedule of the PT_KERNEL_SEGMENTED ablation (the paper's NumIteration[])."""
+        pt_set_segments(self.ctx, intervals)
 
     def gather_bench(self, buffer_bytes: int, record_bytes: int) -> float:
         self._stream()

@@ -10,7 +10,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.environ.get("PT_LIB") or os.path.join(PKG, "libpt.so")  # PT_LIB: experiment builds
-SOURCES = ["pt_api.cu", "pt_kernels.cu", "pt_variants.cu", "pt_mcmc.cu"]
+SOURCES = ["pt_api.cu", "pt_kernels.cu", "pt_variants.cu", "pt_mcmc.cu", "pt_segmented.cu"]
 HEADERS = ["pt_device.cuh", "pt_internal.h", "pt_claim.cuh"]
 
 NVCC_FLAGS = [
@@ -47,7 +47,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [nvcc(), *NVCC_FLAGS, "-I", INCLUDE, "-o", tmp, *[os.path.join(CSRC, s) for s in SOURCES]]
+    extra = os.environ.get("PT_NVCC_EXTRA", "").split()  # experiment builds: -D overrides
+    cmd = [nvcc(), *NVCC_FLAGS, *extra, "-I", INCLUDE, "-o", tmp, *[os.path.join(CSRC, s) for s in SOURCES]]
     if verbose:
         print(" ".join(cmd))
     subprocess.check_call(cmd)

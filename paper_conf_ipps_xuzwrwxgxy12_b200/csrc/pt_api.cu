@@ -78,6 +78,11 @@ struct pt_ctx {
     size_t mtemp_cap = 0;
     uint32_t* d_mcount = nullptr;   // [0] = selected voxels, [1] = work queue
     bool mcmc_done = false;
+    // ablation (ii): segmented relaunch
+    int32_t seg_sched[64] = {1, 2, 5, 10, 20, 50, 100, 200, 500};
+    int32_t seg_n = 9;
+    uint8_t* d_seg = nullptr;       // SegState arrays + second live list + select temp
+    size_t seg_cap = 0;
     uint64_t m_voxels = 0, m_steps = 0;
     // last call
     bool tracked = false;
@@ -224,7 +229,7 @@ void pt_destroy(pt_ctx* c) {
     else cudaDeviceSynchronize();
     void* bufs[] = {c->d_rec, c->d_mask, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_copies, c->d_labels, c->d_conn, c->d_nsteps,
                     c->d_reason, c->d_end, c->d_paths, c->d_stats, c->d_mstats, c->d_mvox, c->d_mflags,
-                    c->d_mtemp, c->d_mcount};
+                    c->d_mtemp, c->d_mcount, c->d_seg};
     for (void* b : bufs)
         if (b) cudaFree(b);
     for (auto& ev : c->ev)
@@ -352,6 +357,9 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     const uint64_t npart = N * P;
     const uint32_t kVariantFlags = PT_BIDIR | PT_INTERP | PT_INIT_RANDOM | PT_INIT_FWEIGHT | PT_KERNEL_VARIANT;
     const bool variant = (p->flags & kVariantFlags) != 0;
+    const bool segmented = (p->flags & PT_KERNEL_SEGMENTED) != 0;
+    if (segmented && (variant || (p->flags & (PT_KERNEL_SIMPLE | PT_REC_PATHS | PT_REC_CONN))))
+        return fail(c, PT_ERR_ARG, "pt_track: PT_KERNEL_SEGMENTED runs the base semantics with nsteps/reason/end outputs only");
     if (variant && (p->flags & PT_KERNEL_SIMPLE))
         return fail(c, PT_ERR_ARG, "pt_track: PT_KERNEL_SIMPLE cannot run the NEXT-3 variants");
     if ((p->flags & PT_INIT_RANDOM) && (p->flags & PT_INIT_FWEIGHT))
@@ -508,8 +516,35 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.init_mode = (fl & PT_INIT_RANDOM) ? 1u : ((fl & PT_INIT_FWEIGHT) ? 2u : 0u);
     a.mask = c->d_mask;
 
-    CK(cudaEventRecord(c->ev[1], st), "pt_track: event");
-    if (variant)
+    if (!segmented) CK(cudaEventRecord(c->ev[1], st), "pt_track: event");
+    if (segmented) {
+        const uint32_t batch = (uint32_t)(npart < (1ull << 26) ? (npart ? npart : 1) : (1ull << 26));
+        const size_t tb = pt::seg_select_temp_bytes(batch);
+        const size_t per = 12 + 12 + 4 + 4 + 8 + 8 + 4 + 1 + 4;  // q p n vox pid li live flag live_b
+        CK(ensure(c->d_seg, c->seg_cap, (size_t)batch * per + tb + 256 + 64), "pt_track: segment state");
+        uint8_t* b = c->d_seg;
+        auto take = [&](size_t bytes) {
+            uint8_t* r = b;
+            b += (bytes + 15) / 16 * 16;
+            return r;
+        };
+        pt::SegState ss;
+        ss.q = reinterpret_cast<float*>(take((size_t)batch * 12));
+        ss.p = reinterpret_cast<float*>(take((size_t)batch * 12));
+        ss.pid = reinterpret_cast<uint64_t*>(take((size_t)batch * 8));
+        ss.li = reinterpret_cast<uint64_t*>(take((size_t)batch * 8));
+        ss.n = reinterpret_cast<uint32_t*>(take((size_t)batch * 4));
+        ss.vox = reinterpret_cast<uint32_t*>(take((size_t)batch * 4));
+        ss.live = reinterpret_cast<uint32_t*>(take((size_t)batch * 4));
+        uint32_t* live_b = reinterpret_cast<uint32_t*>(take((size_t)batch * 4));
+        uint32_t* d_count = reinterpret_cast<uint32_t*>(take(16));
+        ss.flag = take((size_t)batch);
+        void* temp = take(tb);
+        CK(cudaEventRecord(c->ev[1], st), "pt_track: event");
+        CK(pt::run_segmented(a, c->vol.nfibres, c->vol.dtype == PT_F16, ss, batch, c->seg_sched, c->seg_n, live_b,
+                             d_count, temp, tb, st),
+           "pt_track: segmented relaunch");
+    } else if (variant)
         CK(pt::launch_track_var(a, c->vol.nfibres, c->vol.dtype == PT_F16, c->num_sms, st),
            "pt_track: variant tracking kernel launch");
     else
@@ -531,6 +566,17 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     c->last_stride = (fl & PT_REC_PATHS) ? p->path_stride : 0;
     c->last_map = d_map != nullptr;
     c->last_conn_count = want_conn ? N * (uint64_t)c->ntargets : 0;
+    return PT_OK;
+}
+
+pt_status pt_set_segments(pt_ctx* c, const int32_t* intervals, int32_t n) {
+    if (!c) return PT_ERR_ARG;
+    c->err.clear();
+    if (!intervals || n < 1 || n > 64) return fail(c, PT_ERR_ARG, "pt_set_segments: need 1..64 intervals");
+    for (int32_t i = 0; i < n; ++i)
+        if (intervals[i] < 1) return fail(c, PT_ERR_ARG, "pt_set_segments: interval %d < 1", i);
+    for (int32_t i = 0; i < n; ++i) c->seg_sched[i] = intervals[i];
+    c->seg_n = n;
     return PT_OK;
 }
 

@@ -105,6 +105,23 @@ cudaError_t launch_mcmc(const McmcArgs& a, int num_sms, cudaStream_t st);
 cudaError_t launch_samples_to_volume(const double* samples, const uint8_t* mask, uint64_t V, int N, int S,
                                      float* dyads, float* f, cudaStream_t st);
 
+// Ablation (ii): segmented relaunch with device compaction (pt_segmented.cu).  State of a
+// batch of particles, SoA; live / flag are indexed by list position.
+struct SegState {
+    float* q;        // [batch][3] position (centred)
+    float* p;        // [batch][3] previous direction
+    uint32_t* n;     // [batch] committed steps
+    uint32_t* vox;   // [batch] voxel of q
+    uint64_t* pid;   // [batch] RNG particle id
+    uint64_t* li;    // [batch] output index (seed index * P + j)
+    uint32_t* live;  // [batch] live list (identity after init)
+    uint8_t* flag;   // [batch] alive flag per list position
+};
+size_t seg_select_temp_bytes(uint32_t n);
+cudaError_t run_segmented(const TrackArgs& a, int F, bool half, const SegState& s, uint32_t batch,
+                          const int32_t* schedule, int nsched, uint32_t* live_b, uint32_t* d_count, void* temp,
+                          size_t temp_bytes, cudaStream_t st);
+
 // Launchers (return the launch error, if any).
 cudaError_t launch_track(const TrackArgs& a, int nfibres, bool half, bool simple, int num_sms,
                          cudaStream_t st);

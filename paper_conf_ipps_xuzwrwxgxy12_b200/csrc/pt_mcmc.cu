@@ -32,6 +32,9 @@ namespace {
 constexpr uint32_t kTag = 0x4D434D43u;  // "MCMC": Philox counter word 3 (M6)
 constexpr double kTwoPi = 6.283185307179586;
 constexpr int kMcmcThreads = 128;         // 4 voxels (warps) per CTA
+#ifndef PT_MCMC_MIN_BLOCKS
+#define PT_MCMC_MIN_BLOCKS 4  // CTAs per SM the register budget must allow (16 warps)
+#endif
 
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
@@ -40,7 +43,7 @@ __device__ __forceinline__ double warp_sum(double v) {
 }
 
 template <int N, int MPL>
-__global__ void __launch_bounds__(kMcmcThreads) mcmc_kernel(const __grid_constant__ McmcArgs a) {
+__global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(const __grid_constant__ McmcArgs a) {
     constexpr int NP = 3 + 3 * N;
     const uint32_t lane = threadIdx.x & 31u;
     const int n = a.nmeas;
@@ -171,9 +174,13 @@ __global__ void __launch_bounds__(kMcmcThreads) mcmc_kernel(const __grid_constan
 
         // ------------------------------------------------ per-measurement caches (Eq. 1)
         double e0[MPL], ej[N][MPL], dj[N][MPL], A[MPL];
+        double fj[N];
         double sumf = 0.0;
 #pragma unroll
-        for (int j = 0; j < N; ++j) sumf = sumf + w[3 + 3 * j];
+        for (int j = 0; j < N; ++j) {
+            fj[j] = w[3 + 3 * j];
+            sumf = sumf + fj[j];
+        }
         double sse = 0.0;
 #pragma unroll
         for (int m = 0; m < MPL; ++m) {
@@ -186,7 +193,7 @@ __global__ void __launch_bounds__(kMcmcThreads) mcmc_kernel(const __grid_constan
                 const double vx = sth[j] * cph[j], vy = sth[j] * sph[j], vz = cth[j];
                 dj[j][m] = ((double)rx[m] * vx + (double)ry[m] * vy) + (double)rz[m] * vz;
                 ej[j][m] = exp(-(bd * (dj[j][m] * dj[j][m])));
-                acc = acc + w[3 + 3 * j] * ej[j][m];
+                acc = acc + fj[j] * ej[j][m];
             }
             A[m] = acc;
             const double r = (double)yf[m] - w[0] * acc;
@@ -198,25 +205,35 @@ __global__ void __launch_bounds__(kMcmcThreads) mcmc_kernel(const __grid_constan
             if (!(sig >= 1e-3 * w[0])) sig = 1e-3 * w[0];
             w[2] = sig;
         }
-        double lsig = log(w[2]);
-        double lp = -np1 * lsig - sse / (2.0 * w[2] * w[2]);
+        // uniform copies of the parameters the likelihood needs every step
+        double S0 = w[0], dd = w[1], sig = w[2];
+        double lsig = log(sig);
+        double lp = -np1 * lsig - sse / (2.0 * sig * sig);
 #pragma unroll
         for (int j = 0; j < N; ++j) lp = lp + lsin[j];
 
-        // ------------------------------------------------ proposals (M8)
-        double prop[NP];
-        prop[0] = 0.01 * w[0];
-        prop[1] = 0.1 * w[1];
-        prop[2] = 0.1 * w[2];
+        // ------------------------------------------------ lane k owns parameter k: its value,
+        // proposal width (M8), acceptance counters and, for angles, sin / cos (/ ln|sin|)
+        double my_w = w[0];
+#pragma unroll
+        for (int k = 1; k < NP; ++k) my_w = lane == (uint32_t)k ? w[k] : my_w;
+        double my_prop = 0.1;
+        if (lane == 0u) my_prop = 0.01 * S0;
+        else if (lane == 1u) my_prop = 0.1 * dd;
+        else if (lane == 2u) my_prop = 0.1 * sig;
+        else if (lane >= 3u && (lane - 3u) % 3u == 0u) my_prop = 0.05;
+        double my_s = 0.0, my_c = 0.0;  // angle lanes: sin, cos of the current value
 #pragma unroll
         for (int j = 0; j < N; ++j) {
-            prop[3 + 3 * j] = 0.05;
-            prop[4 + 3 * j] = 0.1;
-            prop[5 + 3 * j] = 0.1;
+            if (lane == (uint32_t)(4 + 3 * j)) {
+                my_s = sth[j];
+                my_c = cth[j];
+            } else if (lane == (uint32_t)(5 + 3 * j)) {
+                my_s = sph[j];
+                my_c = cph[j];
+            }
         }
-        uint32_t acc[NP], rej[NP], tot[NP];
-#pragma unroll
-        for (int k = 0; k < NP; ++k) acc[k] = rej[k] = tot[k] = 0u;
+        uint32_t my_acc = 0u, my_rej = 0u, my_tot = 0u;
 
         const uint32_t loops = a.loops;
         for (uint32_t t = 0; t < loops; ++t) {
@@ -229,22 +246,14 @@ __global__ void __launch_bounds__(kMcmcThreads) mcmc_kernel(const __grid_constan
                 const double u3 = ((double)R.z + 0.5) * 0x1p-32;
                 const double z = sqrt(-2.0 * log(u1)) * cos(kTwoPi * u2);
                 clu = log(u3);
-                double wk = w[0], pk = prop[0];
-#pragma unroll
-                for (int k = 1; k < NP; ++k) {
-                    wk = lane == (uint32_t)k ? w[k] : wk;
-                    pk = lane == (uint32_t)k ? prop[k] : pk;
-                }
-                cz = wk + pk * z;
+                cz = my_w + my_prop * z;
                 if (lane == 2u) {
                     ca = log(cz);
                 } else if (lane >= 3u) {
                     const uint32_t r3 = (lane - 3u) % 3u;
-                    if (r3 == 1u) {  // theta: sin, cos, ln|sin|
+                    if (r3 != 0u) {  // theta / phi: sin, cos (theta: and ln|sin|)
                         sincos(cz, &ca, &cb);
-                        cc = log(fabs(ca));
-                    } else if (r3 == 2u) {  // phi: sin, cos
-                        sincos(cz, &ca, &cb);
+                        if (r3 == 1u) cc = log(fabs(ca));
                     }
                 }
             }
@@ -254,36 +263,46 @@ __global__ void __launch_bounds__(kMcmcThreads) mcmc_kernel(const __grid_constan
                 if (a.fixed & (1u << k)) continue;
                 const double cand = __shfl_sync(kFull, cz, k);
                 const double lu = __shfl_sync(kFull, clu, k);
-                const double xa = __shfl_sync(kFull, ca, k);
-                const double xb = __shfl_sync(kFull, cb, k);
-                const double xc = __shfl_sync(kFull, cc, k);
+                const int jf = k >= 3 ? (k - 3) / 3 : 0;       // fibre of an f/theta/phi step
+                const int r3 = k >= 3 ? (k - 3) % 3 : -1;      // 0 f, 1 theta, 2 phi
                 // support (M3)
                 bool ok;
                 double nsumf = sumf;
-                if (k == 0 || k == 1 || k == 2) {
+                if (k < 3) {
                     ok = cand > 0.0;
-                } else if ((k - 3) % 3 == 0) {
+                } else if (r3 == 0) {
                     nsumf = 0.0;
 #pragma unroll
-                    for (int j = 0; j < N; ++j) nsumf = nsumf + (3 + 3 * j == k ? cand : w[3 + 3 * j]);
+                    for (int j = 0; j < N; ++j) nsumf = nsumf + (j == jf ? cand : fj[j]);
                     ok = cand >= 0.0 && nsumf <= 1.0;
                 } else {
                     ok = true;
                 }
                 if (!ok) {
-                    rej[k] += 1u;
+                    if (lane == (uint32_t)k) my_rej += 1u;
                     continue;
                 }
-                const int jf = k >= 3 ? (k - 3) / 3 : 0;  // fibre of an f/theta/phi step
+                double xa = 0.0, xb = 0.0, xc = 0.0;  // the candidate's by-products (lane k)
                 double nvx = 0.0, nvy = 0.0, nvz = 0.0;
-                if (k >= 3 && (k - 3) % 3 == 1) {  // theta' with the current phi
-                    nvx = xa * cph[jf];
-                    nvy = xa * sph[jf];
-                    nvz = xb;
-                } else if (k >= 3 && (k - 3) % 3 == 2) {  // phi' with the current theta
-                    nvx = sth[jf] * xb;
-                    nvy = sth[jf] * xa;
-                    nvz = cth[jf];
+                if (k == 2) {
+                    xa = __shfl_sync(kFull, ca, k);
+                } else if (r3 == 1 || r3 == 2) {
+                    xa = __shfl_sync(kFull, ca, k);
+                    xb = __shfl_sync(kFull, cb, k);
+                    // the fibre's other angle, current value, from its owner lane
+                    const int other = r3 == 1 ? k + 1 : k - 1;
+                    const double os = __shfl_sync(kFull, my_s, other);
+                    const double oc = __shfl_sync(kFull, my_c, other);
+                    if (r3 == 1) {  // theta' with the current phi
+                        xc = __shfl_sync(kFull, cc, k);
+                        nvx = xa * oc;
+                        nvy = xa * os;
+                        nvz = xb;
+                    } else {        // phi' with the current theta
+                        nvx = os * xb;
+                        nvy = os * xa;
+                        nvz = oc;
+                    }
                 }
                 double nsse = 0.0, nlp;
                 double ne[MPL], nd[MPL], nA[MPL], nej[N][MPL];
@@ -304,108 +323,100 @@ __global__ void __launch_bounds__(kMcmcThreads) mcmc_kernel(const __grid_constan
 #pragma unroll
                             for (int j = 0; j < N; ++j) {
                                 nej[j][m] = exp(-(bd * (dj[j][m] * dj[j][m])));
-                                accm = accm + w[3 + 3 * j] * nej[j][m];
+                                accm = accm + fj[j] * nej[j][m];
                             }
                             nA[m] = accm;
-                            mu = w[0] * accm;
-                        } else if ((k - 3) % 3 == 0) {
+                            mu = S0 * accm;
+                        } else if (r3 == 0) {
                             double accm = (1.0 - nsumf) * e0[m];
 #pragma unroll
-                            for (int j = 0; j < N; ++j) accm = accm + (j == jf ? cand : w[3 + 3 * j]) * ej[j][m];
+                            for (int j = 0; j < N; ++j) accm = accm + (j == jf ? cand : fj[j]) * ej[j][m];
                             nA[m] = accm;
-                            mu = w[0] * accm;
+                            mu = S0 * accm;
                         } else {
-                            const double bd = (double)bf[m] * w[1];
+                            const double bd = (double)bf[m] * dd;
                             nd[m] = ((double)rx[m] * nvx + (double)ry[m] * nvy) + (double)rz[m] * nvz;
                             ne[m] = exp(-(bd * (nd[m] * nd[m])));
                             double accm = (1.0 - sumf) * e0[m];
 #pragma unroll
-                            for (int j = 0; j < N; ++j) accm = accm + w[3 + 3 * j] * (j == jf ? ne[m] : ej[j][m]);
+                            for (int j = 0; j < N; ++j) accm = accm + fj[j] * (j == jf ? ne[m] : ej[j][m]);
                             nA[m] = accm;
-                            mu = w[0] * accm;
+                            mu = S0 * accm;
                         }
                         const double r = (double)yf[m] - mu;
                         nsse += valid[m] ? r * r : 0.0;
                     }
                     nsse = warp_sum(nsse);
-                    nlp = -np1 * lsig - nsse / (2.0 * w[2] * w[2]);
+                    nlp = -np1 * lsig - nsse / (2.0 * sig * sig);
 #pragma unroll
-                    for (int j = 0; j < N; ++j) nlp = nlp + ((k >= 3 && (k - 3) % 3 == 1 && j == jf) ? xc : lsin[j]);
+                    for (int j = 0; j < N; ++j) nlp = nlp + ((r3 == 1 && j == jf) ? xc : lsin[j]);
                 }
                 // accept with probability min(r, 1): ln u < lp' - lp
-                if (lu < nlp - lp) {
-                    acc[k] += 1u;
-                    tot[k] += 1u;
-                    w[k] = cand;
+                const bool accept = lu < nlp - lp;
+                if (lane == (uint32_t)k) {
+                    my_acc += accept ? 1u : 0u;
+                    my_tot += accept ? 1u : 0u;
+                    my_rej += accept ? 0u : 1u;
+                    if (accept) {
+                        my_w = cz;
+                        my_s = ca;
+                        my_c = cb;
+                    }
+                }
+                if (accept) {
                     lp = nlp;
-                    if (k == 2) {
+                    if (k == 0) {
+                        S0 = cand;
+                        sse = nsse;
+                    } else if (k == 1) {
+                        dd = cand;
+                        sse = nsse;
+#pragma unroll
+                        for (int m = 0; m < MPL; ++m) {
+                            e0[m] = ne[m];
+#pragma unroll
+                            for (int j = 0; j < N; ++j) ej[j][m] = nej[j][m];
+                            A[m] = nA[m];
+                        }
+                    } else if (k == 2) {
+                        sig = cand;
                         lsig = xa;
                     } else {
                         sse = nsse;
-                        if (k == 1) {
+                        if (r3 == 0) {
+                            fj[jf] = cand;
+                            sumf = nsumf;
+                        } else if (r3 == 1) {
+                            lsin[jf] = xc;
+                        }
 #pragma unroll
-                            for (int m = 0; m < MPL; ++m) {
-                                e0[m] = ne[m];
-#pragma unroll
-                                for (int j = 0; j < N; ++j) ej[j][m] = nej[j][m];
-                                A[m] = nA[m];
+                        for (int m = 0; m < MPL; ++m) {
+                            A[m] = nA[m];
+                            if (r3 != 0) {
+                                dj[jf][m] = nd[m];
+                                ej[jf][m] = ne[m];
                             }
-                        } else if (k >= 3) {
-                            const int r3 = (k - 3) % 3;
-                            if (r3 == 0) {
-                                sumf = nsumf;
-                            } else if (r3 == 1) {
-                                sth[jf] = xa;
-                                cth[jf] = xb;
-                                lsin[jf] = xc;
-                            } else {
-                                sph[jf] = xa;
-                                cph[jf] = xb;
-                            }
-#pragma unroll
-                            for (int m = 0; m < MPL; ++m) {
-                                A[m] = nA[m];
-                                if (r3 != 0) {
-                                    dj[jf][m] = nd[m];
-                                    ej[jf][m] = ne[m];
-                                }
-                            }
-                        } else {
-                            // S0: A unchanged
                         }
                     }
-                } else {
-                    rej[k] += 1u;
                 }
             }
-            // Fig. 2: every K loops the acceptance rates update the proposals (M8)
+            // Fig. 2: every K loops the acceptance rates update the proposals (M8); lane k
+            // updates its own parameter's width
             if ((t + 1u) % a.adapt_every == 0u) {
-#pragma unroll
-                for (int k = 0; k < NP; ++k) {
-                    prop[k] = prop[k] * sqrt((5.0 * (double)(acc[k] + 1u)) / (3.0 * (double)(rej[k] + 1u)));
-                    acc[k] = rej[k] = 0u;
-                }
+                my_prop = my_prop * sqrt((5.0 * (double)(my_acc + 1u)) / (3.0 * (double)(my_rej + 1u)));
+                my_acc = my_rej = 0u;
             }
             // samples after the burn-in, every L loops; lane k writes omega_k
             if (t >= a.burnin && (t - a.burnin + 1u) % a.interval == 0u) {
                 const uint32_t s = (t - a.burnin + 1u) / a.interval - 1u;
-                double wk = w[0];
-#pragma unroll
-                for (int k = 1; k < NP; ++k) wk = lane == (uint32_t)k ? w[k] : wk;
-                if (lane < (uint32_t)NP) a.samples[((uint64_t)lane * a.nsamples + s) * V + v] = wk;
+                if (lane < (uint32_t)NP) a.samples[((uint64_t)lane * a.nsamples + s) * V + v] = my_w;
             }
         }
-        if (a.accepted) {
-            uint32_t tk = tot[0];
-#pragma unroll
-            for (int k = 1; k < NP; ++k) tk = lane == (uint32_t)k ? tot[k] : tk;
-            if (lane < (uint32_t)NP) a.accepted[(uint64_t)lane * V + v] = tk;
-        }
-        if (lane == 0) {
-#pragma unroll
-            for (int k = 0; k < NP; ++k) acc_tot += tot[k];
-        }
+        if (a.accepted && lane < (uint32_t)NP) a.accepted[(uint64_t)lane * V + v] = my_tot;
+        if (lane < (uint32_t)NP) acc_tot += my_tot;
     }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acc_tot += __shfl_xor_sync(kFull, acc_tot, o);
     if (lane == 0 && acc_tot) atomicAdd(a.stats + kMcmcStatAccepted, acc_tot);
 }
 

@@ -584,7 +584,18 @@ MCMC_CONFIGS = {
     "m1": lambda: dwi_brain(96, 96, 48, scale=0.96, gen_seed=43),
     "m2": lambda: dwi_brain(102, 102, 60, scale=1.0803, gen_seed=41),
     "m_small": lambda: dwi_brain(24, 24, 16, scale=1.0, gen_seed=47, burnin=100, nsamples=10),
+    # profiling subset of m2 (every 8th valid voxel): same per-voxel work, 1/8 of the voxels
+    "m2_prof": lambda: mcmc_subset(dwi_brain(102, 102, 60, scale=1.0803, gen_seed=41), 8),
 }
+
+
+def mcmc_subset(d: DwiWorkload, every: int) -> DwiWorkload:
+    """Every ``every``-th valid voxel of a DWI workload (profiling / CPU samples)."""
+    m = d.mask.ravel().copy()
+    idx = np.flatnonzero(m)
+    m[:] = 0
+    m[idx[::every]] = 1
+    return d.replace(mask=m.reshape(d.mask.shape), name=d.name + f"_every{every}")
 
 
 def mcmc_config(name: str) -> DwiWorkload:

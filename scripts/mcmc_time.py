@@ -1,5 +1,6 @@
 """Quick timing of pt_mcmc on an MCMC config (diagnostic; bench.py --config m2 is the bench line)."""
-import sys, time
+import os, sys, time
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
 import phantom
 import paper_conf_ipps_xuzwrwxgxy12_b200 as pt
