@@ -132,6 +132,16 @@ class ClockSampler:
 
 # ----------------------------------------------------------------------------- helpers
 
+def _cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
 def _peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -238,13 +248,10 @@ def _fp64_peak():
 
 def _mcmc_shard(d, rank, world):
     """Voxel v -> rank v mod N (results are keyed by the voxel index, so exact)."""
-    import numpy as np
+    from paper_conf_ipps_xuzwrwxgxy12_b200 import sharding
     if world == 1:
         return d
-    m = d.mask.copy().ravel()
-    idx = np.arange(m.size)
-    m[idx % world != rank] = 0
-    return d.replace(mask=m.reshape(d.mask.shape))
+    return d.replace(mask=sharding.shard_voxels(d.mask, rank, world))
 
 
 def run_mcmc(args):
@@ -340,7 +347,7 @@ def run_mcmc(args):
         t1 = time.perf_counter()
         oracle.mcmc(d, voxels=pick, threads=threads)
         dt = time.perf_counter() - t1
-        cpu = {"value": pick.size / dt, "unit": "voxels/s", "cores": threads, "kind": "oracle",
+        cpu = {"value": pick.size / dt, "unit": "voxels/s", "cores": threads, "kind": "oracle", "cpu_model": _cpu_model(),
                "sample": f"every {max(1, idx.size // nv)}th valid voxel ({pick.size} voxels) in {dt:.1f} s"}
     if rank == 0:
         line = {
@@ -574,7 +581,7 @@ def run_ours(args):
         threads = len(os.sched_getaffinity(0))
         sub, J, every = _cpu_sample(w, args.cpu_seconds, threads)
         s, dt = _run_oracle_sample(sub, J, threads)
-        cpu = {"value": s / dt, "unit": "steps/s", "cores": threads, "kind": "oracle",
+        cpu = {"value": s / dt, "unit": "steps/s", "cores": threads, "kind": "oracle", "cpu_model": _cpu_model(),
                "sample": f"every {every}th WM seed ({sub.nseeds} seeds) x particles j<{J}: "
                          f"{s} steps in {dt:.1f} s"}
 

@@ -36,6 +36,19 @@ constexpr int kMcmcThreads = 128;         // 4 voxels (warps) per CTA
 #define PT_MCMC_MIN_BLOCKS 4  // CTAs per SM the register budget must allow (16 warps)
 #endif
 
+#ifndef PT_MCMC_FMA
+#define PT_MCMC_FMA 1  // contract a*b+c into DFMA in the per-measurement terms
+#endif
+// a * b + c: one fused DFMA (PT_MCMC_FMA) or a rounded product and a rounded sum (the
+// oracle's order; the library is built with -fmad=false, so only this helper fuses)
+__device__ __forceinline__ double madd(double a, double b, double c) {
+#if PT_MCMC_FMA
+    return __fma_rn(a, b, c);
+#else
+    return a * b + c;
+#endif
+}
+
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
@@ -191,13 +204,13 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
 #pragma unroll
             for (int j = 0; j < N; ++j) {
                 const double vx = sth[j] * cph[j], vy = sth[j] * sph[j], vz = cth[j];
-                dj[j][m] = ((double)rx[m] * vx + (double)ry[m] * vy) + (double)rz[m] * vz;
+                dj[j][m] = madd((double)rz[m], vz, madd((double)ry[m], vy, (double)rx[m] * vx));
                 ej[j][m] = exp(-(bd * (dj[j][m] * dj[j][m])));
-                acc = acc + fj[j] * ej[j][m];
+                acc = madd(fj[j], ej[j][m], acc);
             }
             A[m] = acc;
             const double r = (double)yf[m] - w[0] * acc;
-            sse += valid[m] ? r * r : 0.0;
+            sse = valid[m] ? madd(r, r, sse) : sse;
         }
         sse = warp_sum(sse);
         if (!a.init) {
@@ -234,18 +247,29 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
             }
         }
         uint32_t my_acc = 0u, my_rej = 0u, my_tot = 0u;
+        double bz = 0.0, blu = 0.0;  // batched draws (lanes < B * NP)
 
         const uint32_t loops = a.loops;
         for (uint32_t t = 0; t < loops; ++t) {
-            // lane k < NP: draw k of this loop (M6), candidate omega'_k and its by-products
-            double cz = 0.0, clu = 0.0, ca = 0.0, cb = 0.0, cc = 0.0;
-            if (lane < (uint32_t)NP) {
-                const uint4 R = philox4x32_10(make_uint4(t, v, lane, kTag), a.key0, a.key1);
+            // The draws (M6) do not depend on the state: every B = 32 / NP loops, lane
+            // i*NP + k computes draw k of loop t + i (up to 32 draws per batch).
+            constexpr int B = 32 / NP;
+            const uint32_t ph = t % (uint32_t)B;
+            if (ph == 0u && lane < (uint32_t)(B * NP)) {
+                const uint32_t tt = t + lane / (uint32_t)NP, kk = lane % (uint32_t)NP;
+                const uint4 R = philox4x32_10(make_uint4(tt, v, kk, kTag), a.key0, a.key1);
                 const double u1 = ((double)R.x + 0.5) * 0x1p-32;
                 const double u2 = (double)R.y * 0x1p-32;
                 const double u3 = ((double)R.z + 0.5) * 0x1p-32;
-                const double z = sqrt(-2.0 * log(u1)) * cos(kTwoPi * u2);
-                clu = log(u3);
+                bz = sqrt(-2.0 * log(u1)) * cos(kTwoPi * u2);
+                blu = log(u3);
+            }
+            // lane k < NP: draw k of this loop, candidate omega'_k and its by-products
+            const uint32_t src = ph * (uint32_t)NP + (lane < (uint32_t)NP ? lane : 0u);
+            const double z = __shfl_sync(kFull, bz, src);
+            const double clu = __shfl_sync(kFull, blu, src);
+            double cz = 0.0, ca = 0.0, cb = 0.0, cc = 0.0;
+            if (lane < (uint32_t)NP) {
                 cz = my_w + my_prop * z;
                 if (lane == 2u) {
                     ca = log(cz);
@@ -323,28 +347,28 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
 #pragma unroll
                             for (int j = 0; j < N; ++j) {
                                 nej[j][m] = exp(-(bd * (dj[j][m] * dj[j][m])));
-                                accm = accm + fj[j] * nej[j][m];
+                                accm = madd(fj[j], nej[j][m], accm);
                             }
                             nA[m] = accm;
                             mu = S0 * accm;
                         } else if (r3 == 0) {
                             double accm = (1.0 - nsumf) * e0[m];
 #pragma unroll
-                            for (int j = 0; j < N; ++j) accm = accm + (j == jf ? cand : fj[j]) * ej[j][m];
+                            for (int j = 0; j < N; ++j) accm = madd(j == jf ? cand : fj[j], ej[j][m], accm);
                             nA[m] = accm;
                             mu = S0 * accm;
                         } else {
                             const double bd = (double)bf[m] * dd;
-                            nd[m] = ((double)rx[m] * nvx + (double)ry[m] * nvy) + (double)rz[m] * nvz;
+                            nd[m] = madd((double)rz[m], nvz, madd((double)ry[m], nvy, (double)rx[m] * nvx));
                             ne[m] = exp(-(bd * (nd[m] * nd[m])));
                             double accm = (1.0 - sumf) * e0[m];
 #pragma unroll
-                            for (int j = 0; j < N; ++j) accm = accm + fj[j] * (j == jf ? ne[m] : ej[j][m]);
+                            for (int j = 0; j < N; ++j) accm = madd(fj[j], j == jf ? ne[m] : ej[j][m], accm);
                             nA[m] = accm;
                             mu = S0 * accm;
                         }
                         const double r = (double)yf[m] - mu;
-                        nsse += valid[m] ? r * r : 0.0;
+                        nsse = valid[m] ? madd(r, r, nsse) : nsse;
                     }
                     nsse = warp_sum(nsse);
                     nlp = -np1 * lsig - nsse / (2.0 * sig * sig);

@@ -85,6 +85,7 @@ __global__ void __launch_bounds__(256) seg_kernel(const __grid_constant__ TrackA
     using R = Rec<F, HALF>;
     constexpr int RB = R::kBytes;
     unsigned long long my_steps = 0, my_done = 0;
+    uint32_t its = 0;  // loop iterations this lane ran (its SIMD occupancy)
     const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
     if (t < nlive) {
         const uint32_t i = live[t];
@@ -95,6 +96,7 @@ __global__ void __launch_bounds__(256) seg_kernel(const __grid_constant__ TrackA
         const uint64_t pid = s.pid[i];
         int why = -1;
         for (uint32_t it = 0; it < k; ++it) {
+            its += 1;
             if (n == a.max_steps) {  // P:L116, R14
                 why = kSMaxlen;
                 break;
@@ -172,11 +174,14 @@ __global__ void __launch_bounds__(256) seg_kernel(const __grid_constant__ TrackA
         my_steps += __shfl_xor_sync(kFull, my_steps, o);
         my_done += __shfl_xor_sync(kFull, my_done, o);
     }
+    // SIMD efficiency: a warp runs as long as its longest lane
+    const uint32_t its_sum = __reduce_add_sync(kFull, its);
+    const uint32_t its_max = __reduce_max_sync(kFull, its);
     if ((threadIdx.x & 31) == 0) {
         if (my_steps) atomicAdd(a.stats + kStatSteps, my_steps);
         if (my_done) atomicAdd(a.stats + kStatParticles, my_done);
-        atomicAdd(a.stats + kStatLaneActive, (unsigned long long)__popc(__ballot_sync(kFull, t < nlive)) * k);
-        atomicAdd(a.stats + kStatLaneSlots, 32ull * k);
+        atomicAdd(a.stats + kStatLaneActive, (unsigned long long)its_sum);
+        atomicAdd(a.stats + kStatLaneSlots, 32ull * its_max);
     }
 }
 

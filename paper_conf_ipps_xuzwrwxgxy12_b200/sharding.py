@@ -28,6 +28,35 @@ def shard_seeds(seeds: np.ndarray, seed_ids, rank: int, world: int):
     return np.ascontiguousarray(seeds[sel]), np.ascontiguousarray(ids[sel])
 
 
+def shard_voxels(mask: np.ndarray, rank: int, world: int) -> np.ndarray:
+    """MCMC (NEXT-4) sharding: voxel v -> rank v mod world.  The sampler's draws are keyed
+    by the linear voxel index (M6), so every rank's samples equal the single-GPU
+    ones; returns this rank's mask (uint8, same shape)."""
+    if world < 1 or not (0 <= rank < world):
+        raise ValueError(f"bad rank {rank} / world {world}")
+    m = np.ascontiguousarray(mask, np.uint8).copy()
+    flat = m.reshape(-1)
+    flat[np.arange(flat.size) % world != rank] = 0
+    return m
+
+
+def gather_samples(samples, dst: int = 0, group=None):
+    """Combine per-rank MCMC sample tensors (float64, zeros outside each rank's voxels) in
+    place with one reduce(SUM): each voxel is non-zero on exactly one rank, and x + 0 = x
+    exactly in IEEE arithmetic, so the result is bit-identical to the single-GPU samples."""
+    import torch.distributed as dist
+    if not dist.is_available() or not dist.is_initialized() or dist.get_world_size(group) == 1:
+        return samples
+    t = samples
+    staged = samples.is_cuda and dist.get_backend(group) == "gloo"
+    if staged:
+        t = samples.cpu()
+    dist.reduce(t, dst=dst, op=dist.ReduceOp.SUM, group=group)
+    if staged:
+        samples.copy_(t)
+    return samples
+
+
 def reduce_map(map_i32, dst: int = 0, group=None, all_ranks: bool = False):
     """Combine the ranks' maps in place: reduce to ``dst`` (or all-reduce) with SUM over
     the int32 view.  ``map_i32`` is a torch int32 tensor holding uint32 counts."""

@@ -32,3 +32,16 @@ def test_reference_arm_non_zero_rank_exits_quietly():
                           "--config", "c1", "--steps", "1", "--warmup", "1"],
                          capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
     assert out.returncode == 0 and out.stdout.strip() == ""
+
+
+def test_mcmc_reference_arm_json_line():
+    """The MCMC workload's reference arm (the MCMC oracle on a bounded voxel sample)."""
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference",
+                          "--config", "m_small", "--steps", "1", "--warmup", "1", "--cpu-seconds", "0.5"],
+                         capture_output=True, text=True, timeout=600, cwd=ROOT)
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [l for l in out.stdout.splitlines() if l.strip()]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["unit"] == "voxels/s" and d["value"] > 0
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["dtype"] == "f64"
