@@ -366,7 +366,7 @@ def run_mcmc(args):
             "e2e": {"value": voxels / float(te[0]), "unit": "voxels/s",
                     "h2d_bytes_per_step": int(d.dwi.nbytes + d.mask.nbytes + d.bvals.nbytes + d.bvecs.nbytes),
                     "d2h_bytes_per_step": int(out_h.numel() * 8)},
-            "gpu_launches": 3 * args.steps,
+            "gpu_launches": 4 * args.steps,  # mask flags, cub select (2), mcmc_kernel
             "clocks": ck,
         }
         print(json.dumps(line), flush=True)
@@ -667,7 +667,8 @@ def run_ours(args):
             "e2e": {"value": e2e_value, "unit": "steps/s",
                     "h2d_bytes_per_step": int(seeds_h.numel() * 4 + ids_h.numel() * 8),
                     "d2h_bytes_per_step": int(map_h.numel() * 4)},
-            "gpu_launches": 2 * args.steps,
+            # per pt_track: seed_keys + 6 cub radix-sort kernels (seed order), track_kernel, map_sum
+            "gpu_launches": 9 * args.steps,
             "clocks": ck,
         }
         print(json.dumps(line), flush=True)

@@ -31,7 +31,11 @@ namespace {
 
 constexpr uint32_t kTag = 0x4D434D43u;  // "MCMC": Philox counter word 3 (M6)
 constexpr double kTwoPi = 6.283185307179586;
-constexpr int kMcmcThreads = 128;         // 4 voxels (warps) per CTA
+constexpr int kMcmcThreads = 128;         // 4 warps per CTA
+constexpr int kMaxShells = 8;             // distinct b-values handled with one exp each
+#ifndef PT_MCMC_VPW
+#define PT_MCMC_VPW 2  // voxels per warp for nmeas <= 64 (1: one voxel per warp always)
+#endif
 #ifndef PT_MCMC_MIN_BLOCKS
 #define PT_MCMC_MIN_BLOCKS 4  // CTAs per SM the register budget must allow (16 warps)
 #endif
@@ -49,42 +53,83 @@ __device__ __forceinline__ double madd(double a, double b, double c) {
 #endif
 }
 
-__device__ __forceinline__ double warp_sum(double v) {
+// Sum over the LPV lanes of a voxel group (xor butterfly), then the group's first lane's
+// value for every lane of the group (the butterfly's lanes may differ in the last bit).
+template <int LPV>
+__device__ __forceinline__ double group_sum(double v) {
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
-    return __shfl_sync(kFull, v, 0);  // one value for every lane (the butterfly's lanes may differ)
+    for (int o = LPV / 2; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o, LPV);
+    return __shfl_sync(kFull, v, 0, LPV);
 }
 
-template <int N, int MPL>
+// VPW voxels per warp, LPV = 32 / VPW lanes per voxel, MPL measurements per lane.
+template <int N, int MPL, int VPW>
 __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(const __grid_constant__ McmcArgs a) {
     constexpr int NP = 3 + 3 * N;
+    constexpr int LPV = 32 / VPW;
+    static_assert(NP <= LPV, "a lane per parameter");
     const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t gl = lane % (uint32_t)LPV;   // lane within the voxel group
+    const uint32_t grp = lane / (uint32_t)LPV;  // voxel group within the warp
     const int n = a.nmeas;
     const double np1 = (double)(n + 1);
 
-    // per-measurement data (registers): i = lane + 32 m
-    bool valid[MPL];
-    float yf[MPL], bf[MPL], rx[MPL], ry[MPL], rz[MPL];
-#pragma unroll
-    for (int m = 0; m < MPL; ++m) {
-        const int i = (int)lane + 32 * m;
-        valid[m] = i < n;
-        bf[m] = valid[m] ? a.bvals[i] : 0.f;
-        rx[m] = valid[m] ? a.bvecs[3 * i] : 0.f;
-        ry[m] = valid[m] ? a.bvecs[3 * i + 1] : 0.f;
-        rz[m] = valid[m] ? a.bvecs[3 * i + 2] : 0.f;
+    // the gradient table (b, r) is the same for every voxel: shared memory, SoA (a lane
+    // reads entry gl + LPV m: distinct banks within a group, broadcast across groups);
+    // entries >= n are zero.  Measurement i of the voxel: i = gl + LPV m.
+    __shared__ float s_b[LPV * MPL], s_rx[LPV * MPL], s_ry[LPV * MPL], s_rz[LPV * MPL];
+    // the distinct b-values ("shells", <= kMaxShells) and each measurement's shell: a d
+    // proposal then needs one e^{-b d'} per shell instead of one per measurement
+    __shared__ float s_shell[kMaxShells];
+    __shared__ int s_sidx[LPV * MPL];
+    __shared__ int s_nshell;
+    for (int i = threadIdx.x; i < LPV * MPL; i += blockDim.x) {
+        const bool in = i < n;
+        s_b[i] = in ? a.bvals[i] : 0.f;
+        s_rx[i] = in ? a.bvecs[3 * i] : 0.f;
+        s_ry[i] = in ? a.bvecs[3 * i + 1] : 0.f;
+        s_rz[i] = in ? a.bvecs[3 * i + 2] : 0.f;
     }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int ns = 0;
+        for (int i = 0; i < LPV * MPL; ++i) {
+            int u = 0;
+            while (u < ns && s_shell[u] != s_b[i]) ++u;
+            if (u == ns) {
+                if (ns == kMaxShells) {
+                    ns = 0;  // too many shells: per-measurement exponentials
+                    break;
+                }
+                s_shell[ns++] = s_b[i];
+            }
+            s_sidx[i] = u;
+        }
+        s_nshell = ns;
+    }
+    __syncthreads();
+    const int nshell = s_nshell;
+#define BF(m) s_b[gl + LPV * (m)]
+#define RX(m) s_rx[gl + LPV * (m)]
+#define RY(m) s_ry[gl + LPV * (m)]
+#define RZ(m) s_rz[gl + LPV * (m)]
+    bool valid[MPL];
+    float yf[MPL];
+#pragma unroll
+    for (int m = 0; m < MPL; ++m) valid[m] = (int)gl + LPV * m < n;
     unsigned long long acc_tot = 0ull;
 
     for (;;) {
-        uint32_t slot = 0;
-        if (lane == 0) slot = atomicAdd(a.queue, 1u);
-        slot = __shfl_sync(kFull, slot, 0);
-        if (slot >= a.nvox) break;
-        const uint32_t v = a.vox[slot];
+        uint32_t base = 0;
+        if (lane == 0) base = atomicAdd(a.queue, (uint32_t)VPW);
+        base = __shfl_sync(kFull, base, 0);
+        if (base >= a.nvox) break;
+        const uint32_t slot = base + grp;
+        const bool gact = slot < a.nvox;  // a group without a voxel computes on base's, writes nothing
+        const uint32_t v = a.vox[gact ? slot : base];
         const uint64_t V = a.V;
 #pragma unroll
-        for (int m = 0; m < MPL; ++m) yf[m] = valid[m] ? a.dwi[(uint64_t)(lane + 32 * m) * V + v] : 0.f;
+        for (int m = 0; m < MPL; ++m) yf[m] = valid[m] ? a.dwi[(uint64_t)(gl + LPV * m) * V + v] : 0.f;
 
         double w[NP];
         double sth[N], cth[N], sph[N], cph[N], lsin[N];
@@ -100,23 +145,23 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
                 if (!valid[m]) continue;
                 const double y = (double)yf[m];
                 ymax = y > ymax ? y : ymax;
-                if (bf[m] == 0.f) {
+                if (BF(m) == 0.f) {
                     s0 += y;
                     c0 += 1;
                 } else {
                     sd += y;
-                    bsum += (double)bf[m];
+                    bsum += (double)BF(m);
                     cd += 1;
                 }
             }
-            s0 = warp_sum(s0);
-            sd = warp_sum(sd);
-            bsum = warp_sum(bsum);
+            s0 = group_sum<LPV>(s0);
+            sd = group_sum<LPV>(sd);
+            bsum = group_sum<LPV>(bsum);
 #pragma unroll
-            for (int o = 16; o > 0; o >>= 1) {
-                c0 += __shfl_xor_sync(kFull, c0, o);
-                cd += __shfl_xor_sync(kFull, cd, o);
-                ymax = fmax(ymax, __shfl_xor_sync(kFull, ymax, o));
+            for (int o = LPV / 2; o > 0; o >>= 1) {
+                c0 += __shfl_xor_sync(kFull, c0, o, LPV);
+                cd += __shfl_xor_sync(kFull, cd, o, LPV);
+                ymax = fmax(ymax, __shfl_xor_sync(kFull, ymax, o, LPV));
             }
             double S0 = c0 ? s0 / (double)c0 : ymax;
             if (!(S0 > 0.0)) S0 = 1.0;
@@ -134,23 +179,23 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
                 int bi = 0x7FFFFFFF;
 #pragma unroll
                 for (int m = 0; m < MPL; ++m) {
-                    bool ok = valid[m] && bf[m] != 0.f;
+                    bool ok = valid[m] && BF(m) != 0.f;
 #pragma unroll
                     for (int k = 0; k < j; ++k) {
-                        const double dot = ((double)rx[m] * (double)px[k] + (double)ry[m] * (double)py[k]) +
-                                           (double)rz[m] * (double)pz[k];
+                        const double dot = ((double)RX(m) * (double)px[k] + (double)RY(m) * (double)py[k]) +
+                                           (double)RZ(m) * (double)pz[k];
                         if (have[k]) ok = ok && fabs(dot) < 0.5;  // a missing pick constrains nothing
                     }
-                    const int i = (int)lane + 32 * m;
+                    const int i = (int)gl + LPV * m;
                     if (ok && (yf[m] < by || (yf[m] == by && i < bi))) {
                         by = yf[m];
                         bi = i;
                     }
                 }
 #pragma unroll
-                for (int o = 16; o > 0; o >>= 1) {
-                    const float oy = __shfl_xor_sync(kFull, by, o);
-                    const int oi = __shfl_xor_sync(kFull, bi, o);
+                for (int o = LPV / 2; o > 0; o >>= 1) {
+                    const float oy = __shfl_xor_sync(kFull, by, o, LPV);
+                    const int oi = __shfl_xor_sync(kFull, bi, o, LPV);
                     if (oy < by || (oy == by && oi < bi)) {
                         by = oy;
                         bi = oi;
@@ -186,7 +231,7 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
         }
 
         // ------------------------------------------------ per-measurement caches (Eq. 1)
-        double e0[MPL], ej[N][MPL], dj[N][MPL], A[MPL];
+        double e0[MPL], ej[N][MPL], dj[N][MPL];
         double fj[N];
         double sumf = 0.0;
 #pragma unroll
@@ -197,22 +242,21 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
         double sse = 0.0;
 #pragma unroll
         for (int m = 0; m < MPL; ++m) {
-            const double b = (double)bf[m];
+            const double b = (double)BF(m);
             const double bd = b * w[1];
             e0[m] = exp(-bd);
             double acc = (1.0 - sumf) * e0[m];
 #pragma unroll
             for (int j = 0; j < N; ++j) {
                 const double vx = sth[j] * cph[j], vy = sth[j] * sph[j], vz = cth[j];
-                dj[j][m] = madd((double)rz[m], vz, madd((double)ry[m], vy, (double)rx[m] * vx));
+                dj[j][m] = madd((double)RZ(m), vz, madd((double)RY(m), vy, (double)RX(m) * vx));
                 ej[j][m] = exp(-(bd * (dj[j][m] * dj[j][m])));
                 acc = madd(fj[j], ej[j][m], acc);
             }
-            A[m] = acc;
             const double r = (double)yf[m] - w[0] * acc;
             sse = valid[m] ? madd(r, r, sse) : sse;
         }
-        sse = warp_sum(sse);
+        sse = group_sum<LPV>(sse);
         if (!a.init) {
             double sig = sqrt(sse / (double)n);
             if (!(sig >= 1e-3 * w[0])) sig = 1e-3 * w[0];
@@ -221,7 +265,8 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
         // uniform copies of the parameters the likelihood needs every step
         double S0 = w[0], dd = w[1], sig = w[2];
         double lsig = log(sig);
-        double lp = -np1 * lsig - sse / (2.0 * sig * sig);
+        double inv2s2 = 1.0 / (2.0 * sig * sig);  // 1 / (2 sigma^2), refreshed when sigma moves
+        double lp = -np1 * lsig - sse * inv2s2;
 #pragma unroll
         for (int j = 0; j < N; ++j) lp = lp + lsin[j];
 
@@ -229,19 +274,19 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
         // proposal width (M8), acceptance counters and, for angles, sin / cos (/ ln|sin|)
         double my_w = w[0];
 #pragma unroll
-        for (int k = 1; k < NP; ++k) my_w = lane == (uint32_t)k ? w[k] : my_w;
+        for (int k = 1; k < NP; ++k) my_w = gl == (uint32_t)k ? w[k] : my_w;
         double my_prop = 0.1;
-        if (lane == 0u) my_prop = 0.01 * S0;
-        else if (lane == 1u) my_prop = 0.1 * dd;
-        else if (lane == 2u) my_prop = 0.1 * sig;
-        else if (lane >= 3u && (lane - 3u) % 3u == 0u) my_prop = 0.05;
+        if (gl == 0u) my_prop = 0.01 * S0;
+        else if (gl == 1u) my_prop = 0.1 * dd;
+        else if (gl == 2u) my_prop = 0.1 * sig;
+        else if (gl >= 3u && (gl - 3u) % 3u == 0u) my_prop = 0.05;
         double my_s = 0.0, my_c = 0.0;  // angle lanes: sin, cos of the current value
 #pragma unroll
         for (int j = 0; j < N; ++j) {
-            if (lane == (uint32_t)(4 + 3 * j)) {
+            if (gl == (uint32_t)(4 + 3 * j)) {
                 my_s = sth[j];
                 my_c = cth[j];
-            } else if (lane == (uint32_t)(5 + 3 * j)) {
+            } else if (gl == (uint32_t)(5 + 3 * j)) {
                 my_s = sph[j];
                 my_c = cph[j];
             }
@@ -253,10 +298,10 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
         for (uint32_t t = 0; t < loops; ++t) {
             // The draws (M6) do not depend on the state: every B = 32 / NP loops, lane
             // i*NP + k computes draw k of loop t + i (up to 32 draws per batch).
-            constexpr int B = 32 / NP;
+            constexpr int B = LPV / NP;
             const uint32_t ph = t % (uint32_t)B;
-            if (ph == 0u && lane < (uint32_t)(B * NP)) {
-                const uint32_t tt = t + lane / (uint32_t)NP, kk = lane % (uint32_t)NP;
+            if (ph == 0u && gl < (uint32_t)(B * NP)) {
+                const uint32_t tt = t + gl / (uint32_t)NP, kk = gl % (uint32_t)NP;
                 const uint4 R = philox4x32_10(make_uint4(tt, v, kk, kTag), a.key0, a.key1);
                 const double u1 = ((double)R.x + 0.5) * 0x1p-32;
                 const double u2 = (double)R.y * 0x1p-32;
@@ -265,28 +310,23 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
                 blu = log(u3);
             }
             // lane k < NP: draw k of this loop, candidate omega'_k and its by-products
-            const uint32_t src = ph * (uint32_t)NP + (lane < (uint32_t)NP ? lane : 0u);
-            const double z = __shfl_sync(kFull, bz, src);
-            const double clu = __shfl_sync(kFull, blu, src);
-            double cz = 0.0, ca = 0.0, cb = 0.0, cc = 0.0;
-            if (lane < (uint32_t)NP) {
-                cz = my_w + my_prop * z;
-                if (lane == 2u) {
-                    ca = log(cz);
-                } else if (lane >= 3u) {
-                    const uint32_t r3 = (lane - 3u) % 3u;
-                    if (r3 != 0u) {  // theta / phi: sin, cos (theta: and ln|sin|)
-                        sincos(cz, &ca, &cb);
-                        if (r3 == 1u) cc = log(fabs(ca));
-                    }
-                }
-            }
+            const uint32_t src = ph * (uint32_t)NP + (gl < (uint32_t)NP ? gl : 0u);
+            const double z = __shfl_sync(kFull, bz, src, LPV);
+            const double clu = __shfl_sync(kFull, blu, src, LPV);
+            // branch-free by-products (one sincos and one log per lane instead of a
+            // divergent branch per parameter kind): sigma lane: ca = ln sigma'; theta lanes:
+            // (sin, cos, ln|sin|); phi lanes: (sin, cos); the others' values are unused
+            const double cz = my_w + my_prop * z;
+            double sn, cs;
+            sincos(gl >= 3u ? cz : 0.0, &sn, &cs);
+            const double lx = log(gl == 2u ? cz : fabs(sn));
+            const double ca = gl == 2u ? lx : sn, cb = cs, cc = lx;
             // Fig. 2: the MH step, repeated NumParameters times
 #pragma unroll
             for (int k = 0; k < NP; ++k) {
                 if (a.fixed & (1u << k)) continue;
-                const double cand = __shfl_sync(kFull, cz, k);
-                const double lu = __shfl_sync(kFull, clu, k);
+                const double cand = __shfl_sync(kFull, cz, k, LPV);
+                const double lu = __shfl_sync(kFull, clu, k, LPV);
                 const int jf = k >= 3 ? (k - 3) / 3 : 0;       // fibre of an f/theta/phi step
                 const int r3 = k >= 3 ? (k - 3) % 3 : -1;      // 0 f, 1 theta, 2 phi
                 // support (M3)
@@ -302,23 +342,21 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
                 } else {
                     ok = true;
                 }
-                if (!ok) {
-                    if (lane == (uint32_t)k) my_rej += 1u;
-                    continue;
-                }
+                // (no early exit: the groups of a warp may disagree; a candidate outside the
+                // support is evaluated and then rejected through `ok`)
                 double xa = 0.0, xb = 0.0, xc = 0.0;  // the candidate's by-products (lane k)
                 double nvx = 0.0, nvy = 0.0, nvz = 0.0;
                 if (k == 2) {
-                    xa = __shfl_sync(kFull, ca, k);
+                    xa = __shfl_sync(kFull, ca, k, LPV);
                 } else if (r3 == 1 || r3 == 2) {
-                    xa = __shfl_sync(kFull, ca, k);
-                    xb = __shfl_sync(kFull, cb, k);
+                    xa = __shfl_sync(kFull, ca, k, LPV);
+                    xb = __shfl_sync(kFull, cb, k, LPV);
                     // the fibre's other angle, current value, from its owner lane
                     const int other = r3 == 1 ? k + 1 : k - 1;
-                    const double os = __shfl_sync(kFull, my_s, other);
-                    const double oc = __shfl_sync(kFull, my_c, other);
+                    const double os = __shfl_sync(kFull, my_s, other, LPV);
+                    const double oc = __shfl_sync(kFull, my_c, other, LPV);
                     if (r3 == 1) {  // theta' with the current phi
-                        xc = __shfl_sync(kFull, cc, k);
+                        xc = __shfl_sync(kFull, cc, k, LPV);
                         nvx = xa * oc;
                         nvy = xa * os;
                         nvz = xb;
@@ -329,55 +367,64 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
                     }
                 }
                 double nsse = 0.0, nlp;
-                double ne[MPL], nd[MPL], nA[MPL], nej[N][MPL];
+                double ne[MPL], nd[MPL], nej[N][MPL];
+                double eshell = 0.0;
+                if (k == 1 && nshell)  // same operations as the per-measurement e^{-b d'}
+                    eshell = exp(-((double)s_shell[gl < (uint32_t)nshell ? gl : 0u] * cand));
+                double ninv = inv2s2;
                 if (k == 2) {
-                    nlp = -np1 * xa - sse / (2.0 * cand * cand);
+                    ninv = 1.0 / (2.0 * cand * cand);
+                    nlp = -np1 * xa - sse * ninv;
 #pragma unroll
                     for (int j = 0; j < N; ++j) nlp = nlp + lsin[j];
                 } else {
 #pragma unroll
                     for (int m = 0; m < MPL; ++m) {
                         double mu;
-                        if (k == 0) {
-                            mu = cand * A[m];
+                        if (k == 0) {  // the mixture is recomputed (3 DP ops) instead of cached
+                            double accm = (1.0 - sumf) * e0[m];
+#pragma unroll
+                            for (int j = 0; j < N; ++j) accm = madd(fj[j], ej[j][m], accm);
+                            mu = cand * accm;
                         } else if (k == 1) {
-                            const double bd = (double)bf[m] * cand;
-                            ne[m] = exp(-bd);
+                            const double bd = (double)BF(m) * cand;
+                            if (nshell) {  // e^{-b d'} of this measurement's shell (lane u: shell u)
+                                ne[m] = __shfl_sync(kFull, eshell, s_sidx[gl + LPV * m], LPV);
+                            } else {
+                                ne[m] = exp(-bd);
+                            }
                             double accm = (1.0 - sumf) * ne[m];
 #pragma unroll
                             for (int j = 0; j < N; ++j) {
                                 nej[j][m] = exp(-(bd * (dj[j][m] * dj[j][m])));
                                 accm = madd(fj[j], nej[j][m], accm);
                             }
-                            nA[m] = accm;
                             mu = S0 * accm;
                         } else if (r3 == 0) {
                             double accm = (1.0 - nsumf) * e0[m];
 #pragma unroll
                             for (int j = 0; j < N; ++j) accm = madd(j == jf ? cand : fj[j], ej[j][m], accm);
-                            nA[m] = accm;
                             mu = S0 * accm;
                         } else {
-                            const double bd = (double)bf[m] * dd;
-                            nd[m] = madd((double)rz[m], nvz, madd((double)ry[m], nvy, (double)rx[m] * nvx));
+                            const double bd = (double)BF(m) * dd;
+                            nd[m] = madd((double)RZ(m), nvz, madd((double)RY(m), nvy, (double)RX(m) * nvx));
                             ne[m] = exp(-(bd * (nd[m] * nd[m])));
                             double accm = (1.0 - sumf) * e0[m];
 #pragma unroll
                             for (int j = 0; j < N; ++j) accm = madd(fj[j], j == jf ? ne[m] : ej[j][m], accm);
-                            nA[m] = accm;
                             mu = S0 * accm;
                         }
                         const double r = (double)yf[m] - mu;
                         nsse = valid[m] ? madd(r, r, nsse) : nsse;
                     }
-                    nsse = warp_sum(nsse);
-                    nlp = -np1 * lsig - nsse / (2.0 * sig * sig);
+                    nsse = group_sum<LPV>(nsse);
+                    nlp = -np1 * lsig - nsse * inv2s2;
 #pragma unroll
                     for (int j = 0; j < N; ++j) nlp = nlp + ((r3 == 1 && j == jf) ? xc : lsin[j]);
                 }
                 // accept with probability min(r, 1): ln u < lp' - lp
-                const bool accept = lu < nlp - lp;
-                if (lane == (uint32_t)k) {
+                const bool accept = ok && lu < nlp - lp;
+                if (gl == (uint32_t)k) {
                     my_acc += accept ? 1u : 0u;
                     my_tot += accept ? 1u : 0u;
                     my_rej += accept ? 0u : 1u;
@@ -400,11 +447,11 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
                             e0[m] = ne[m];
 #pragma unroll
                             for (int j = 0; j < N; ++j) ej[j][m] = nej[j][m];
-                            A[m] = nA[m];
                         }
                     } else if (k == 2) {
                         sig = cand;
                         lsig = xa;
+                        inv2s2 = ninv;
                     } else {
                         sse = nsse;
                         if (r3 == 0) {
@@ -415,7 +462,6 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
                         }
 #pragma unroll
                         for (int m = 0; m < MPL; ++m) {
-                            A[m] = nA[m];
                             if (r3 != 0) {
                                 dj[jf][m] = nd[m];
                                 ej[jf][m] = ne[m];
@@ -433,25 +479,30 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
             // samples after the burn-in, every L loops; lane k writes omega_k
             if (t >= a.burnin && (t - a.burnin + 1u) % a.interval == 0u) {
                 const uint32_t s = (t - a.burnin + 1u) / a.interval - 1u;
-                if (lane < (uint32_t)NP) a.samples[((uint64_t)lane * a.nsamples + s) * V + v] = my_w;
+                if (gact && gl < (uint32_t)NP) a.samples[((uint64_t)gl * a.nsamples + s) * V + v] = my_w;
             }
         }
-        if (a.accepted && lane < (uint32_t)NP) a.accepted[(uint64_t)lane * V + v] = my_tot;
-        if (lane < (uint32_t)NP) acc_tot += my_tot;
+        if (a.accepted && gact && gl < (uint32_t)NP) a.accepted[(uint64_t)gl * V + v] = my_tot;
+        if (gact && gl < (uint32_t)NP) acc_tot += my_tot;
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) acc_tot += __shfl_xor_sync(kFull, acc_tot, o);
     if (lane == 0 && acc_tot) atomicAdd(a.stats + kMcmcStatAccepted, acc_tot);
+#undef BF
+#undef RX
+#undef RY
+#undef RZ
 }
 
-template <int N, int MPL>
+template <int N, int MPL, int VPW>
 cudaError_t launch_m(const McmcArgs& a, int num_sms, cudaStream_t st) {
-    auto k = mcmc_kernel<N, MPL>;
+    auto k = mcmc_kernel<N, MPL, VPW>;
     int per_sm = 0;
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kMcmcThreads, 0);
     if (e != cudaSuccess) return e;
     if (per_sm < 1) return cudaErrorInvalidConfiguration;
-    const uint64_t need = ((uint64_t)a.nvox + kMcmcThreads / 32 - 1) / (kMcmcThreads / 32);
+    const uint64_t per_cta = (uint64_t)(kMcmcThreads / 32) * VPW;  // voxels in flight per CTA
+    const uint64_t need = ((uint64_t)a.nvox + per_cta - 1) / per_cta;
     const uint64_t full = (uint64_t)num_sms * (uint64_t)per_sm;
     const uint64_t grid = need < full ? need : full;
     if (grid == 0) return cudaSuccess;
@@ -461,11 +512,22 @@ cudaError_t launch_m(const McmcArgs& a, int num_sms, cudaStream_t st) {
 
 template <int N>
 cudaError_t launch_mn(const McmcArgs& a, int num_sms, cudaStream_t st) {
+    // up to 64 measurements: two voxels per warp (16 lanes each, <= 4 measurements per lane),
+    // which halves the per-voxel cost of the serial part of an MH step (reduction, decision)
+    if (PT_MCMC_VPW == 2 && a.nmeas <= 64) {
+        switch ((a.nmeas + 15) / 16) {
+            case 1: return launch_m<N, 1, 2>(a, num_sms, st);
+            case 2: return launch_m<N, 2, 2>(a, num_sms, st);
+            case 3: return launch_m<N, 3, 2>(a, num_sms, st);
+            case 4: return launch_m<N, 4, 2>(a, num_sms, st);
+            default: return cudaErrorInvalidValue;
+        }
+    }
     switch ((a.nmeas + 31) / 32) {
-        case 1: return launch_m<N, 1>(a, num_sms, st);
-        case 2: return launch_m<N, 2>(a, num_sms, st);
-        case 3: return launch_m<N, 3>(a, num_sms, st);
-        case 4: return launch_m<N, 4>(a, num_sms, st);
+        case 1: return launch_m<N, 1, 1>(a, num_sms, st);
+        case 2: return launch_m<N, 2, 1>(a, num_sms, st);
+        case 3: return launch_m<N, 3, 1>(a, num_sms, st);
+        case 4: return launch_m<N, 4, 1>(a, num_sms, st);
         default: return cudaErrorInvalidValue;
     }
 }

@@ -1,0 +1,4 @@
+set -x
+timeout 900 python -m pytest tests/test_gpu_mcmc.py -q -x > gpurun_out/pytest_gpu_mcmc6.log 2>&1; tail -3 gpurun_out/pytest_gpu_mcmc6.log
+for v in mb3 mb5; do PT_LIB=$PWD/scripts/libpt_mcmc_$v.so timeout 300 python scripts/mcmc_time.py m2 2>&1 | sed "s/^/$v /" | tail -1; done
+timeout 300 python scripts/mcmc_time.py m2 2>&1 | sed "s/^/mb4 /" | tail -1

@@ -57,6 +57,22 @@ def test_mcmc_parity_uniform(pt, tracker, N, ndirs, nb0):
     assert st["accepted"] == int(gacc.sum())
 
 
+@pytest.mark.parametrize("shells", [3, 40])
+def test_mcmc_parity_multishell(pt, tracker, shells):
+    """b-values on `shells` distinct shells: <= 8 shells take one e^{-b d'} per shell and
+    proposal, more fall back to one per measurement; both must match the oracle."""
+    rng = np.random.default_rng(shells)
+    d = phantom.dwi_uniform(nvox=64, gen_seed=17, burnin=50, nsamples=10, interval=2, adapt_every=10)
+    levels = np.round(rng.uniform(0.3, 3.0, shells), 3)
+    b = d.bvals.copy()
+    b[4:] = levels[np.arange(b.size - 4) % shells].astype(np.float32)
+    d = d.replace(bvals=b)
+    g, gacc, _ = _run(tracker, d)
+    r = oracle.mcmc(d, threads=_threads())
+    if _compare(g, r["samples"], 64) == 0:
+        assert np.array_equal(gacc, r["accepted"])
+
+
 def test_mcmc_parity_brain_small(pt, tracker):
     """Brain-shaped DWI (mask, mixed fibre configurations, automatic initial states)."""
     d = phantom.mcmc_config("m_small")

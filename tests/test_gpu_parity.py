@@ -175,6 +175,43 @@ def test_whole_brain_full_size_sampled(pt, tracker, cfg):
     assert r["nsteps"].mean() > 10
 
 
+def test_c5_hcp_scale_sampled(pt, tracker):
+    """configs[4] (HCP-scale 145x174x145, 50 samples x 3 fibres, fp16 records (32-B records,
+    one sector per step), 10^4 particles per seed): every 64th WM seed at full P, the global
+    invariants and 1500 sampled particles recomputed one by one by the oracle."""
+    import psutil
+    import torch
+    if psutil.virtual_memory().total < 40e9:
+        pytest.skip("c5 generation needs ~14 GB of host memory")
+    w = phantom.wm_seeds(phantom.config("c5"), every=64)
+    tracker.load_volume(w.volume)
+    m = tracker.track_workload(w, flags=REC_ALL)
+    torch.cuda.synchronize()
+    st = tracker.stats()
+    out = tracker.get_paths(on_device=True)
+    nst = out["nsteps"].to(torch.int64)
+    gm = m.cpu().numpy().view(np.uint32)
+    assert st["particles"] == w.nparticles
+    assert st["total_steps"] == int(nst.sum().item()) == int(gm.sum(dtype=np.uint64))
+    assert np.all(gm[w.volume.mask == 0] == 0)
+    pick = np.sort(np.random.default_rng(55).choice(w.nparticles, 1500, replace=False))
+    idx_t = torch.as_tensor(pick, device=out["nsteps"].device)
+    g = {"nsteps": out["nsteps"][idx_t].cpu().numpy().view(np.uint16),
+         "reason": out["reason"][idx_t].cpu().numpy(), "end": out["end"][idx_t].cpu().numpy()}
+    P = w.particles_per_seed
+    rn, rr, re_ = [], [], []
+    for li in pick:
+        si, j = divmod(int(li), P)
+        r = oracle.track(w.replace(seeds=w.seeds[si:si + 1], seed_ids=w.ids()[si:si + 1]), j, j + 1,
+                         want_map=False)
+        rn.append(r["nsteps"][0])
+        rr.append(r["reason"][0])
+        re_.append(r["end"][0])
+    assert np.array_equal(g["nsteps"].astype(np.int64), np.array(rn))
+    assert np.array_equal(g["reason"], np.array(rr))
+    assert np.array_equal(g["end"].view(np.uint32), np.array(re_).view(np.uint32))
+
+
 # ----------------------------------------------------------------------------- invariances
 
 def test_sharding_invariance(pt, tracker):
