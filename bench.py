@@ -51,9 +51,10 @@ MCMC_TEXT = {
 # Table III: valid voxels, CPU time, GPU time (HD 5870), context only
 PAPER_TABLE3 = {"m1": {"voxels": 205082, "cpu_s": 1383, "gpu_s": 41.3, "speedup": 33.6},
                 "m2": {"voxels": 402194, "cpu_s": 2724, "gpu_s": 80.1, "speedup": 34.0}}
-# executed fp64 lane-instructions per voxel-loop of the MCMC kernel (ncu SASS count,
-# profiles/r01f_mcmc_ncu.md); None until measured
-MCMC_FP64_OPS_PER_VOXEL_LOOP = None
+# executed FP64 lane-instructions (DFMA + DMUL + DADD) per voxel-loop of the MCMC kernel for
+# the Table III shape (n = 64, N = 2): ncu SASS count of the current kernel (v5),
+# profiles/r01f_v5_mcmc_ncu.md.  Per-unit figure of the MCMC roofline (bound "alu", FP64 pipe).
+MCMC_FP64_OPS_PER_VOXEL_LOOP = {"m1": 14322, "m2": 14322, "m2_prof": 14322}
 
 # Table II of the paper, for context beside the NEXT-1 paper-mode workloads:
 # (total fibre length = total steps, longest fibre) on the real CABI datasets, HD 5870.
@@ -326,12 +327,14 @@ def run_mcmc(args):
     kmean = sum(kms) / len(kms)
     roof = None
     peak = _fp64_peak()
-    if MCMC_FP64_OPS_PER_VOXEL_LOOP:
-        ach = st["voxels"] * d.loops * MCMC_FP64_OPS_PER_VOXEL_LOOP / (kmean * 1e-3)
-        roof = {"bound": "alu", "achieved": ach / 1e12, "peak": peak / 1e12, "unit": "T fp64 lane-ops/s",
-                "frac": ach / peak, "traffic": None, "kernel_ms": kmean,
-                "ops_per_voxel_loop": MCMC_FP64_OPS_PER_VOXEL_LOOP,
-                "peak_source": "derived: 148 SMs x 64 FP64 lanes x sm_max_mhz"}
+    ops = MCMC_FP64_OPS_PER_VOXEL_LOOP.get(args.config)
+    if ops:
+        ach = st["voxels"] * d.loops * ops / (kmean * 1e-3)
+        roof = {"bound": "alu", "achieved": ach / 1e12, "peak": peak / 1e12,
+                "unit": "T FP64 lane-instructions/s", "frac": ach / peak, "traffic": None,
+                "kernel_ms": kmean, "fp64_lane_instructions_per_voxel_loop": ops,
+                "per_unit_source": "ncu SASS count (DFMA + DMUL + DADD), profiles/r01f_v5_mcmc_ncu.md",
+                "peak_source": "derived: 148 SMs x 64 FP64 lanes per clock x sm_max_mhz (FMA = 1 instruction)"}
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         import oracle

@@ -25,6 +25,9 @@
 #include "pt_device.cuh"
 #include "pt_internal.h"
 
+#ifndef PT_RUNLEN
+#define PT_RUNLEN 1  // merge consecutive visits of a voxel before the RED (0: ablation iv, one RED per step)
+#endif
 #ifndef PT_SLOTS
 #define PT_SLOTS 1  // particles per lane in the persistent kernel (1 or 2; 2 measured no faster)
 #endif
@@ -153,10 +156,14 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
         x.qz = c ? nz_ : x.qz;
         x.n += c ? 1 : 0;
         if (has_map) {
+#if PT_RUNLEN
             const bool change = v != x.run_vox;
             red_add_if(c && change && x.run_cnt != 0u, map + x.run_vox, x.run_cnt);
             x.run_cnt = c ? (change ? 1u : x.run_cnt + 1u) : x.run_cnt;
             x.run_vox = c ? v : x.run_vox;
+#else
+            red_add_if(c, map + v, 1u);  // ablation (iv): one global RED per committed step
+#endif
         }
         if (OUT && a.conn && c) {  // NEXT-2: targets entered by committed steps (R21)
             const uint32_t lbl = __ldg(a.labels + v);

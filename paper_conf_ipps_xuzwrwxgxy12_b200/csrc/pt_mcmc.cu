@@ -63,7 +63,8 @@ __device__ __forceinline__ double group_sum(double v) {
 }
 
 // VPW voxels per warp, LPV = 32 / VPW lanes per voxel, MPL measurements per lane.
-template <int N, int MPL, int VPW>
+// FULL: n == LPV * MPL (every measurement slot holds a measurement; no masking).
+template <int N, int MPL, int VPW, bool FULL>
 __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(const __grid_constant__ McmcArgs a) {
     constexpr int NP = 3 + 3 * N;
     constexpr int LPV = 32 / VPW;
@@ -78,6 +79,10 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
     // reads entry gl + LPV m: distinct banks within a group, broadcast across groups);
     // entries >= n are zero.  Measurement i of the voxel: i = gl + LPV m.
     __shared__ float s_b[LPV * MPL], s_rx[LPV * MPL], s_ry[LPV * MPL], s_rz[LPV * MPL];
+    // the same in binary64 for the hot loops (no float->double conversion per use)
+    __shared__ double s_bd[LPV * MPL], s_rxd[LPV * MPL], s_ryd[LPV * MPL], s_rzd[LPV * MPL];
+    // each lane's measurements of its voxel in binary64 (lane-private slots)
+    __shared__ double s_y[kMcmcThreads / 32][MPL][32];
     // the distinct b-values ("shells", <= kMaxShells) and each measurement's shell: a d
     // proposal then needs one e^{-b d'} per shell instead of one per measurement
     __shared__ float s_shell[kMaxShells];
@@ -89,6 +94,10 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
         s_rx[i] = in ? a.bvecs[3 * i] : 0.f;
         s_ry[i] = in ? a.bvecs[3 * i + 1] : 0.f;
         s_rz[i] = in ? a.bvecs[3 * i + 2] : 0.f;
+        s_bd[i] = (double)s_b[i];
+        s_rxd[i] = (double)s_rx[i];
+        s_ryd[i] = (double)s_ry[i];
+        s_rzd[i] = (double)s_rz[i];
     }
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -113,10 +122,15 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
 #define RX(m) s_rx[gl + LPV * (m)]
 #define RY(m) s_ry[gl + LPV * (m)]
 #define RZ(m) s_rz[gl + LPV * (m)]
+#define BD(m) s_bd[gl + LPV * (m)]
+#define RXD(m) s_rxd[gl + LPV * (m)]
+#define RYD(m) s_ryd[gl + LPV * (m)]
+#define RZD(m) s_rzd[gl + LPV * (m)]
+#define YD(m) s_y[threadIdx.x >> 5][m][lane]
     bool valid[MPL];
     float yf[MPL];
 #pragma unroll
-    for (int m = 0; m < MPL; ++m) valid[m] = (int)gl + LPV * m < n;
+    for (int m = 0; m < MPL; ++m) valid[m] = FULL || (int)gl + LPV * m < n;
     unsigned long long acc_tot = 0ull;
 
     for (;;) {
@@ -129,7 +143,10 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
         const uint32_t v = a.vox[gact ? slot : base];
         const uint64_t V = a.V;
 #pragma unroll
-        for (int m = 0; m < MPL; ++m) yf[m] = valid[m] ? a.dwi[(uint64_t)(gl + LPV * m) * V + v] : 0.f;
+        for (int m = 0; m < MPL; ++m) {
+            yf[m] = valid[m] ? a.dwi[(uint64_t)(gl + LPV * m) * V + v] : 0.f;
+            YD(m) = (double)yf[m];
+        }
 
         double w[NP];
         double sth[N], cth[N], sph[N], cph[N], lsin[N];
@@ -242,18 +259,18 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
         double sse = 0.0;
 #pragma unroll
         for (int m = 0; m < MPL; ++m) {
-            const double b = (double)BF(m);
+            const double b = BD(m);
             const double bd = b * w[1];
             e0[m] = exp(-bd);
             double acc = (1.0 - sumf) * e0[m];
 #pragma unroll
             for (int j = 0; j < N; ++j) {
                 const double vx = sth[j] * cph[j], vy = sth[j] * sph[j], vz = cth[j];
-                dj[j][m] = madd((double)RZ(m), vz, madd((double)RY(m), vy, (double)RX(m) * vx));
+                dj[j][m] = madd(RZD(m), vz, madd(RYD(m), vy, RXD(m) * vx));
                 ej[j][m] = exp(-(bd * (dj[j][m] * dj[j][m])));
                 acc = madd(fj[j], ej[j][m], acc);
             }
-            const double r = (double)yf[m] - w[0] * acc;
+            const double r = YD(m) - w[0] * acc;
             sse = valid[m] ? madd(r, r, sse) : sse;
         }
         sse = group_sum<LPV>(sse);
@@ -387,7 +404,7 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
                             for (int j = 0; j < N; ++j) accm = madd(fj[j], ej[j][m], accm);
                             mu = cand * accm;
                         } else if (k == 1) {
-                            const double bd = (double)BF(m) * cand;
+                            const double bd = BD(m) * cand;
                             if (nshell) {  // e^{-b d'} of this measurement's shell (lane u: shell u)
                                 ne[m] = __shfl_sync(kFull, eshell, s_sidx[gl + LPV * m], LPV);
                             } else {
@@ -406,15 +423,15 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
                             for (int j = 0; j < N; ++j) accm = madd(j == jf ? cand : fj[j], ej[j][m], accm);
                             mu = S0 * accm;
                         } else {
-                            const double bd = (double)BF(m) * dd;
-                            nd[m] = madd((double)RZ(m), nvz, madd((double)RY(m), nvy, (double)RX(m) * nvx));
+                            const double bd = BD(m) * dd;
+                            nd[m] = madd(RZD(m), nvz, madd(RYD(m), nvy, RXD(m) * nvx));
                             ne[m] = exp(-(bd * (nd[m] * nd[m])));
                             double accm = (1.0 - sumf) * e0[m];
 #pragma unroll
                             for (int j = 0; j < N; ++j) accm = madd(fj[j], j == jf ? ne[m] : ej[j][m], accm);
                             mu = S0 * accm;
                         }
-                        const double r = (double)yf[m] - mu;
+                        const double r = YD(m) - mu;
                         nsse = valid[m] ? madd(r, r, nsse) : nsse;
                     }
                     nsse = group_sum<LPV>(nsse);
@@ -492,11 +509,17 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
 #undef RX
 #undef RY
 #undef RZ
+#undef BD
+#undef RXD
+#undef RYD
+#undef RZD
+#undef YD
 }
 
 template <int N, int MPL, int VPW>
 cudaError_t launch_m(const McmcArgs& a, int num_sms, cudaStream_t st) {
-    auto k = mcmc_kernel<N, MPL, VPW>;
+    constexpr int LPV = 32 / VPW;
+    auto k = a.nmeas == LPV * MPL ? mcmc_kernel<N, MPL, VPW, true> : mcmc_kernel<N, MPL, VPW, false>;
     int per_sm = 0;
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, kMcmcThreads, 0);
     if (e != cudaSuccess) return e;
