@@ -34,6 +34,8 @@ CONFIG_TEXT = {
     "c2": "configs[1]: 64x64x32 two-bundle 90deg crossing, 50 samples x 2 fibres, 1k seeds x 5000",
     "c2_dispersed": "configs[1] shape, dispersed (sigma 0.15, f jitter 0.03)",
     "c1": "configs[0]: 32x32x16 straight tube, 64 seeds x 1000",
+    "c5": "configs[4]: HCP-scale 145x174x145, 50 samples x 3 fibres, fp16 records, all WM seeds x 10^4 "
+          "particles (BASELINE quotes it on 8 B200; here per GPU)",
     "d1": "NEXT-1 paper mode: dataset-1-shaped 96x96x48, every brain voxel x 50 (one streamline per "
           "sample volume), step 0.1, dot threshold 0.9, MaxStep 1888 (Table II row 1 parameters)",
     "d2": "NEXT-1 paper mode: dataset-2-shaped 102x102x60, every brain voxel x 50, step 0.1, "
