@@ -1,21 +1,23 @@
 // pt_mcmc.cu -- NEXT-4: Metropolis-Hastings sampling of the multiple partial volume model
 // (Eq. 1; Sec. IV-A and Fig. 2) on sm_100a, binary64 (reading M4).
 //
-// The paper runs one thread per voxel.  Here one WARP owns a voxel and its lanes
-// own the voxel's measurements (lane l holds i = l, l+32, ...): the per-measurement terms
-// of Eq. 1 stay in registers for the whole chain (e^{-b d}, e^{-b d (r.v_j)^2}, r.v_j,
-// the mixture A_i), so a proposal of S0, sigma or f_j costs no exponential at all, a
-// proposal of an angle costs one per measurement and a proposal of d costs N+1; the sum of
-// squared residuals is a warp reduction.  The NP draws of a loop do not depend on the state
-// (counter-based Philox, M6), and omega'_k only depends on omega_k, which no other MH step
-// of the loop changes: lane k computes draw k, the candidate and its transcendental
-// by-products (ln sigma', sincos, ln|sin theta'|) for all NP steps of the loop in parallel
-// at the loop's start; step k then only broadcasts them from lane k.
+// The paper runs one thread per voxel.  Here a group of LPV lanes owns a voxel (two
+// voxels per warp, 16 lanes each, for n <= 64; one voxel per warp above) and lane l of a
+// group holds measurements l, l + LPV, ...: the per-measurement terms of Eq. 1 stay in
+// registers for the whole chain (e^{-b d}, e^{-b d (r.v_j)^2}, r.v_j), so a proposal of S0,
+// sigma or f_j costs no exponential, an angle proposal one per measurement and a d proposal
+// N per measurement plus one per b-shell; the sum of squared residuals is a group
+// reduction.  Lane k of a group owns parameter k (value, proposal width, counters, sin/cos).
+// The draws are counter-based (M6) and omega'_k only depends on omega_k, which no other MH
+// step of the loop changes: the lanes compute the Box-Muller draws of several loops at
+// once, lane k forms candidate k and its transcendental by-products (ln sigma', sincos,
+// ln|sin theta'|) at the loop's start, and step k only broadcasts them from lane k.
 //
 // Results follow contract C-MCMC of DESIGN.md §12 in the oracle's operation order; the
-// oracle uses glibc's exp/log/sin/cos, this file CUDA's (both within an ulp or two), and
-// the residual sum is a warp tree instead of a sequential loop, so samples agree to
-// ~1e-13 relative rather than bit for bit (the parity bar of DESIGN.md §12).
+// oracle uses glibc's exp/log/sin/cos, this file CUDA's (both within an ulp or two), the
+// residual sum is a lane tree instead of a sequential loop and a*b+c is fused into a DFMA,
+// so samples agree to ~1e-13 relative rather than bit for bit (the parity bar of DESIGN.md
+// §12).
 #include <cuda_runtime.h>
 #include <cub/device/device_select.cuh>
 #include <thrust/iterator/counting_iterator.h>
