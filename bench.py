@@ -659,6 +659,8 @@ def run_ours(args):
                        "steps_per_pass": int(total_steps),
                        "mean_steps_per_streamline": total_steps / (total_seeds * w.particles_per_seed),
                        "record_bytes": rb, "records": "fp16" if w.volume.is_half else "fp32",
+                       "record_layout": "bricks of %d^3 voxels" % (1 << int(os.environ.get("PT_BRICK", "4")))
+                                        if int(os.environ.get("PT_BRICK", "4")) else "raster",
                        "parallelism": f"seed-sharded x{world}" + (" + NCCL reduce" if world > 1 else ""),
                        "l2": "inputs > L2 (record volume %.2f GB) and a 256 MiB L2 flush between steps"
                              % (V * w.volume.nsamples * rb / 1e9)},

@@ -108,6 +108,12 @@ typedef struct {
 /* Load the per-voxel orientation samples (the six sample volumes f1,f2,theta1,theta2,
  * phi1,phi2 of P:L125, with (theta, phi) given as Cartesian unit vectors, R20) and the
  * tracking mask, and repack them on the device into one record per (voxel, sample).
+ * The device records are voxel-major and BRICKED: the volume is cut into bricks of
+ * 2^b x 2^b x 2^b voxels (b from the environment variable PT_BRICK: 4, the default, or 0 = plain
+ * raster order; any other value is PT_ERR_ARG), so the records of a 3-D neighbourhood
+ * are contiguous.
+ * The layout is internal: it changes no result, only the padded device footprint
+ * (ceil(n/2^b)*2^b per axis x S x record bytes).
  *   dyads: [F][S][nz][ny][nx][3] (x fastest, xyz innermost), float32 or binary16 bits
  *   f    : [F][S][nz][ny][nx], same dtype
  *   mask : [nz][ny][nx] uint8, != 0 inside

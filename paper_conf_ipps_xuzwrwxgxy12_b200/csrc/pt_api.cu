@@ -10,6 +10,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -24,6 +25,9 @@
 // c3 74.6/75.3/76.0/76.4/77.0/77.2/76.9 G steps/s; 32 is the default).
 #define PT_SEEDS_PER_CLAIM 32
 #endif
+#ifndef PT_BRICK_DEFAULT
+#define PT_BRICK_DEFAULT 4  // record layout brick log2 edge (0 = raster, 4 = 16^3 bricks, measured best)
+#endif
 
 struct pt_ctx {
     int device = 0;
@@ -34,6 +38,7 @@ struct pt_ctx {
     bool loaded = false;
     pt_volume vol{};
     int rec_bytes = 0;
+    pt::RecLayout layout{};       // record voxel order (bricked, rec_vox)
     uint8_t* d_rec = nullptr;
     size_t rec_size = 0;
     uint8_t* d_mask = nullptr;    // tracking mask copy (the variant kernel's interpolation)
@@ -268,7 +273,15 @@ pt_status pt_load_samples(pt_ctx* c, const pt_volume* v, const void* dyads, cons
     const uint64_t S = (uint64_t)v->nsamples, F = (uint64_t)v->nfibres;
     const size_t esz = v->dtype == PT_F16 ? 2 : 4;
     const size_t dy_bytes = F * S * V * 3 * esz, f_bytes = F * S * V * esz, m_bytes = V;
-    const size_t rec_size = V * S * (size_t)rb;
+    // record layout: bricks of 2^b voxels per axis (PT_BRICK env var = b, 0 = raster)
+    uint32_t blog = PT_BRICK_DEFAULT;
+    if (const char* e = getenv("PT_BRICK")) blog = (uint32_t)atoi(e);
+    if (blog != 0u && blog != pt::kBrickLog)
+        return fail(c, PT_ERR_ARG, "pt_load_samples: PT_BRICK must be 0 (raster) or %u (16^3 bricks), got %u",
+                    pt::kBrickLog, blog);
+    const pt::RecLayout L = pt::rec_layout(v->nx, v->ny, v->nz, blog);
+    if (L.nvox() > 0xFFFFFFFFull) return fail(c, PT_ERR_ARG, "pt_load_samples: padded volume exceeds 2^32-1 voxels");
+    const size_t rec_size = L.nvox() * S * (size_t)rb;
 
     // stage host inputs on the device (device inputs are read in place)
     const void* d_dy = dyads;
@@ -317,7 +330,7 @@ pt_status pt_load_samples(pt_ctx* c, const pt_volume* v, const void* dyads, cons
     if (e == cudaSuccess) e = cudaMemcpyAsync(c->d_mask, d_m, (size_t)V, cudaMemcpyDeviceToDevice, c->stream);
     if (e == cudaSuccess) e = cudaMemsetAsync(c->d_stats + pt::kStatBadInput, 0, sizeof(unsigned long long), c->stream);
     if (e == cudaSuccess)
-        e = pt::launch_repack(d_dy, d_f, d_m, c->d_rec, (int64_t)V, v->nsamples, v->nfibres,
+        e = pt::launch_repack(d_dy, d_f, d_m, c->d_rec, v->nx, v->ny, v->nz, L, v->nsamples, v->nfibres,
                               v->dtype == PT_F16, rb, c->d_stats + pt::kStatBadInput, c->stream);
     unsigned long long bad = 0;
     if (e == cudaSuccess)
@@ -328,6 +341,7 @@ pt_status pt_load_samples(pt_ctx* c, const pt_volume* v, const void* dyads, cons
     if (bad) return fail(c, PT_ERR_ARG, "pt_load_samples: %llu records inside the mask hold non-finite values", bad);
     c->vol = *v;
     c->rec_bytes = rb;
+    c->layout = L;
     c->loaded = true;
     c->tracked = false;
     c->ntargets = 0;  // targets belong to a volume shape
@@ -447,6 +461,9 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
 
     pt::TrackArgs a{};
     a.rec = c->d_rec;
+    a.rb_log = c->layout.b;
+    a.rb_nbx = c->layout.nbx;
+    a.rb_nby = c->layout.nby;
     a.nx = nxv;
     a.ny = nyv;
     a.nz = nzv;

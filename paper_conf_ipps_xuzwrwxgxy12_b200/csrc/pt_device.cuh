@@ -153,4 +153,26 @@ __device__ __forceinline__ int axis_index(float q, int c) {
     return c + __float2int_rz(q) - (int)(__float_as_uint(q) >> 31);
 }
 
+// ---------------------------------------------------------------------------- record layout
+// Position of voxel (ix, iy, iz) in the record volume.  Bricked layout: the volume is cut
+// into bricks of 2^b x 2^b x 2^b voxels (bricks raster-ordered, nbx x nby per z-slab of
+// bricks; voxels raster-ordered inside a brick), so the records of a 3-D neighbourhood --
+// everything a tract touches over a few steps -- sit in a few contiguous MB instead of
+// being strided by whole planes (fewer DRAM pages and TLB entries per neighbourhood).
+// b = 0 is the plain raster layout (nbx = nx, nby = ny).  Layout only: which record a
+// step reads is unchanged, so results are unaffected.
+__device__ __forceinline__ uint32_t rec_vox(int ix, int iy, int iz, uint32_t b, uint32_t nbx, uint32_t nby) {
+    const uint32_t m = (1u << b) - 1u;
+    const uint32_t x = (uint32_t)ix, y = (uint32_t)iy, z = (uint32_t)iz;
+    const uint32_t br = ((z >> b) * nby + (y >> b)) * nbx + (x >> b);
+    return (br << (3u * b)) | ((z & m) << (2u * b)) | ((y & m) << b) | (x & m);
+}
+// the same from a raster voxel index (variant / ablation kernels, repack)
+__device__ __forceinline__ uint32_t rec_vox_raster(uint32_t v, uint32_t nx, uint32_t ny, uint32_t b, uint32_t nbx,
+                                                   uint32_t nby) {
+    if (b == 0u) return v;
+    const uint32_t z = v / (nx * ny), r = v - z * (nx * ny), y = r / nx, x = r - y * nx;
+    return rec_vox((int)x, (int)y, (int)z, b, nbx, nby);
+}
+
 }  // namespace pt

@@ -41,7 +41,8 @@ enum StatIdx {
 };
 
 struct TrackArgs {
-    const uint8_t* rec;          // [V][S] records of rec_bytes
+    const uint8_t* rec;          // [V'][S] records of rec_bytes, voxel order rec_vox() (bricked)
+    uint32_t rb_log, rb_nbx, rb_nby;  // record layout: brick edge 2^rb_log (0 or kBrickLog), bricks per row / column
     int nx, ny, nz;
     int cx, cy, cz;              // floor(N/2) per axis
     float fcx, fcy, fcz;         // the same as floats
@@ -128,8 +129,16 @@ cudaError_t launch_track(const TrackArgs& a, int nfibres, bool half, bool simple
 // NEXT-3 variant kernel (bidirectional / interpolation / first-fibre modes; also runs the
 // default semantics when forced with PT_KERNEL_VARIANT).
 cudaError_t launch_track_var(const TrackArgs& a, int nfibres, bool half, int num_sms, cudaStream_t st);
+// Record layout (see rec_vox in pt_device.cuh): b = brick log2 edge, 0 (raster) or
+// kBrickLog (the default; the main tracking kernel is compiled for these two).
+constexpr uint32_t kBrickLog = 4;
+struct RecLayout {
+    uint32_t b, nbx, nby, nbz;
+    uint64_t nvox() const { return (uint64_t)nbx * nby * nbz << (3u * b); }  // allocated voxels (padded)
+};
+RecLayout rec_layout(int nx, int ny, int nz, uint32_t b);
 cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask, uint8_t* rec,
-                          int64_t V, int S, int F, bool half, int rec_bytes,
+                          int nx, int ny, int nz, const RecLayout& L, int S, int F, bool half, int rec_bytes,
                           unsigned long long* bad, cudaStream_t st);
 // Z-order processing permutation of the seeds: perm[k] = index of the k-th seed in Morton
 // order of its voxel (ties by input index; stable radix sort).  keys, keys_out, idx, perm:

@@ -28,6 +28,9 @@
 #ifndef PT_RUNLEN
 #define PT_RUNLEN 1  // merge consecutive visits of a voxel before the RED (0: ablation iv, one RED per step)
 #endif
+#ifndef PT_REFILL_MIN
+#define PT_REFILL_MIN 2  // free lanes a warp waits for before refilling (amortises the refill block)
+#endif
 #ifndef PT_SLOTS
 #define PT_SLOTS 1  // particles per lane in the persistent kernel (1 or 2; 2 measured no faster)
 #endif
@@ -44,6 +47,7 @@ struct Slot {
     float qx, qy, qz;  // committed position, centred coordinates (R10)
     float px, py, pz;  // direction of the last (candidate) step
     uint32_t gvox;     // voxel read by the round-start gather (seed or pending candidate)
+    uint32_t grv;      // its position in the record volume (rec_vox)
     int n;             // committed steps
     uint64_t pid;      // global particle id = seed_id * P + j (RNG key, R16)
     uint32_t run_vox, run_cnt;  // run-length merge of consecutive visits
@@ -65,7 +69,9 @@ struct Cta {
 // the no-refill ablation).  SLOTS: particles per lane; with 2, a lane interleaves the steps
 // of two independent particles so that one particle's gather is in flight while the other
 // computes (more gathers in flight per SM without more threads, all from the same claim).
-template <int F, bool HALF, bool REFILL, bool OUT, int SLOTS>
+// BL: record layout, log2 brick edge (0 = raster), a compile-time constant so
+// the record position costs a few shift/mask instructions with immediates.
+template <int F, bool HALF, bool REFILL, bool OUT, int SLOTS, int BL>
 __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(const __grid_constant__ TrackArgs a) {
     using R = Rec<F, HALF>;
     constexpr int RB = R::kBytes;
@@ -96,6 +102,7 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
         P[sl].qx = P[sl].qy = P[sl].qz = 0.f;
         P[sl].px = P[sl].py = P[sl].pz = 0.f;
         P[sl].gvox = 0u;
+        P[sl].grv = 0u;
         P[sl].n = 0;
         P[sl].pid = 0ull;
         P[sl].run_vox = 0u;
@@ -112,6 +119,14 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
     uint32_t my_steps = 0, my_particles = 0, my_active = 0, rounds = 0;
     bool exhausted = false;  // warp-uniform
 
+    // position of voxel (ix, iy, iz) = raster index v in the record volume (rec_vox)
+    auto recv = [&](int ix, int iy, int iz, uint32_t v) -> uint32_t {
+        if (BL == 0) return v;
+        constexpr uint32_t m = (1u << BL) - 1u;
+        const uint32_t x = (uint32_t)ix, y = (uint32_t)iy, z = (uint32_t)iz;
+        const uint32_t br = ((z >> BL) * a.rb_nby + (y >> BL)) * a.rb_nbx + (x >> BL);
+        return (br << (3 * BL)) | ((z & m) << (2 * BL)) | ((y & m) << BL) | (x & m);
+    };
     // a termination only records the reason; outputs and the count flush are written once
     // per round for all ended particles at the top of the loop
     auto end = [&](Slot<F, HALF>& x, int w) {
@@ -182,7 +197,7 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
         if (OUT) s_li[sl * TPB + threadIdx.x] = li;
         const uint64_t sid = a.seed_ids ? a.seed_ids[si] : si;
         x.pid = sid * a.P + j;
-        x.sfix = (uint32_t)(j % a.S);
+        x.sfix = a.sample_mode ? (uint32_t)(j % a.S) : 0u;
         x.tmask = 0ull;
         x.sidx = (uint32_t)si;
         x.qx = __fsub_rn(a.seeds[3 * si + 0], a.fcx);
@@ -201,6 +216,7 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
         const int ix = axis_index(x.qx, a.cx), iy = axis_index(x.qy, a.cy), iz = axis_index(x.qz, a.cz);
         if ((unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny && (unsigned)iz < (unsigned)a.nz) {
             x.gvox = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
+            x.grv = recv(ix, iy, iz, x.gvox);
         } else {
             end(x, kEndMask);  // seed outside the volume (R12): finished right away, so the
             finish(x, sl);     // refill loop may hand this lane another particle
@@ -252,7 +268,8 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
         if (k < 2) {
             const uint32_t w = (k == 0) ? x.W.y : x.W.z;
             const uint32_t sk = a.sample_mode ? x.sfix : sample_of(w, a.S);
-            ldg_record_if<RB>(go, a.rec + ((uint64_t)v * a.S + sk) * RB, x.rv.w);
+            const uint32_t rvx = recv(ix, iy, iz, v);
+            ldg_record_if<RB>(go, a.rec + ((uint64_t)rvx * a.S + sk) * RB, x.rv.w);
             const bool outside = go && x.rv.outside();  // candidate outside the mask (R11)
             x.why = outside ? kEndMask : x.why;
             x.alive = go && !outside;
@@ -260,6 +277,7 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
         } else {
             x.pend = go;  // next round's start gathers and tests it
             x.gvox = go ? v : x.gvox;
+            if (BL != 0) x.grv = go ? recv(ix, iy, iz, v) : x.grv;
         }
     };
 
@@ -279,10 +297,11 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
         // ------------------------------------------------ lane refill (replaces the
         // paper's CPU Reduction()/segment relaunch)
         if (REFILL) {
-            bool any_need = false;
+            // refill once at least PT_REFILL_MIN slots of the warp are free (or none is live)
+            uint32_t nfree = 0;
 #pragma unroll
-            for (int sl = 0; sl < SLOTS; ++sl) any_need |= !P[sl].alive;
-            if (__any_sync(kFull, any_need) && !exhausted) {
+            for (int sl = 0; sl < SLOTS; ++sl) nfree += (uint32_t)__popc(__ballot_sync(kFull, !P[sl].alive));
+            if (!exhausted && nfree != 0u && (nfree >= (uint32_t)PT_REFILL_MIN || nfree == 32u * SLOTS)) {
                 uint32_t cseed = s_q[wib][0], cnext = s_q[wib][1], cend = s_q[wib][2];
 #pragma unroll
                 for (int sl = 0; sl < SLOTS; ++sl) {
@@ -333,7 +352,7 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
             const uint32_t t0 = (uint32_t)x.n + (x.pend ? 1u : 0u);  // a multiple of 3
             x.W = philox4x32_10(make_uint4(t0 / 3u, (uint32_t)x.pid, (uint32_t)(x.pid >> 32), 0u), a.key0, a.key1);
             const uint32_t s0 = a.sample_mode ? x.sfix : sample_of(x.W.x, a.S);
-            ldg_record_if<RB>(x.alive, a.rec + ((uint64_t)x.gvox * a.S + s0) * RB, x.rv.w);
+            ldg_record_if<RB>(x.alive, a.rec + ((uint64_t)(BL == 0 ? x.gvox : x.grv) * a.S + s0) * RB, x.rv.w);
         }
 #pragma unroll
         for (int sl = 0; sl < SLOTS; ++sl) {
@@ -378,7 +397,8 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(cons
 template <bool HALF>
 __global__ void repack_kernel(const void* __restrict__ dyads, const void* __restrict__ fr,
                               const uint8_t* __restrict__ mask, uint8_t* __restrict__ rec,
-                              int64_t V, int S, int F, int RB, unsigned long long* bad) {
+                              int nx, int ny, int64_t V, RecLayout L, int S, int F, int RB,
+                              unsigned long long* bad) {
     const int64_t total = V * (int64_t)S;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
          i += (int64_t)gridDim.x * blockDim.x) {
@@ -416,7 +436,8 @@ __global__ void repack_kernel(const void* __restrict__ dyads, const void* __rest
         } else if (!ok) {
             atomicAdd(bad, 1ull);
         }
-        uint8_t* out = rec + i * RB;
+        const uint64_t rv = rec_vox_raster((uint32_t)vox, (uint32_t)nx, (uint32_t)ny, L.b, L.nbx, L.nby);
+        uint8_t* out = rec + (rv * (uint64_t)S + (uint64_t)s) * RB;
         if (RB == 8) {
             *reinterpret_cast<uint2*>(out) = make_uint2(w[0], w[1]);
         } else {
@@ -524,10 +545,10 @@ __global__ void __launch_bounds__(256) gather_bench_kernel(const uint8_t* __rest
 }
 
 // ------------------------------------------------------------------------- launchers
-template <int F, bool HALF, bool REFILL, bool OUT>
-static cudaError_t launch_t(const TrackArgs& a, int num_sms, cudaStream_t st) {
+template <int F, bool HALF, bool REFILL, bool OUT, int BL>
+static cudaError_t launch_tb(const TrackArgs& a, int num_sms, cudaStream_t st) {
     constexpr int SL = REFILL ? PT_SLOTS : 1;
-    auto k = track_kernel<F, HALF, REFILL, OUT, SL>;
+    auto k = track_kernel<F, HALF, REFILL, OUT, SL, BL>;
     constexpr int TPB = Cta<REFILL, SL>::kTPB;
     if (a.nparticles == 0) return cudaSuccess;
     unsigned grid;
@@ -544,6 +565,14 @@ static cudaError_t launch_t(const TrackArgs& a, int num_sms, cudaStream_t st) {
     }
     k<<<grid, TPB, 0, st>>>(a);
     return cudaGetLastError();
+}
+
+// record layouts compiled into the tracking kernel: raster and 16^3 bricks
+template <int F, bool HALF, bool REFILL, bool OUT>
+static cudaError_t launch_t(const TrackArgs& a, int num_sms, cudaStream_t st) {
+    if (a.rb_log == 0) return launch_tb<F, HALF, REFILL, OUT, 0>(a, num_sms, st);
+    if (a.rb_log == kBrickLog) return launch_tb<F, HALF, REFILL, OUT, kBrickLog>(a, num_sms, st);
+    return cudaErrorInvalidValue;
 }
 
 template <int F, bool HALF>
@@ -566,17 +595,28 @@ cudaError_t launch_track(const TrackArgs& a, int nfibres, bool half, bool simple
     }
 }
 
+RecLayout rec_layout(int nx, int ny, int nz, uint32_t b) {
+    RecLayout L;
+    const uint32_t e = 1u << b;
+    L.b = b;
+    L.nbx = ((uint32_t)nx + e - 1u) >> b;
+    L.nby = ((uint32_t)ny + e - 1u) >> b;
+    L.nbz = ((uint32_t)nz + e - 1u) >> b;
+    return L;
+}
+
 cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask, uint8_t* rec,
-                          int64_t V, int S, int F, bool half, int rec_bytes,
+                          int nx, int ny, int nz, const RecLayout& L, int S, int F, bool half, int rec_bytes,
                           unsigned long long* bad, cudaStream_t st) {
+    const int64_t V = (int64_t)nx * ny * nz;
     const int64_t total = V * (int64_t)S;
     int64_t blocks = (total + 255) / 256;
     if (blocks > 148 * 64) blocks = 148 * 64;
     if (blocks < 1) blocks = 1;
     if (half)
-        repack_kernel<true><<<(unsigned)blocks, 256, 0, st>>>(dyads, f, mask, rec, V, S, F, rec_bytes, bad);
+        repack_kernel<true><<<(unsigned)blocks, 256, 0, st>>>(dyads, f, mask, rec, nx, ny, V, L, S, F, rec_bytes, bad);
     else
-        repack_kernel<false><<<(unsigned)blocks, 256, 0, st>>>(dyads, f, mask, rec, V, S, F, rec_bytes, bad);
+        repack_kernel<false><<<(unsigned)blocks, 256, 0, st>>>(dyads, f, mask, rec, nx, ny, V, L, S, F, rec_bytes, bad);
     return cudaGetLastError();
 }
 

@@ -128,7 +128,8 @@ __global__ void __launch_bounds__(kVarThreads, 1) track_var_kernel(const __grid_
                     u = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
             }
         }
-        ldg_record<RB>(a.rec + ((uint64_t)u * a.S + x.s) * RB, x.rv.w);
+        const uint32_t ur = rec_vox_raster(u, (uint32_t)a.nx, (uint32_t)a.ny, a.rb_log, a.rb_nbx, a.rb_nby);
+        ldg_record<RB>(a.rec + ((uint64_t)ur * a.S + x.s) * RB, x.rv.w);
         if (a.interp) x.mb = __ldg(a.mask + nv);
     };
     // GetStartPoint() of the current half: centred seed position, RNG stream,
@@ -310,7 +311,7 @@ __global__ void __launch_bounds__(kVarThreads, 1) track_var_kernel(const __grid_
         }
 
         // ---- B: the interpolated voxel was outside the mask => nearest voxel (R23)
-        if (a.interp && x.rv.outside()) ldg_record<RB>(a.rec + ((uint64_t)x.vox * a.S + x.s) * RB, x.rv.w);
+        if (a.interp && x.rv.outside()) ldg_record<RB>(a.rec + ((uint64_t)rec_vox_raster(x.vox, (uint32_t)a.nx, (uint32_t)a.ny, a.rb_log, a.rb_nbx, a.rb_nby) * a.S + x.s) * RB, x.rv.w);
 
         // ---- C: fibre choice, curvature, step
         const bool first = x.n == 0 && x.half == 0u;

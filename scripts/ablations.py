@@ -6,6 +6,7 @@
         schedules A_1, A_10, A_50, strategy B and C (Table IV)
   (iii) fp32 vs fp16 records (c3 vs c4)
   (v)   raster vs Morton seed order (PT_SEED_ORDER_INPUT)
+  (vi)  raster vs bricked record layout (PT_BRICK=0 vs the default 16^3 bricks)
   plus the NEXT-3 variant kernel on the default semantics (PT_KERNEL_VARIANT).
 
 Every run's total steps must equal the main kernel's (same parity contract: the results
@@ -59,19 +60,23 @@ def main():
         ("(ii) segmented strategy C", pt.PT_KERNEL_SEGMENTED, pt.SEGMENTS_C, w),
         ("(ii) segmented A_2000 (one segment)", pt.PT_KERNEL_SEGMENTED, (2000,), w),
     ]
+    variants = [v + ("4",) for v in variants]
+    variants.insert(1, ("(vi) raster record layout (PT_BRICK=0)", 0, None, w, "0"))
+    variants.append(("(vi) raster record layout, no refill (PT_BRICK=0)", pt.PT_KERNEL_SIMPLE, None, w, "0"))
     if args.config == "c3" and not args.only:
-        variants.append(("(iii) fp16 records (c4)", 0, None, None))
+        variants.append(("(iii) fp16 records (c4)", 0, None, None, "4"))
     rows = []
     ref_steps = None
     loaded = None
-    for name, flags, sched, wv in variants:
+    for name, flags, sched, wv, brick in variants:
         if args.only and args.only not in name:
             continue
         if wv is None:
             wv = phantom.to_half(w)
-        if loaded is not wv:
+        if loaded != (id(wv), brick):
+            os.environ["PT_BRICK"] = brick  # read by pt_load_samples
             tr.load_volume(wv.volume)
-            loaded = wv
+            loaded = (id(wv), brick)
         if sched:
             tr.set_segments(sched)
         best = None

@@ -132,6 +132,45 @@ def test_crossing_dispersed_paths(pt, tracker, simple):
     assert paths_equal(g["paths"], r["paths"])
 
 
+# ----------------------------------------------------------------------------- record layout
+
+@pytest.mark.parametrize("brick", [0, 4])
+def test_record_layout_bricks(pt, tracker, brick, monkeypatch):
+    """The bricked record layout (PT_BRICK = log2 brick edge) changes where a
+    record lives, never which record a step reads: on a volume whose dims are multiples of
+    no brick edge (41 x 37 x 23, so every brick row / column / slab is ragged) the main
+    kernel, the no-refill kernel and the variant kernel stay bit-exact with the oracle."""
+    import torch
+    monkeypatch.setenv("PT_BRICK", str(brick))
+    w = phantom.whole_brain(nx=41, ny=37, nz=23, semi=(18.0, 16.0, 10.0), nsamples=12, nfibres=2,
+                            particles_per_seed=33)
+    w = phantom.wm_seeds(w, every=max(1, w.nseeds // 120))
+    r = oracle.track(w, threads=_threads())
+    for extra in (0, pt.PT_KERNEL_SIMPLE, pt.PT_KERNEL_VARIANT):
+        g = gpu_run(tracker, w, REC_ALL | extra)
+        assert_parity(g, r)
+    # a variant that reads other voxels than the nearest one (probabilistic interpolation)
+    wb = phantom.whole_brain(nx=41, ny=37, nz=23, semi=(18.0, 16.0, 10.0), nsamples=12, nfibres=2,
+                             particles_per_seed=9)
+    wb = phantom.wm_seeds(wb, every=max(1, wb.nseeds // 60)).replace(bidir=1, interp=1)
+    gi = gpu_run(tracker, wb)
+    ri = oracle.track(wb, threads=_threads())
+    assert_parity(gi, ri)
+    torch.cuda.synchronize()
+
+
+def test_record_layout_rejects_other_bricks(pt, monkeypatch):
+    """Only the two compiled layouts are accepted (PT_ERR_ARG otherwise, nothing loaded)."""
+    monkeypatch.setenv("PT_BRICK", "3")
+    w = phantom.tube()
+    t = pt.Tracker(0)
+    try:
+        with pytest.raises(pt.PtError, match="PT_BRICK"):
+            t.load_volume(w.volume)
+    finally:
+        t.close()
+
+
 # ----------------------------------------------------------------------------- full size, sampled
 
 @pytest.mark.parametrize("cfg", ["c3", "c4"])
