@@ -171,7 +171,9 @@ def _workload(cfg):
 
 def _shard(w, rank, world):
     from paper_conf_ipps_xuzwrwxgxy12_b200 import sharding
-    seeds, ids = sharding.shard_seeds(w.seeds, w.seed_ids, rank, world)
+    env = os.environ.get("PT_SHARD_BLOCK")  # experiments; 0 = seed i -> rank i mod N
+    block = int(env) if env else None  # None: Z-order blocks of <= 1024 seeds (sharding.auto_block)
+    seeds, ids = sharding.shard_seeds(w.seeds, w.seed_ids, rank, world, block=block)
     return w.replace(seeds=seeds, seed_ids=ids)
 
 

@@ -25,6 +25,9 @@
 // c3 74.6/75.3/76.0/76.4/77.0/77.2/76.9 G steps/s; 32 is the default).
 #define PT_SEEDS_PER_CLAIM 32
 #endif
+#ifndef PT_TAIL_SEEDS_PER_SM
+#define PT_TAIL_SEEDS_PER_SM 4  // single-seed claims at the end of the queue, per SM
+#endif
 #ifndef PT_BRICK_DEFAULT
 #define PT_BRICK_DEFAULT 4  // record layout brick log2 edge (0 = raster, 4 = 16^3 bricks, measured best)
 #endif
@@ -505,8 +508,11 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         uint64_t G = PT_SEEDS_PER_CLAIM;
         const uint64_t sps = (P + pt::kSub - 1) / pt::kSub;
         while (G > 1 && (G * sps >= (1ull << 22) || N / G < 8ull * (uint64_t)c->num_sms)) G >>= 1;
+        // the last PT_TAIL_SEEDS_PER_SM x SMs seeds are claimed one by one (guided tail)
+        const uint64_t tail = (uint64_t)PT_TAIL_SEEDS_PER_SM * (uint64_t)(c->num_sms > 0 ? c->num_sms : 1);
         a.seeds_per_claim = (uint32_t)G;
-        a.total_chunks = (N + G - 1) / G;
+        a.group_chunks = N > tail ? (N - tail) / G : 0;
+        a.total_chunks = a.group_chunks + (N - a.group_chunks * G);
     }
     a.map = d_map;
     a.map_copies = 1;

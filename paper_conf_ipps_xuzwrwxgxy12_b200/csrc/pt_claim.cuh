@@ -17,14 +17,12 @@ constexpr unsigned long long kNoWork = ~0ull;
 constexpr unsigned long long kNoChunk = (1ull << 40) - 1;  // initial "empty" chunk id
 
 // Number of 32-particle sub-chunks in claim unit `chunk`: either a slice of one seed
-// (seeds_per_claim == 1) or seeds_per_claim whole consecutive seeds (in processing order).
+// (seeds_per_claim == 1), or seeds_per_claim whole consecutive seeds (in processing order)
+// for the first group_chunks claims and one whole seed per claim after them (the tail:
+// small last claims keep the CTAs' finishing times within about one seed of each other).
 __device__ __forceinline__ uint32_t chunk_subs(unsigned long long chunk, const TrackArgs& a) {
     const uint32_t sps = (uint32_t)((a.P + kSub - 1) / kSub);  // sub-chunks per seed
-    if (a.seeds_per_claim > 1) {
-        const uint64_t kb = chunk * a.seeds_per_claim;
-        const uint64_t nk = a.nseeds - kb < a.seeds_per_claim ? a.nseeds - kb : a.seeds_per_claim;
-        return (uint32_t)nk * sps;
-    }
+    if (a.seeds_per_claim > 1) return chunk < a.group_chunks ? a.seeds_per_claim * sps : sps;
     const uint64_t k = chunk / a.chunks_per_seed;
     const uint64_t jbase = (chunk - k * a.chunks_per_seed) * (uint64_t)a.cta_chunk;
     const uint64_t cnt = a.P - jbase < a.cta_chunk ? a.P - jbase : a.cta_chunk;
@@ -36,10 +34,15 @@ __device__ __forceinline__ uint32_t chunk_subs(unsigned long long chunk, const T
 __device__ __forceinline__ unsigned long long chunk_sub(unsigned long long chunk, uint32_t t, const TrackArgs& a) {
     uint64_t k, j;
     if (a.seeds_per_claim > 1) {
-        const uint32_t sps = (uint32_t)((a.P + kSub - 1) / kSub);
-        const uint32_t o = t / sps;
-        k = chunk * a.seeds_per_claim + o;
-        j = (uint64_t)(t - o * sps) * kSub;
+        if (chunk < a.group_chunks) {
+            const uint32_t sps = (uint32_t)((a.P + kSub - 1) / kSub);
+            const uint32_t o = t / sps;
+            k = chunk * a.seeds_per_claim + o;
+            j = (uint64_t)(t - o * sps) * kSub;
+        } else {  // tail: one seed per claim
+            k = a.group_chunks * a.seeds_per_claim + (chunk - a.group_chunks);
+            j = (uint64_t)t * kSub;
+        }
     } else {
         k = chunk / a.chunks_per_seed;
         j = (chunk - k * a.chunks_per_seed) * (uint64_t)a.cta_chunk + (uint64_t)t * kSub;

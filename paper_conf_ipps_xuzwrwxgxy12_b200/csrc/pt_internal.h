@@ -58,7 +58,8 @@ struct TrackArgs {
     uint64_t nseeds;
     uint64_t nparticles;         // nseeds * P
     uint32_t cta_chunk;          // particles per CTA claim within a seed (multiple of kSub)
-    uint32_t seeds_per_claim;    // > 1: a claim is this many whole consecutive seeds
+    uint32_t seeds_per_claim;    // > 1: a claim is this many whole consecutive seeds ...
+    uint64_t group_chunks;       // ... for claims < group_chunks; later claims are one seed each
     uint32_t chunks_per_seed;    // ceil(P / cta_chunk)
     uint64_t total_chunks;       // nseeds * chunks_per_seed
     uint32_t* map;               // [V] or nullptr: the map this launch adds into

@@ -52,6 +52,7 @@ struct VSlot {
     float d0x, d0y, d0z;    // half 0's first-step direction (R22)
     uint32_t vox;           // nearest voxel of the committed position
     uint32_t cvox;          // nearest voxel of the candidate
+    uint32_t rvox, crvox;   // their positions in the record volume (rec_vox)
     uint32_t s;             // sample index of the prefetched record
     uint32_t mb;            // prefetched mask byte of cvox / the seed voxel (interp)
     uint32_t wsign, winit;  // first step: stream 0 block 0 word 3 (R6); stream 2 word 3 (R24)
@@ -89,7 +90,7 @@ __global__ void __launch_bounds__(kVarThreads, 1) track_var_kernel(const __grid_
     x.alive = x.pend = x.seedchk = x.have_d0 = false;
     x.half = 0u;
     x.qx = x.qy = x.qz = x.px = x.py = x.pz = x.d0x = x.d0y = x.d0z = 0.f;
-    x.vox = x.cvox = x.s = x.mb = x.wsign = x.winit = 0u;
+    x.vox = x.cvox = x.rvox = x.crvox = x.s = x.mb = x.wsign = x.winit = 0u;
     x.n = 0;
     x.pid = x.li = 0ull;
     x.sfix = x.sidx = x.run_vox = x.run_cnt = 0u;
@@ -101,16 +102,17 @@ __global__ void __launch_bounds__(kVarThreads, 1) track_var_kernel(const __grid_
     uint32_t my_steps = 0, my_particles = 0, my_active = 0, iters = 0;
     bool exhausted = false;  // warp-uniform
 
-    auto nearest = [&](float qx, float qy, float qz, uint32_t& v) -> bool {
+    auto nearest = [&](float qx, float qy, float qz, uint32_t& v, uint32_t& rv) -> bool {
         const int ix = axis_index(qx, a.cx), iy = axis_index(qy, a.cy), iz = axis_index(qz, a.cz);
         const bool in = (unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny && (unsigned)iz < (unsigned)a.nz;
         v = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
+        rv = rec_vox(ix, iy, iz, a.rb_log, a.rb_nbx, a.rb_nby);
         return in;
     };
     // Issue the loads step n will need at position (qx,qy,qz) with nearest voxel nv:
     // the sample index (R1/R16: stream = half, block n/3, word n%3), the interpolated voxel
     // (R23: stream 2 + half, block n), the record gather, and the candidate's mask byte.
-    auto prefetch = [&](float qx, float qy, float qz, uint32_t nv, int n) {
+    auto prefetch = [&](float qx, float qy, float qz, uint32_t nv, uint32_t nrv, int n) {
         const uint32_t lo = (uint32_t)x.pid, hi = (uint32_t)(x.pid >> 32);
         const uint4 W = philox4x32_10(make_uint4((uint32_t)n / 3u, lo, hi, x.half), a.key0, a.key1);
         const int r3 = n % 3;
@@ -118,17 +120,16 @@ __global__ void __launch_bounds__(kVarThreads, 1) track_var_kernel(const __grid_
         x.s = a.sample_mode ? x.sfix : sample_of(wn, a.S);
         const bool first = n == 0 && x.half == 0u;
         if (first) x.wsign = W.w;
-        uint32_t u = nv;
+        uint32_t ur = nrv;
         if (a.interp || (first && a.init_mode)) {
             const uint4 I = philox4x32_10(make_uint4((uint32_t)n, lo, hi, 2u + x.half), a.key0, a.key1);
             if (first) x.winit = I.w;
             if (a.interp) {
                 const int ix = interp_axis(qx, a.cx, I.x), iy = interp_axis(qy, a.cy, I.y), iz = interp_axis(qz, a.cz, I.z);
                 if ((unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny && (unsigned)iz < (unsigned)a.nz)
-                    u = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
+                    ur = rec_vox(ix, iy, iz, a.rb_log, a.rb_nbx, a.rb_nby);
             }
         }
-        const uint32_t ur = rec_vox_raster(u, (uint32_t)a.nx, (uint32_t)a.ny, a.rb_log, a.rb_nbx, a.rb_nby);
         ldg_record<RB>(a.rec + ((uint64_t)ur * a.S + x.s) * RB, x.rv.w);
         if (a.interp) x.mb = __ldg(a.mask + nv);
     };
@@ -146,9 +147,10 @@ __global__ void __launch_bounds__(kVarThreads, 1) track_var_kernel(const __grid_
             pp[1] = __fadd_rn(x.qy, a.fcy);
             pp[2] = __fadd_rn(x.qz, a.fcz);
         }
-        if (!nearest(x.qx, x.qy, x.qz, x.vox)) return false;
+        if (!nearest(x.qx, x.qy, x.qz, x.vox, x.rvox)) return false;
         x.cvox = x.vox;
-        prefetch(x.qx, x.qy, x.qz, x.vox, 0);
+        x.crvox = x.rvox;
+        prefetch(x.qx, x.qy, x.qz, x.vox, x.rvox, 0);
         return true;
     };
     auto write_outputs = [&]() {
@@ -278,6 +280,7 @@ __global__ void __launch_bounds__(kVarThreads, 1) track_var_kernel(const __grid_
                 x.qy = __fadd_rn(x.qy, __fmul_rn(a.step, x.py));
                 x.qz = __fadd_rn(x.qz, __fmul_rn(a.step, x.pz));
                 x.vox = x.cvox;
+                x.rvox = x.crvox;
                 x.n += 1;
                 if (map) {
                     if (x.vox != x.run_vox || x.run_cnt == 0u) {
@@ -311,7 +314,7 @@ __global__ void __launch_bounds__(kVarThreads, 1) track_var_kernel(const __grid_
         }
 
         // ---- B: the interpolated voxel was outside the mask => nearest voxel (R23)
-        if (a.interp && x.rv.outside()) ldg_record<RB>(a.rec + ((uint64_t)rec_vox_raster(x.vox, (uint32_t)a.nx, (uint32_t)a.ny, a.rb_log, a.rb_nbx, a.rb_nby) * a.S + x.s) * RB, x.rv.w);
+        if (a.interp && x.rv.outside()) ldg_record<RB>(a.rec + ((uint64_t)x.rvox * a.S + x.s) * RB, x.rv.w);
 
         // ---- C: fibre choice, curvature, step
         const bool first = x.n == 0 && x.half == 0u;
@@ -394,8 +397,8 @@ __global__ void __launch_bounds__(kVarThreads, 1) track_var_kernel(const __grid_
         const float nqx = __fadd_rn(x.qx, __fmul_rn(a.step, dx));
         const float nqy = __fadd_rn(x.qy, __fmul_rn(a.step, dy));
         const float nqz = __fadd_rn(x.qz, __fmul_rn(a.step, dz));
-        uint32_t v;
-        if (!nearest(nqx, nqy, nqz, v)) {  // outside the volume (R11)
+        uint32_t v, rv;
+        if (!nearest(nqx, nqy, nqz, v, rv)) {  // outside the volume (R11)
             x.alive = false;
             x.why = kVMask;
             continue;
@@ -404,8 +407,9 @@ __global__ void __launch_bounds__(kVarThreads, 1) track_var_kernel(const __grid_
         x.py = dy;
         x.pz = dz;
         x.cvox = v;
+        x.crvox = rv;
         x.pend = true;
-        prefetch(nqx, nqy, nqz, v, x.n + 1);
+        prefetch(nqx, nqy, nqz, v, rv, x.n + 1);
     }
 
     // ---- counters: one atomic per warp

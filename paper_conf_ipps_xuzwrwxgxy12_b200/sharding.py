@@ -20,11 +20,54 @@ def shard_indices(nseeds: int, rank: int, world: int) -> np.ndarray:
     return np.arange(rank, nseeds, world, dtype=np.int64)
 
 
-def shard_seeds(seeds: np.ndarray, seed_ids, rank: int, world: int):
-    """(seeds, global seed ids) of this rank's shard."""
+def _spread3(v: np.ndarray) -> np.ndarray:
+    x = v.astype(np.uint64) & np.uint64(0x3FF)
+    for sh, m in ((16, 0x030000FF), (8, 0x0300F00F), (4, 0x030C30C3), (2, 0x09249249)):
+        x = (x | (x << np.uint64(sh))) & np.uint64(m)
+    return x
+
+
+def morton_order(seeds: np.ndarray) -> np.ndarray:
+    """Stable Z-order permutation of the seeds by their voxel (10 bits per axis, coordinates
+    clamped to [0, 1023]) -- the order pt_track claims seeds in on the device."""
+    c = np.clip(np.floor(np.asarray(seeds, np.float64)), 0, 1023).astype(np.uint64)
+    key = _spread3(c[:, 0]) | (_spread3(c[:, 1]) << np.uint64(1)) | (_spread3(c[:, 2]) << np.uint64(2))
+    return np.argsort(key, kind="stable")
+
+
+def shard_blocks(seeds: np.ndarray, rank: int, world: int, block: int = 1024) -> np.ndarray:
+    """Block-interleaved spatial sharding: the seeds in Z-order are cut into blocks of
+    `block` consecutive seeds (a compact 3-D neighbourhood each) and block b goes to rank
+    b mod world.  Every rank draws blocks from the whole volume, so the work balances
+    statistically like the plain interleave, but a rank's seeds stay as dense as on one
+    GPU inside each block: neighbouring seeds share tracts and hence L1/L2 lines (plain
+    i mod world thins every neighbourhood by world and cost ~8 % per rank at 8 ranks).
+    Emulated on c3 at 8 ranks: block 64 / 256 / 512 / 1024 / 2048 project
+    950 / 970 / 981 / 999-1003 / 988 G steps/s (plain interleave 928 G); larger blocks keep
+    more locality but balance worse (max/mean 1.003 -> 1.04)."""
+    if world < 1 or not (0 <= rank < world):
+        raise ValueError(f"bad rank {rank} / world {world}")
+    if block < 1:
+        raise ValueError("block must be >= 1")
+    perm = morton_order(seeds)
+    b = np.arange(perm.size, dtype=np.int64) // block
+    return np.sort(perm[b % world == rank])
+
+
+def auto_block(nseeds: int, world: int, cap: int = 1024) -> int:
+    """Z-order block size: `cap` seeds, but small enough that every rank gets >= 16 blocks."""
+    return max(1, min(cap, nseeds // (16 * max(1, world))))
+
+
+def shard_seeds(seeds: np.ndarray, seed_ids, rank: int, world: int, block=None):
+    """(seeds, global seed ids) of this rank's shard (block-interleaved in Z-order,
+    `shard_blocks`, block None = auto_block; block = 0 selects the plain interleave seed
+    i -> rank i mod world)."""
     n = int(seeds.shape[0])
+    if block is None:
+        block = auto_block(n, world)
     ids = np.arange(n, dtype=np.uint64) if seed_ids is None else np.asarray(seed_ids, np.uint64)
-    sel = shard_indices(n, rank, world)
+    sel = shard_indices(n, rank, world) if block == 0 or world == 1 else shard_blocks(seeds, rank, world, block)
     return np.ascontiguousarray(seeds[sel]), np.ascontiguousarray(ids[sel])
 
 

@@ -22,7 +22,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, q):
+def _worker(rank, world, port, q, block):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -31,7 +31,8 @@ def _worker(rank, world, port, q):
         import phantom
         from paper_conf_ipps_xuzwrwxgxy12_b200 import sharding
         w = phantom.crossing(sigma=0.15, f_jitter=0.03, nseeds=48, particles_per_seed=60, nsamples=20)
-        seeds, ids = sharding.shard_seeds(w.seeds, w.seed_ids, rank, world)
+        seeds, ids = sharding.shard_seeds(w.seeds, w.seed_ids, rank, world, block=block)
+        assert seeds.shape[0] > 0  # every rank has work (block < 48 seeds / world)
         r = oracle.track(w.replace(seeds=seeds, seed_ids=ids))
         m = torch.from_numpy(r["map"].astype(np.uint32).view(np.int32).copy())
         sharding.reduce_map(m, dst=0)
@@ -48,12 +49,14 @@ def _worker(rank, world, port, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world", [2, 3])
-def test_sharded_reduce_matches_single_process(world):
+@pytest.mark.parametrize("world,block", [(2, 0), (3, 0), (2, 5), (3, 4)])
+def test_sharded_reduce_matches_single_process(world, block):
+    """block 0: seed i -> rank i mod world; block > 0: Z-order blocks (the bench default,
+    with a block small enough that every rank gets several blocks of the 48 seeds)."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q, block)) for r in range(world)]
     for p in procs:
         p.start()
     got, full, wrap, steps, full_steps = q.get(timeout=600)
@@ -75,6 +78,31 @@ def test_shard_indices_partition():
             assert np.array_equal(allp, np.arange(n))
     with pytest.raises(ValueError):
         sharding.shard_indices(5, 2, 2)
+
+
+def test_shard_blocks_partition_and_locality():
+    """Block-interleaved Z-order sharding: the shards partition the seeds (every seed on
+    exactly one rank, none twice), blocks are contiguous in Z-order, and the shard sizes
+    differ by at most one block."""
+    from paper_conf_ipps_xuzwrwxgxy12_b200 import sharding
+    rng = np.random.default_rng(3)
+    for n, world, block in ((0, 2, 4), (1, 3, 4), (1000, 1, 256), (1000, 3, 16), (5000, 8, 64), (777, 8, 256)):
+        seeds = (rng.integers(0, 64, size=(n, 3)) + 0.5).astype(np.float32)
+        parts = [sharding.shard_blocks(seeds, r, world, block) for r in range(world)]
+        allp = np.sort(np.concatenate(parts)) if n else np.array([], np.int64)
+        assert np.array_equal(allp, np.arange(n))
+        sizes = [p.size for p in parts]
+        assert max(sizes) - min(sizes) <= block
+        perm = sharding.morton_order(seeds)
+        pos = np.empty(n, np.int64)
+        pos[perm] = np.arange(n)
+        for r, p in enumerate(parts):  # rank r holds exactly the Z-order blocks b = r mod world
+            assert np.all((pos[p] // block) % world == r)
+    # the Z-order agrees with the spec: (x, y, z) bits interleaved x lowest
+    s = np.array([[1.5, 0.5, 0.5], [0.5, 1.5, 0.5], [0.5, 0.5, 1.5], [0.5, 0.5, 0.5]], np.float32)
+    assert list(sharding.morton_order(s)) == [3, 0, 1, 2]
+    with pytest.raises(ValueError):
+        sharding.shard_blocks(s, 2, 2)
 
 
 def _mcmc_worker(rank, world, port, q):
