@@ -668,6 +668,9 @@ def run_ours(args):
                              % (V * w.volume.nsamples * rb / 1e9)},
             "seeds_per_s": total_seeds * args.steps / (ms * 1e-3),
             "active_lane_fraction": lane_frac,
+            # PT_KERNEL_SPEC ablation: fraction of steps taken with the speculative 2nd gather
+            "spec_step_fraction": (st.get("spec_hits", 0) / my_steps) if my_steps else None,
+            "steps_per_lane_iteration": (my_steps / st["lane_active"]) if st["lane_active"] else None,
             "lengths": lengths,
             "emulated_scaling": emulated,
             "roofline": roof,

@@ -83,6 +83,11 @@ typedef enum { PT_END_MASK = 0, PT_END_CURV = 1, PT_END_MAXLEN = 2 } pt_reason;
                                         between segments, schedule of pt_set_segments.
                                         Same results; synchronous; not combinable with
                                         PT_REC_PATHS, PT_REC_CONN or the NEXT-3 variants */
+#define PT_KERNEL_SPEC    (1u << 17) /* ablation: the speculative kernel (a second record
+                                        gather per lane and iteration at the extrapolated
+                                        next voxel, two steps per iteration on a hit;
+                                        DESIGN.md §13) instead of the default 3-step-round
+                                        kernel; same results                             */
 
 /* Create a context on CUDA device `cuda_device` (the caller's current device is left
  * unchanged).  *out receives the context or NULL.  The stream defaults to the legacy
@@ -209,7 +214,8 @@ pt_status pt_get_paths(pt_ctx* ctx, pt_paths* out);
  *   map_sum          : sum of the map cells after the call (mod 2^64)
  *   overflow         : 1 if a map cell wrapped (detected as map_sum != expected)
  *   kernel_ms        : device time of the tracking kernel (CUDA events on ctx's stream)
- *   track_ms         : device time of the whole pt_track enqueue (zeroing, kernel, checks) */
+ *   track_ms         : device time of the whole pt_track enqueue (zeroing, kernel, checks)
+ *   spec_hits        : steps taken with the speculative record (PT_KERNEL_SPEC; else 0) */
 typedef struct {
     uint64_t total_steps;
     uint64_t particles;
@@ -219,6 +225,7 @@ typedef struct {
     int32_t overflow;
     float kernel_ms;
     float track_ms;
+    uint64_t spec_hits;
 } pt_stats;
 pt_status pt_get_stats(pt_ctx* ctx, pt_stats* out);
 

@@ -27,7 +27,7 @@ __all__ = [
     "PT_REC_PATHS", "PT_MAP_ACCUMULATE", "PT_KERNEL_SIMPLE", "PT_SEED_ORDER_INPUT",
     "PT_SAMPLE_PER_STREAMLINE", "PT_REC_CONN", "PT_BIDIR", "PT_INTERP", "PT_INIT_RANDOM",
     "PT_INIT_FWEIGHT", "PT_KERNEL_VARIANT", "variant_flags", "pt_mcmc", "pt_get_mcmc_stats",
-    "pt_mcmc_to_volume", "pt_dwi_shape", "pt_mcmc_params", "PT_KERNEL_SEGMENTED", "pt_set_segments",
+    "pt_mcmc_to_volume", "pt_dwi_shape", "pt_mcmc_params", "PT_KERNEL_SEGMENTED", "pt_set_segments", "PT_KERNEL_SPEC",
     "SEGMENTS_B", "SEGMENTS_C", "pt_load_targets", "pt_get_connectivity", "PT_END_MASK", "PT_END_CURV",
     "PT_END_MAXLEN", "EXPORTS",
 ]
@@ -50,6 +50,7 @@ PT_INIT_RANDOM = 1 << 13
 PT_INIT_FWEIGHT = 1 << 14
 PT_KERNEL_VARIANT = 1 << 15
 PT_KERNEL_SEGMENTED = 1 << 16
+PT_KERNEL_SPEC = 1 << 17  # ablation: speculative 2nd-gather kernel (pt_spec.cu)
 # the paper's increasing-interval segmentation strategies
 SEGMENTS_B = (1, 2, 5, 10, 20, 50, 100, 200, 500)
 SEGMENTS_C = (1, 1, 2, 2, 5, 5, 10, 10, 20, 20, 50, 50, 100, 100, 200, 200)
@@ -97,7 +98,8 @@ class pt_stats(ctypes.Structure):
     _fields_ = [("total_steps", ctypes.c_uint64), ("particles", ctypes.c_uint64),
                 ("lane_active", ctypes.c_uint64), ("lane_slots", ctypes.c_uint64),
                 ("map_sum", ctypes.c_uint64), ("overflow", ctypes.c_int32),
-                ("kernel_ms", ctypes.c_float), ("track_ms", ctypes.c_float)]
+                ("kernel_ms", ctypes.c_float), ("track_ms", ctypes.c_float),
+                ("spec_hits", ctypes.c_uint64)]
 
 
 class pt_dwi_shape(ctypes.Structure):

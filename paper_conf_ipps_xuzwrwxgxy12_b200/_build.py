@@ -10,7 +10,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.environ.get("PT_LIB") or os.path.join(PKG, "libpt.so")  # PT_LIB: experiment builds
-SOURCES = ["pt_api.cu", "pt_kernels.cu", "pt_variants.cu", "pt_mcmc.cu", "pt_segmented.cu"]
+SOURCES = ["pt_api.cu", "pt_kernels.cu", "pt_variants.cu", "pt_mcmc.cu", "pt_segmented.cu", "pt_spec.cu"]
 HEADERS = ["pt_device.cuh", "pt_internal.h", "pt_claim.cuh"]
 
 NVCC_FLAGS = [

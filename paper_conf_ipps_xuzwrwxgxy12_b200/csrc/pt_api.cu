@@ -570,6 +570,9 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     } else if (variant)
         CK(pt::launch_track_var(a, c->vol.nfibres, c->vol.dtype == PT_F16, c->num_sms, st),
            "pt_track: variant tracking kernel launch");
+    else if ((fl & PT_KERNEL_SPEC) && !(fl & PT_KERNEL_SIMPLE))
+        CK(pt::launch_track_spec(a, c->vol.nfibres, c->vol.dtype == PT_F16, c->num_sms, st),
+           "pt_track: tracking kernel launch");
     else
         CK(pt::launch_track(a, c->vol.nfibres, c->vol.dtype == PT_F16, (fl & PT_KERNEL_SIMPLE) != 0, c->num_sms, st),
            "pt_track: tracking kernel launch");
@@ -652,6 +655,7 @@ pt_status pt_get_stats(pt_ctx* c, pt_stats* out) {
     out->lane_active = s[pt::kStatLaneActive];
     out->lane_slots = s[pt::kStatLaneSlots];
     out->map_sum = s[pt::kStatMapAfter];
+    out->spec_hits = s[pt::kStatSpecHits];
     out->overflow = (c->last_map && s[pt::kStatMapAfter] != s[pt::kStatMapBefore] + s[pt::kStatSteps]) ? 1 : 0;
     float ms = 0.f;
     CK(cudaEventElapsedTime(&ms, c->ev[1], c->ev[2]), "pt_get_stats: kernel time");

@@ -37,7 +37,8 @@ enum StatIdx {
     kStatMapBefore = 5,  // sum of map cells before the kernel (accumulate mode)
     kStatQueue = 6,      // work-queue counter (chunks claimed)
     kStatBadInput = 7,   // repack: non-finite value inside the mask
-    kNumStats = 8
+    kStatSpecHits = 8,   // steps taken with the speculative record (pt_spec.cu)
+    kNumStats = 9
 };
 
 struct TrackArgs {
@@ -127,6 +128,9 @@ cudaError_t run_segmented(const TrackArgs& a, int F, bool half, const SegState& 
 // Launchers (return the launch error, if any).
 cudaError_t launch_track(const TrackArgs& a, int nfibres, bool half, bool simple, int num_sms,
                          cudaStream_t st);
+// Speculative tracking kernel (PT_KERNEL_SPEC ablation): persistent + refill + a second
+// gather at the extrapolated next voxel (pt_spec.cu).
+cudaError_t launch_track_spec(const TrackArgs& a, int nfibres, bool half, int num_sms, cudaStream_t st);
 // NEXT-3 variant kernel (bidirectional / interpolation / first-fibre modes; also runs the
 // default semantics when forced with PT_KERNEL_VARIANT).
 cudaError_t launch_track_var(const TrackArgs& a, int nfibres, bool half, int num_sms, cudaStream_t st);

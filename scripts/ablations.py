@@ -7,7 +7,7 @@
   (iii) fp32 vs fp16 records (c3 vs c4)
   (v)   raster vs Morton seed order (PT_SEED_ORDER_INPUT)
   (vi)  raster vs bricked record layout (PT_BRICK=0 vs the default 16^3 bricks)
-  plus the NEXT-3 variant kernel on the default semantics (PT_KERNEL_VARIANT).
+  plus the speculative-gather kernel (PT_KERNEL_SPEC) and the NEXT-3 variant kernel on the default semantics (PT_KERNEL_VARIANT).
 
 Every run's total steps must equal the main kernel's (same parity contract: the results
 are identical, only the schedule differs).  Prints one JSON line per variant and a markdown
@@ -50,6 +50,7 @@ def main():
 
     variants = [
         ("main (persistent, lane refill, Morton)", 0, None, w),
+        ("speculative 2nd gather, 2 steps/iteration on a hit (PT_KERNEL_SPEC)", pt.PT_KERNEL_SPEC, None, w),
         ("(v) raster seed order", pt.PT_SEED_ORDER_INPUT, None, w),
         ("variant kernel, default semantics", pt.PT_KERNEL_VARIANT, None, w),
         ("(i) no refill, one thread per particle (A_MaxStep)", pt.PT_KERNEL_SIMPLE, None, w),
