@@ -31,6 +31,9 @@
 #ifndef PT_REFILL_MIN
 #define PT_REFILL_MIN 2  // free lanes a warp waits for before refilling (amortises the refill block)
 #endif
+#ifndef PT_CTA_MINB
+#define PT_CTA_MINB 1  // resident CTAs per SM the persistent kernel is compiled for (occupancy sweeps)
+#endif
 #ifndef PT_SLOTS
 #define PT_SLOTS 1  // particles per lane in the persistent kernel (1 or 2; 2 measured no faster)
 #endif
@@ -72,7 +75,7 @@ struct Cta {
 // BL: record layout, log2 brick edge (0 = raster), a compile-time constant so
 // the record position costs a few shift/mask instructions with immediates.
 template <int F, bool HALF, bool REFILL, bool OUT, int SLOTS, int BL>
-__global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, 1) track_kernel(const __grid_constant__ TrackArgs a) {
+__global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, REFILL ? PT_CTA_MINB : 1) track_kernel(const __grid_constant__ TrackArgs a) {
     using R = Rec<F, HALF>;
     constexpr int RB = R::kBytes;
     constexpr int TPB = Cta<REFILL, SLOTS>::kTPB;
