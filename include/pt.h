@@ -87,7 +87,9 @@ typedef enum { PT_END_MASK = 0, PT_END_CURV = 1, PT_END_MAXLEN = 2 } pt_reason;
                                         gather per lane and iteration at the extrapolated
                                         next voxel, two steps per iteration on a hit;
                                         DESIGN.md §13) instead of the default 3-step-round
-                                        kernel; same results                             */
+                                        kernel; same results.  PT_ERR_ARG with
+                                        PT_KERNEL_SIMPLE, PT_KERNEL_SEGMENTED or a NEXT-3
+                                        variant flag                                     */
 
 /* Create a context on CUDA device `cuda_device` (the caller's current device is left
  * unchanged).  *out receives the context or NULL.  The stream defaults to the legacy

@@ -379,6 +379,8 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         return fail(c, PT_ERR_ARG, "pt_track: PT_KERNEL_SEGMENTED runs the base semantics with nsteps/reason/end outputs only");
     if (variant && (p->flags & PT_KERNEL_SIMPLE))
         return fail(c, PT_ERR_ARG, "pt_track: PT_KERNEL_SIMPLE cannot run the NEXT-3 variants");
+    if ((p->flags & PT_KERNEL_SPEC) && (variant || segmented || (p->flags & PT_KERNEL_SIMPLE)))
+        return fail(c, PT_ERR_ARG, "pt_track: PT_KERNEL_SPEC runs the base semantics only (no SIMPLE, SEGMENTED or NEXT-3 variants)");
     if ((p->flags & PT_INIT_RANDOM) && (p->flags & PT_INIT_FWEIGHT))
         return fail(c, PT_ERR_ARG, "pt_track: PT_INIT_RANDOM and PT_INIT_FWEIGHT are exclusive");
     const uint64_t H = (p->flags & PT_BIDIR) ? 2 : 1;   // output entries per particle
@@ -570,7 +572,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     } else if (variant)
         CK(pt::launch_track_var(a, c->vol.nfibres, c->vol.dtype == PT_F16, c->num_sms, st),
            "pt_track: variant tracking kernel launch");
-    else if ((fl & PT_KERNEL_SPEC) && !(fl & PT_KERNEL_SIMPLE))
+    else if (fl & PT_KERNEL_SPEC)
         CK(pt::launch_track_spec(a, c->vol.nfibres, c->vol.dtype == PT_F16, c->num_sms, st),
            "pt_track: tracking kernel launch");
     else

@@ -83,3 +83,11 @@ def test_spec_whole_brain_sampled(pt, tracker):
     g = gpu_run(tracker, w, _rec(pt))
     r = oracle.track(w, threads=_threads())
     assert_parity(g, r)
+
+
+def test_spec_rejects_other_kernels(pt, tracker):
+    w = phantom.config("c1")
+    tracker.load_volume(w.volume)
+    for bad in (pt.PT_KERNEL_SIMPLE, pt.PT_KERNEL_SEGMENTED, pt.PT_BIDIR, pt.PT_KERNEL_VARIANT):
+        with pytest.raises(pt.PtError):
+            tracker.track_workload(w, flags=pt.PT_KERNEL_SPEC | bad)
