@@ -26,7 +26,8 @@
 #include "pt_internal.h"
 
 #ifndef PT_RUNLEN
-#define PT_RUNLEN 1  // merge consecutive visits of a voxel before the RED (0: ablation iv, one RED per step)
+#define PT_RUNLEN 1  // merge consecutive visits of a voxel before the RED (0: ablation iv, one RED per step;
+                     // 2: ablation iv, run-length merge + warp aggregation of same-voxel flushes)
 #endif
 #ifndef PT_REFILL_MIN
 #define PT_REFILL_MIN 2  // free lanes a warp waits for before refilling (amortises the refill block)
@@ -174,7 +175,18 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, REFILL ? PT_CTA_MINB
         x.qz = c ? nz_ : x.qz;
         x.n += c ? 1 : 0;
         if (has_map) {
-#if PT_RUNLEN
+#if PT_RUNLEN == 2
+            // lanes flushing the same voxel form one group (__match_any_sync); the group's
+            // lowest lane issues one RED with the group's summed count (labelled-partition
+            // reduction: every lane of a group passes the same member mask)
+            const bool change = v != x.run_vox;
+            const bool fl = c && change && x.run_cnt != 0u;
+            const uint32_t grp = __match_any_sync(kFull, fl ? x.run_vox : 0xFFFFFFFFu);
+            const uint32_t sum = __reduce_add_sync(grp, fl ? x.run_cnt : 0u);
+            red_add_if(fl && lane == (uint32_t)(__ffs(grp) - 1), map + x.run_vox, sum);
+            x.run_cnt = c ? (change ? 1u : x.run_cnt + 1u) : x.run_cnt;
+            x.run_vox = c ? v : x.run_vox;
+#elif PT_RUNLEN
             const bool change = v != x.run_vox;
             red_add_if(c && change && x.run_cnt != 0u, map + x.run_vox, x.run_cnt);
             x.run_cnt = c ? (change ? 1u : x.run_cnt + 1u) : x.run_cnt;
