@@ -11,11 +11,12 @@
 // Design notes: one lane owns one particle at a time; particles are
 // claimed in chunks of kChunk from a global atomic work queue and dead lanes are refilled
 // with a ballot/popc prefix at the start of every round, so the warp stays converged while
-// path lengths are exponentially distributed.  A round is 3 steps: one
-// Philox block per round supplies the three sample indices (R16).  The gather of the next
-// step's record doubles as the mask test of the candidate voxel (sentinel records, R11);
-// the third step's gather is deferred to the next round's start, where it is issued by
-// the same instruction as the first gather of freshly refilled lanes.
+// path lengths are exponentially distributed.  A round is 3 x PT_ROUND_BLOCKS
+// steps (default 6): each Philox block supplies three sample indices (R16); the first is
+// computed at the round start, the next one before the round's 3rd step.  The gather of
+// the next step's record doubles as the mask test of the candidate voxel (sentinel records,
+// R11); the round's last gather is deferred to the next round's start, where it is issued
+// by the same instruction as the first gather of freshly refilled lanes.
 #include <cuda_runtime.h>
 #include <cub/device/device_radix_sort.cuh>
 
@@ -34,6 +35,9 @@
 #endif
 #ifndef PT_CTA_MINB
 #define PT_CTA_MINB 1  // resident CTAs per SM the persistent kernel is compiled for (occupancy sweeps)
+#endif
+#ifndef PT_ROUND_BLOCKS
+#define PT_ROUND_BLOCKS 2  // Philox blocks (3 steps each) per refill round: 6-step rounds (1: 0.99x, 3: 1.00x)
 #endif
 #ifndef PT_SLOTS
 #define PT_SLOTS 1  // particles per lane in the persistent kernel (1 or 2; 2 measured no faster)
@@ -280,8 +284,14 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, REFILL ? PT_CTA_MINB
         x.px = go ? dx : x.px;
         x.py = go ? dy : x.py;
         x.pz = go ? dz : x.pz;
-        if (k < 2) {
-            const uint32_t w = (k == 0) ? x.W.y : x.W.z;
+        if (k < 3 * PT_ROUND_BLOCKS - 1) {
+            if ((k + 1) % 3 == 0) {
+                // the next step opens the round's next Philox block: a live lane has
+                // committed t0 + k steps, so that block is (n + 1) / 3 (R16)
+                x.W = philox4x32_10(make_uint4(((uint32_t)x.n + 1u) / 3u, (uint32_t)x.pid, (uint32_t)(x.pid >> 32), 0u),
+                                    a.key0, a.key1);
+            }
+            const uint32_t w = ((k + 1) % 3 == 0) ? x.W.x : ((k + 1) % 3 == 1) ? x.W.y : x.W.z;
             const uint32_t sk = a.sample_mode ? x.sfix : sample_of(w, a.S);
             const uint32_t rvx = recv(ix, iy, iz, v);
             ldg_record_if<RB>(go, a.rec + ((uint64_t)rvx * a.S + sk) * RB, x.rv.w);
@@ -382,9 +392,9 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, REFILL ? PT_CTA_MINB
             x.pend = false;
         }
 
-        // ------------------------------------------------ three steps, slots interleaved
+        // ------------------------------------------------ 3 x PT_ROUND_BLOCKS steps, slots interleaved
 #pragma unroll
-        for (int k = 0; k < 3; ++k) {
+        for (int k = 0; k < 3 * PT_ROUND_BLOCKS; ++k) {
 #pragma unroll
             for (int sl = 0; sl < SLOTS; ++sl) step(P[sl], sl, k);
         }
@@ -401,7 +411,7 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, REFILL ? PT_CTA_MINB
         atomicAdd(a.stats + kStatSteps, (unsigned long long)my_steps);
         atomicAdd(a.stats + kStatParticles, (unsigned long long)my_particles);
         atomicAdd(a.stats + kStatLaneActive, (unsigned long long)my_active);
-        atomicAdd(a.stats + kStatLaneSlots, (unsigned long long)rounds * 3ull * 32ull * SLOTS);
+        atomicAdd(a.stats + kStatLaneSlots, (unsigned long long)rounds * (3ull * PT_ROUND_BLOCKS) * 32ull * SLOTS);
     }
 }
 
