@@ -39,6 +39,9 @@
 #ifndef PT_ROUND_BLOCKS
 #define PT_ROUND_BLOCKS 2  // Philox blocks (3 steps each) per refill round: 6-step rounds (1: 0.99x, 3: 1.00x)
 #endif
+#ifndef PT_REC_AFFINE
+#define PT_REC_AFFINE 0  // brick position as a sum of per-axis affine terms (experiment builds: 1)
+#endif
 #ifndef PT_SLOTS
 #define PT_SLOTS 1  // particles per lane in the persistent kernel (1 or 2; 2 measured no faster)
 #endif
@@ -128,8 +131,26 @@ __global__ void __launch_bounds__(Cta<REFILL, SLOTS>::kTPB, REFILL ? PT_CTA_MINB
     bool exhausted = false;  // warp-uniform
 
     // position of voxel (ix, iy, iz) = raster index v in the record volume (rec_vox)
+#if PT_REC_AFFINE
+    // rec_vox as a sum of per-axis terms: with b = BL and u = u_b * 2^b + (u & m),
+    //   (x & m) = x - 2^b x_b, (y & m) << b = 2^b y - 2^2b y_b, (z & m) << 2b = 2^2b z - 2^3b z_b,
+    // so rec_vox = x + x_b Kx + 2^b y + y_b Ky + 2^2b z + z_b Kz (mod 2^32; the exact value
+    // is < 2^32, checked at load) with the constants below
+    const uint32_t rKx = (1u << (3 * BL)) - (1u << BL);
+    const uint32_t rKy = (a.rb_nbx << (3 * BL)) - (1u << (2 * BL));
+    const uint32_t rKz = ((a.rb_nbx * a.rb_nby) << (3 * BL)) - (1u << (3 * BL));
+#endif
     auto recv = [&](int ix, int iy, int iz, uint32_t v) -> uint32_t {
         if (BL == 0) return v;
+#if PT_REC_AFFINE
+        {
+            const uint32_t x = (uint32_t)ix, y = (uint32_t)iy, z = (uint32_t)iz;
+            uint32_t r = x + (x >> BL) * rKx;
+            r += (y >> BL) * rKy + (y << BL);
+            r += (z >> BL) * rKz + (z << (2 * BL));
+            return r;
+        }
+#endif
         constexpr uint32_t m = (1u << BL) - 1u;
         const uint32_t x = (uint32_t)ix, y = (uint32_t)iy, z = (uint32_t)iz;
         const uint32_t br = ((z >> BL) * a.rb_nby + (y >> BL)) * a.rb_nbx + (x >> BL);
