@@ -86,7 +86,7 @@ typedef enum { PT_END_MASK = 0, PT_END_CURV = 1, PT_END_MAXLEN = 2 } pt_reason;
 #define PT_KERNEL_SPEC    (1u << 17) /* ablation: the speculative kernel (a second record
                                         gather per lane and iteration at the extrapolated
                                         next voxel, two steps per iteration on a hit;
-                                        DESIGN.md §13) instead of the default 3-step-round
+                                        DESIGN.md §13) instead of the default 6-step-round
                                         kernel; same results.  PT_ERR_ARG with
                                         PT_KERNEL_SIMPLE, PT_KERNEL_SEGMENTED or a NEXT-3
                                         variant flag                                     */

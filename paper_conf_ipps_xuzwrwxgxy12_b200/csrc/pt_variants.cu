@@ -10,7 +10,7 @@
 //
 // Same work distribution as the main kernel (persistent CTAs, global claims, warp
 // sub-chunks, ballot/popc lane refill; pt_claim.cuh) but one step per iteration instead of
-// 3-step rounds, so a lane's RNG stream position, its half and the interpolation draws stay
+// the main kernel's 6-step rounds, so a lane's RNG stream position, its half and the interpolation draws stay
 // simple per-lane state.  Each step issues the next step's record gather (and, with
 // interpolation, the 1-byte mask read of the candidate's nearest voxel) as soon as the
 // candidate position is known, so one memory latency is exposed per step.  Without
