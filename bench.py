@@ -8,8 +8,9 @@ tracking kernel, the map-sum overflow check) and, for N > 1, the NCCL reduce of 
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config c3]
 
-For N > 1 run under torchrun (one rank per GPU, seeds sharded i mod N, global seed ids).
-Prints ONE JSON line on rank 0.
+For N > 1 bench.py launches itself as N ranks (torch.distributed.run, one process per GPU,
+NCCL) unless it already runs under torchrun; seeds are sharded in Z-order blocks with their
+global ids and the maps are combined with one NCCL reduce.  Prints ONE JSON line on rank 0.
 """
 from __future__ import annotations
 
@@ -178,9 +179,10 @@ def _shard(w, rank, world):
 
 
 def _cpu_sample(w, target_s: float, threads: int):
-    """Oracle on a bounded sample of workload w: every k-th seed x particles j < J, sized
-    from a calibration run so the whole sample takes ~target_s of wall time on `threads`
-    host threads.  Returns (steps/s, description, steps, seconds, sample workload, J)."""
+    """Oracle sample of workload w: every k-th seed x ALL its particles (so the GPU can run
+    the same pids through the bench's own launch and the two maps compare bit for bit),
+    k sized from a calibration run so the sample takes ~target_s of wall time on `threads`
+    host threads.  Returns (sample workload, particles per seed, every)."""
     import oracle
     import phantom
     cal = phantom.wm_seeds(w, every=max(1, w.nseeds // 64))
@@ -190,18 +192,20 @@ def _cpu_sample(w, target_s: float, threads: int):
     rate1 = max(1.0, r["nsteps"].sum() / max(dt, 1e-6))          # steps/s on one core
     mean_len = max(1.0, float(r["nsteps"].mean()))
     particles = target_s * rate1 * threads / mean_len
-    J = int(min(w.particles_per_seed, max(8, particles / max(1, threads * 32))))
-    nseeds = int(max(threads, min(w.nseeds, particles / J)))
+    P = w.particles_per_seed
+    nseeds = int(max(threads, min(w.nseeds, particles / P)))
     every = max(1, w.nseeds // nseeds)
     sub = phantom.wm_seeds(w, every=every)
-    return sub, J, every
+    return sub, P, every
 
 
-def _run_oracle_sample(sub, J, threads):
+def _run_oracle_sample(sub, J, threads, keep=False):
     import oracle
     t = time.perf_counter()
     r = oracle.track(sub, 0, J, want_map=True, threads=threads)
     dt = time.perf_counter() - t
+    if keep:
+        return int(r["nsteps"].sum()), dt, r
     return int(r["nsteps"].sum()), dt
 
 
@@ -225,8 +229,8 @@ def run_reference(args):
         steps += s
         secs += dt
     v = steps / secs
-    desc = (f"{args.config}: every {every}th WM seed ({sub.nseeds} seeds) x particles j<{J} of "
-            f"{w.particles_per_seed}; oracle single-threaded per worker, {threads} worker threads")
+    desc = (f"{args.config}: every {every}th WM seed ({sub.nseeds} seeds) x all {J} particles; "
+            f"oracle single-threaded per worker, {threads} worker threads")
     line = {
         "impl": "reference", "metric": METRIC, "value": v, "unit": "steps/s", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / args.steps,
@@ -422,6 +426,8 @@ def run_mcmc_reference(args):
 # ----------------------------------------------------------------------------- our arm
 
 def run_ours(args):
+    import hashlib
+
     import numpy as np
     import torch
     import torch.distributed as dist
@@ -432,6 +438,9 @@ def run_ours(args):
     world = _env_int("WORLD_SIZE", 1)
     rank = _env_int("RANK", 0)
     local = _env_int("LOCAL_RANK", 0)
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE {world} ranks (launch through "
+                         "bench.py itself or torch.distributed.run with --nproc-per-node {args.gpus})")
     # BENCH_DIST_BACKEND=gloo + BENCH_SINGLE_DEVICE=1: test hook that runs the multi-rank
     # path with every rank on cuda:0 (NCCL cannot put two ranks on one GPU)
     backend = os.environ.get("BENCH_DIST_BACKEND", "nccl")
@@ -443,6 +452,9 @@ def run_ours(args):
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         else:
             dist.init_process_group(backend)
+        print(f"[bench rank {rank}/{world}] process group '{dist.get_backend()}' on cuda:{local} "
+              f"({torch.cuda.get_device_name(local)}), nccl {torch.cuda.nccl.version()}",
+              file=sys.stderr, flush=True)
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
 
@@ -452,31 +464,41 @@ def run_ours(args):
         w = phantom.wm_seeds(w, every=args.seed_every)
     mine = _shard(w, rank, world)
     tr = pt.Tracker(local)
-    tr.load_volume(w.volume)
+    # load through the C ABI from pinned host memory: the paper's Copy3DImagesToGPU (P:L165,
+    # "Transfer" in Table II), reported separately (load) and inside e2e_with_load
+    vol = w.volume
+    dy_h = torch.from_numpy(vol.dyads).pin_memory()
+    f_h = torch.from_numpy(vol.f).pin_memory()
+    m_h = torch.from_numpy(vol.mask).pin_memory()
+
+    def load():
+        tr.load_samples(dy_h, f_h, m_h, vol.nsamples, vol.nfibres)
+        return tr.load_stats()
+
+    load()
+    ls = load()
+    base_flags = args.track_flags | (pt.PT_SAMPLE_PER_STREAMLINE if getattr(w, "sample_mode", 0) else 0)
     if args.segments:
         tr.set_segments({"B": pt.SEGMENTS_B, "C": pt.SEGMENTS_C}.get(args.segments) or
                         [int(x) for x in args.segments.split(",")])
-    base_flags = args.track_flags | (pt.PT_SAMPLE_PER_STREAMLINE if getattr(w, "sample_mode", 0) else 0)
-    V = w.volume.nx * w.volume.ny * w.volume.nz
-    rb = pt.pt_record_bytes(w.volume.nfibres, pt.PT_F16 if w.volume.is_half else pt.PT_F32)
+    V = vol.nx * vol.ny * vol.nz
+    rb = pt.pt_record_bytes(vol.nfibres, pt.PT_F16 if vol.is_half else pt.PT_F32)
     seeds_d = torch.as_tensor(mine.seeds, device=dev).contiguous()
     ids_d = torch.as_tensor(mine.ids().astype(np.int64), device=dev).contiguous()
-    out_map = torch.empty((w.volume.nz, w.volume.ny, w.volume.nx), dtype=torch.int32, device=dev)
+    out_map = torch.empty((vol.nz, vol.ny, vol.nx), dtype=torch.int32, device=dev)
     flush_buf = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)  # > L2 (126 MB)
+    tparams = dict(step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr, max_steps=w.max_steps,
+                   rng_seed=w.rng_seed, particles_per_seed=w.particles_per_seed)
 
     def one_step():
         flush_buf.fill_(1)  # evict L2 between steps
-        tr.track(seeds_d, ids_d, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
-                 max_steps=w.max_steps, rng_seed=w.rng_seed,
-                 particles_per_seed=w.particles_per_seed, out_map=out_map, flags=base_flags,
-                 want_map=not args.no_map)
+        tr.track(seeds_d, ids_d, out_map=out_map, flags=base_flags, want_map=not args.no_map, **tparams)
         if world > 1 and not args.no_map:
             sharding.reduce_map(out_map, dst=0)  # one NCCL reduce; int32 sum == uint32 sum
 
     for _ in range(args.warmup):
         one_step()
     torch.cuda.synchronize()
-    st0 = tr.stats()
 
     clocks = ClockSampler(local)
     clocks.start()
@@ -486,15 +508,13 @@ def run_ours(args):
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
     kern_ms, track_ms = [], []
-    steps_done = 0
     e0.record()
     for _ in range(args.steps):
         one_step()
-        s = tr.stats() if args.per_step_stats else None
-        if s:
+        if args.per_step_stats:
+            s = tr.stats()
             kern_ms.append(s["kernel_ms"])
             track_ms.append(s["track_ms"])
-            steps_done += s["total_steps"]
     e1.record()
     torch.cuda.synchronize()
     if world > 1:
@@ -504,10 +524,16 @@ def run_ours(args):
     st = tr.stats()
     if not args.per_step_stats:
         kern_ms = [st["kernel_ms"]]
-        steps_done = st["total_steps"] * args.steps
     my_steps = st["total_steps"]  # identical every step (deterministic)
+    map_sha = None
+    if rank == 0 and not args.no_map:
+        mh = out_map.cpu().numpy().view(np.uint32)
+        map_sha = hashlib.sha256(mh.tobytes()).hexdigest()
+        if args.dump_map:
+            np.save(args.dump_map, mh)
     t = torch.tensor([ms, float(my_steps), float(mine.nseeds), float(st["lane_active"]),
-                      float(st["lane_slots"])], dtype=torch.float64, device=dev)
+                      float(st["lane_slots"]), float(st["unique_visits"])], dtype=torch.float64, device=dev)
+
     def allreduce(x, op):
         # gloo (test hook) reduces host tensors
         if backend == "gloo" and x.is_cuda:
@@ -522,42 +548,49 @@ def run_ours(args):
         allreduce(tmax, dist.ReduceOp.MAX)
         allreduce(t, dist.ReduceOp.SUM)
         ms = float(tmax[0])
-    total_steps = float(t[1]) if world > 1 else float(my_steps)
-    total_seeds = float(t[2]) if world > 1 else float(mine.nseeds)
+    total_steps = float(t[1])
+    total_seeds = float(t[2])
     lane_frac = float(t[3] / t[4]) if float(t[4]) else None
+    unique_visits = float(t[5])
 
-    # ---- e2e through the C ABI with host buffers (pinned seeds in, pinned map out)
+    # ---- e2e through the C ABI with host buffers (pinned seeds in, pinned map out), and the
+    # same with the sample-volume load (pinned host volumes -> H2D + repack) in every step
     seeds_h = torch.as_tensor(mine.seeds).pin_memory()
     ids_h = torch.as_tensor(mine.ids().astype(np.int64)).pin_memory()
-    map_h = torch.empty((w.volume.nz, w.volume.ny, w.volume.nx), dtype=torch.int32).pin_memory()
+    map_h = torch.empty((vol.nz, vol.ny, vol.nx), dtype=torch.int32).pin_memory()
     e2e_steps = max(1, min(args.steps, 3))
-    tr.track(seeds_h, ids_h, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
-             max_steps=w.max_steps, rng_seed=w.rng_seed, particles_per_seed=w.particles_per_seed,
-             out_map=map_h)  # warm
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    t0 = time.perf_counter()
-    for _ in range(e2e_steps):
+
+    def e2e_step(with_load):
         flush_buf.fill_(1)
-        tr.track(seeds_h, ids_h, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
-                 max_steps=w.max_steps, rng_seed=w.rng_seed,
-                 particles_per_seed=w.particles_per_seed, out_map=map_h, flags=base_flags)
+        if with_load:
+            load()
+        tr.track(seeds_h, ids_h, out_map=map_h, flags=base_flags, **tparams)
         if world > 1:
             # the host map is reduced over the process group as the step's result
             mt = map_h.to(dev, non_blocking=True)
             sharding.reduce_map(mt, dst=0)
             if rank == 0:
                 map_h.copy_(mt)
-    torch.cuda.synchronize()
-    e2e_s = time.perf_counter() - t0
-    te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
-    if world > 1:
-        allreduce(te, dist.ReduceOp.MAX)
-    e2e_value = total_steps * e2e_steps / float(te[0])
+
+    e2e_step(False)  # warm
+    e2e_vals = {}
+    for with_load in (False, True):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(e2e_steps):
+            e2e_step(with_load)
+        torch.cuda.synchronize()
+        te = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
+        if world > 1:
+            allreduce(te, dist.ReduceOp.MAX)
+        e2e_vals[with_load] = total_steps * e2e_steps / float(te[0])
 
     # ---- roofline (dominant kernel = the tracking kernel)
     kms = sum(kern_ms) / len(kern_ms)
+    # SURVEY §8(d) algorithmic bytes per committed step: one record read + one 4-B map
+    # atomic (read-modify-write: 8 B); per particle 12 B of seed + 8 B of id, amortised
     alg_bytes = my_steps * (rb + 8) + mine.nseeds * (12 + 8)
     achieved = alg_bytes / (kms * 1e-3) / 1e9
     peaks = _peaks()
@@ -569,7 +602,7 @@ def run_ours(args):
             "kernel_ms_steps": kern_ms, "track_ms_steps": track_ms}
     gather = None
     if rank == 0 and not args.no_gather_bench:
-        rec_bytes_total = V * w.volume.nsamples * rb
+        rec_bytes_total = V * vol.nsamples * rb
         r_hbm = tr.gather_bench(int(rec_bytes_total), rb)
         r_l2 = tr.gather_bench(64 * 1024 * 1024, rb)
         sec_per_step = max(1, rb // 32)
@@ -582,33 +615,52 @@ def run_ours(args):
                   "sectors_per_step": sec_per_step}
 
     cpu = None
+    parity = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         import oracle
         oracle.build()
         threads = len(os.sched_getaffinity(0))
         sub, J, every = _cpu_sample(w, args.cpu_seconds, threads)
-        s, dt = _run_oracle_sample(sub, J, threads)
+        s, dt, r = _run_oracle_sample(sub, J, threads, keep=True)
         cpu = {"value": s / dt, "unit": "steps/s", "cores": threads, "kind": "oracle", "cpu_model": _cpu_model(),
-               "sample": f"every {every}th WM seed ({sub.nseeds} seeds) x particles j<{J}: "
+               "sample": f"every {every}th WM seed ({sub.nseeds} seeds) x all {J} particles: "
                          f"{s} steps in {dt:.1f} s"}
+        if not args.no_parity:
+            # the same pids through the bench's own launch (flags as timed: no per-particle
+            # outputs) -> map; and through the outputs instantiation -> per-streamline results
+            sd = torch.as_tensor(sub.seeds, device=dev).contiguous()
+            si = torch.as_tensor(sub.ids().astype(np.int64), device=dev).contiguous()
+            gm = tr.track(sd, si, flags=base_flags, **tparams)
+            torch.cuda.synchronize()
+            gmap = gm.cpu().numpy().view(np.uint32).astype(np.uint64)
+            rec = pt.PT_REC_LEN | pt.PT_REC_REASON | pt.PT_REC_END
+            tr.track(sd, si, flags=base_flags | rec, want_map=False, **tparams)
+            torch.cuda.synchronize()
+            g = tr.get_paths()
+            div = ((g["nsteps"].astype(np.int64) != r["nsteps"]) | (g["reason"] != r["reason"]) |
+                   np.any(g["end"].view(np.uint32) != r["end"].view(np.uint32), axis=1))
+            l1 = float(np.abs(gmap.astype(np.int64) - r["map"].astype(np.int64)).sum()) / max(1, int(r["map"].sum()))
+            parity = {"sample": cpu["sample"], "streamlines": int(div.size), "divergent": int(div.sum()),
+                      "divergent_fraction": float(div.mean()), "map_l1_rel": l1,
+                      "map_bit_exact": bool(np.array_equal(gmap, r["map"])),
+                      "kernel": "map: the timed launch (flags as benched); per-streamline: the outputs instantiation",
+                      "bar": "divergent <= 1e-4, map L1 rel <= 1e-4 (north_star); expected 0 / 0"}
 
     emulated = None
     if rank == 0 and world == 1 and args.emulate_ranks:
-        # Projected multi-GPU scaling on ONE GPU: the shard of each rank of an N-way split
-        # (seed i -> rank i mod N, global ids) is timed back to back; N GPUs would finish
-        # when the slowest shard does, plus one NCCL reduce of the map (not timed here).
+        # Projected multi-GPU scaling on ONE GPU: each rank's shard of an N-way split is
+        # timed back to back; N GPUs would finish when the slowest shard does, plus one NCCL
+        # reduce of the map (not timed here).  Context only: SCALE runs measure the real thing.
         emulated = {}
         for N in args.emulate_ranks:
             times, steps_r = [], []
-            for r in range(N):
-                sub = _shard(w, r, N)
-                sd = torch.as_tensor(sub.seeds, device=dev).contiguous()
-                si = torch.as_tensor(sub.ids().astype(np.int64), device=dev).contiguous()
+            for r_ in range(N):
+                sub_ = _shard(w, r_, N)
+                sd = torch.as_tensor(sub_.seeds, device=dev).contiguous()
+                si = torch.as_tensor(sub_.ids().astype(np.int64), device=dev).contiguous()
                 for it in range(2):  # warm-up + timed
                     flush_buf.fill_(1)
-                    tr.track(sd, si, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
-                             max_steps=w.max_steps, rng_seed=w.rng_seed,
-                             particles_per_seed=w.particles_per_seed, out_map=out_map, flags=base_flags)
+                    tr.track(sd, si, out_map=out_map, flags=base_flags, **tparams)
                     st_r = tr.stats()
                 times.append(st_r["track_ms"])
                 steps_r.append(st_r["total_steps"])
@@ -618,11 +670,9 @@ def run_ours(args):
         torch.cuda.synchronize()
 
     lengths = None
-    if rank == 0 and (args.lengths or args.config in PAPER_TABLE2):
+    if rank == 0 and not args.no_lengths and not (base_flags & pt.PT_MAP_UNIQUE):
         # one more (untimed) pass with per-particle lengths: the Eq. 4 / Fig. 5 statistics
-        tr.track(seeds_d, ids_d, step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr,
-                 max_steps=w.max_steps, rng_seed=w.rng_seed, particles_per_seed=w.particles_per_seed,
-                 out_map=out_map, flags=base_flags | pt.PT_REC_LEN)
+        tr.track(seeds_d, ids_d, out_map=out_map, flags=base_flags | pt.PT_REC_LEN, **tparams)
         torch.cuda.synchronize()
         ns = tr.get_paths(nsteps=True, reason=False, end=False, on_device=True)["nsteps"]
         hist = torch.zeros(65536, dtype=torch.int64, device=dev)
@@ -644,7 +694,8 @@ def run_ours(args):
                    "longest": int(nz.max()) if nz.size else 0,
                    "lambda_mle": 1.0 / mean if mean > 0 else None,
                    "lambda_semilog_fit": -slope if slope is not None else None,
-                   "fit_range": [int(xs[0]), int(xs[-1])]}
+                   "fit_range": [int(xs[0]), int(xs[-1])],
+                   "context": "Eq. 4 / Fig. 5 (P:L229-249): exponential fibre-length law"}
         if args.config in PAPER_TABLE2:
             lengths["paper_table2_context"] = PAPER_TABLE2[args.config]
 
@@ -659,27 +710,38 @@ def run_ours(args):
                        "seeds": int(total_seeds), "particles_per_seed": w.particles_per_seed,
                        "particles": int(total_seeds) * w.particles_per_seed,
                        "steps_per_pass": int(total_steps),
-                       "mean_steps_per_streamline": total_steps / (total_seeds * w.particles_per_seed),
-                       "record_bytes": rb, "records": "fp16" if w.volume.is_half else "fp32",
+                       "mean_steps_per_streamline": total_steps / max(1.0, total_seeds * w.particles_per_seed),
+                       "record_bytes": rb, "records": "fp16" if vol.is_half else "fp32",
                        "record_layout": "bricks of %d^3 voxels" % (1 << int(os.environ.get("PT_BRICK", "4")))
                                         if int(os.environ.get("PT_BRICK", "4")) else "raster",
+                       "track_flags": base_flags,
                        "parallelism": f"seed-sharded x{world}" + (" + NCCL reduce" if world > 1 else ""),
                        "l2": "inputs > L2 (record volume %.2f GB) and a 256 MiB L2 flush between steps"
-                             % (V * w.volume.nsamples * rb / 1e9)},
+                             % (V * vol.nsamples * rb / 1e9)},
             "seeds_per_s": total_seeds * args.steps / (ms * 1e-3),
             "active_lane_fraction": lane_frac,
-            # PT_KERNEL_SPEC ablation: fraction of steps taken with the speculative 2nd gather
-            "spec_step_fraction": (st.get("spec_hits", 0) / my_steps) if my_steps else None,
             "steps_per_lane_iteration": (my_steps / st["lane_active"]) if st["lane_active"] else None,
+            "unique_visits_per_pass": int(unique_visits) if (base_flags & pt.PT_MAP_UNIQUE) else None,
+            "parity": parity,
+            "map_sha256": map_sha,
             "lengths": lengths,
+            "load": {"h2d_ms": ls["h2d_ms"], "repack_ms": ls["repack_ms"], "h2d_bytes": ls["h2d_bytes"],
+                     "record_bytes": ls["record_bytes"],
+                     "h2d_gb_per_s": ls["h2d_bytes"] / max(1e-9, ls["h2d_ms"] * 1e-3) / 1e9,
+                     "what": "pt_load_samples from pinned host volumes: the paper's Copy3DImagesToGPU "
+                             "(P:L165, Table II 'Transfer'), per GPU, untimed in value"},
             "emulated_scaling": emulated,
             "roofline": roof,
             "gather_roofline": gather,
             "cpu_baseline": cpu,
-            "e2e": {"value": e2e_value, "unit": "steps/s",
+            "e2e": {"value": e2e_vals[False], "unit": "steps/s",
                     "h2d_bytes_per_step": int(seeds_h.numel() * 4 + ids_h.numel() * 8),
                     "d2h_bytes_per_step": int(map_h.numel() * 4)},
-            # per pt_track: seed_keys + 6 cub radix-sort kernels (seed order), track_kernel, map_sum
+            "e2e_with_load": {"value": e2e_vals[True], "unit": "steps/s",
+                              "h2d_bytes_per_step": int(seeds_h.numel() * 4 + ids_h.numel() * 8 + ls["h2d_bytes"]),
+                              "d2h_bytes_per_step": int(map_h.numel() * 4)},
+            # per pt_track: seed_keys + cub radix sort (upsweep/scan/downsweep x passes), the
+            # tracking kernel, map_sum; counted from the ncu launch list (profiles/)
             "gpu_launches": 9 * args.steps,
             "clocks": ck,
         }
@@ -688,6 +750,25 @@ def run_ours(args):
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def _self_launch(args, argv):
+    """bench.py --gpus N with N > 1 and no torch.distributed environment: re-launch this
+    script as N ranks (torch.distributed.run, one process per GPU, NCCL), with NCCL's
+    communicator initialisation log on stderr so the rank count is visible."""
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    env.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes", "1", "--nproc-per-node", str(args.gpus),
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *argv]
+    print("bench.py: launching " + " ".join(cmd), file=sys.stderr, flush=True)
+    return subprocess.call(cmd, env=env)
 
 
 def main(argv=None):
@@ -705,8 +786,11 @@ def main(argv=None):
     ap.add_argument("--emulate-ranks", type=lambda x: [int(v) for v in x.split(",") if v], default=[],
                     help="e.g. 2,4,8: time each rank's seed shard back to back on one GPU and "
                          "report the projected N-GPU throughput (max shard time)")
-    ap.add_argument("--lengths", action="store_true",
-                    help="report streamline-length statistics (untimed extra pass with PT_REC_LEN)")
+    ap.add_argument("--no-lengths", action="store_true",
+                    help="skip the streamline-length statistics (untimed extra pass with PT_REC_LEN)")
+    ap.add_argument("--no-parity", action="store_true",
+                    help="skip the GPU run of the cpu_baseline sample (the parity report)")
+    ap.add_argument("--dump-map", default="", help="rank 0 saves the (reduced) map of the last step (.npy)")
     ap.add_argument("--tag", default="", help="free-form label echoed by experiment scripts")
     ap.add_argument("--seed-every", type=int, default=1,
                     help="diagnostic (profiling only): every k-th seed of the workload")
@@ -716,7 +800,10 @@ def main(argv=None):
     ap.add_argument("--segments", default="",
                     help="schedule of the PT_KERNEL_SEGMENTED ablation (--track-flags 65536): "
                          "B, C or a comma list of intervals (the paper's NumIteration[])")
+    argv = sys.argv[1:] if argv is None else list(argv)
     args = ap.parse_args(argv)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return _self_launch(args, argv)
     if args.warmup < 3 and args.impl == "ours" and not os.environ.get("BENCH_ALLOW_FEW_WARMUP"):
         args.warmup = 3
     if args.config.startswith("m"):

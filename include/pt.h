@@ -83,13 +83,13 @@ typedef enum { PT_END_MASK = 0, PT_END_CURV = 1, PT_END_MAXLEN = 2 } pt_reason;
                                         between segments, schedule of pt_set_segments.
                                         Same results; synchronous; not combinable with
                                         PT_REC_PATHS, PT_REC_CONN or the NEXT-3 variants */
-#define PT_KERNEL_SPEC    (1u << 17) /* ablation: the speculative kernel (a second record
-                                        gather per lane and iteration at the extrapolated
-                                        next voxel, two steps per iteration on a hit;
-                                        DESIGN.md §13) instead of the default 6-step-round
-                                        kernel; same results.  PT_ERR_ARG with
-                                        PT_KERNEL_SIMPLE, PT_KERNEL_SEGMENTED or a NEXT-3
-                                        variant flag                                     */
+#define PT_MAP_UNIQUE     (1u << 18) /* NEXT-2: the map counts streamlines, not steps: map[v]
+                                        += 1 for every streamline (both halves of a
+                                        bidirectional one together) with at least one
+                                        committed step landing in voxel v ("counting
+                                        the number of streamlines passing through B"; R25).
+                                        Exact (a per-lane hash set of entered voxels).
+                                        PT_ERR_ARG with PT_KERNEL_SIMPLE / SEGMENTED       */
 
 /* Create a context on CUDA device `cuda_device` (the caller's current device is left
  * unchanged).  *out receives the context or NULL.  The stream defaults to the legacy
@@ -140,7 +140,8 @@ typedef struct {
     int32_t max_steps;          /* 1..65535 (maximum number of steps; R14)        */
     uint64_t rng_seed;          /* Philox-4x32-10 key (R16)                               */
     int64_t particles_per_seed; /* P >= 1; particle j of seed id k has pid = k*P + j      */
-    uint32_t flags;             /* PT_REC_* | PT_MAP_ACCUMULATE | PT_KERNEL_SIMPLE |
+    uint32_t flags;             /* PT_REC_* | PT_MAP_ACCUMULATE | PT_MAP_UNIQUE |
+                                   PT_KERNEL_SIMPLE | PT_KERNEL_SEGMENTED |
                                    PT_SEED_ORDER_INPUT | PT_SAMPLE_PER_STREAMLINE |
                                    PT_BIDIR | PT_INTERP | PT_INIT_* | PT_KERNEL_VARIANT   */
     int32_t path_stride;        /* points stored per particle with PT_REC_PATHS (>= 1)    */
@@ -196,7 +197,9 @@ pt_status pt_get_connectivity(pt_ctx* ctx, uint32_t* out, int64_t capacity, int6
  * corner coordinates; paths [count][path_stride][3] float32 (point 0 = start, point k =
  * after the k-th committed step, unused points NaN).  Requesting an output that the
  * last pt_track did not record is PT_ERR_STATE; capacity < count is PT_ERR_ARG.
- * Synchronises ctx's stream; returns PT_ERR_OVERFLOW if the map wrapped. */
+ * Synchronises ctx's stream; returns PT_ERR_OVERFLOW if the map wrapped.  Paper: the
+ * fibre paths of Fig. 1 and the end points of Alg. 1 (SetEndPoint() /
+ * ReadEndPointFromGPU()). */
 typedef struct {
     uint16_t* nsteps;
     uint8_t* reason;
@@ -217,7 +220,10 @@ pt_status pt_get_paths(pt_ctx* ctx, pt_paths* out);
  *   overflow         : 1 if a map cell wrapped (detected as map_sum != expected)
  *   kernel_ms        : device time of the tracking kernel (CUDA events on ctx's stream)
  *   track_ms         : device time of the whole pt_track enqueue (zeroing, kernel, checks)
- *   spec_hits        : steps taken with the speculative record (PT_KERNEL_SPEC; else 0) */
+ *   unique_visits    : with PT_MAP_UNIQUE, the counts added to the map (sum over
+ *                      streamlines of the voxels they entered); else 0
+ * Errors: PT_ERR_OVERFLOW (see overflow); PT_ERR_ARG if a device-resident seed id made
+ * seed_id*P + j overflow 64 bits (those particles ran with seed id 0). */
 typedef struct {
     uint64_t total_steps;
     uint64_t particles;
@@ -227,9 +233,32 @@ typedef struct {
     int32_t overflow;
     float kernel_ms;
     float track_ms;
-    uint64_t spec_hits;
+    uint64_t unique_visits;
 } pt_stats;
 pt_status pt_get_stats(pt_ctx* ctx, pt_stats* out);
+
+/* Timing of the last pt_load_samples (the paper's Copy3DImagesToGPU(), timed as
+ * "Transfer" in Table II): device time of the host-to-device copies of the host inputs
+ * (0 if every input was a device pointer) and of the repack kernel, bytes copied from the
+ * host, bytes of the repacked record volume.  Errors: PT_ERR_STATE before a load. */
+typedef struct {
+    float h2d_ms;
+    float repack_ms;
+    uint64_t h2d_bytes;
+    uint64_t record_bytes;
+} pt_load_stats;
+pt_status pt_get_load_stats(pt_ctx* ctx, pt_load_stats* out);
+
+/* Device self-test of the tracking RNG (R16): for i < n,
+ * words[4i..4i+3] = Philox4x32-10(ctr = {block[i], lo32(pid[i]), hi32(pid[i]), stream[i]},
+ * key = {lo32(rng_seed), hi32(rng_seed)}) and samples[3i+k] = floor(words[4i+k] * nsamples
+ * / 2^32), k < 3, computed by the SAME device functions the tracking kernel uses; the
+ * kernel also recomputes each block with the CUDA library's curand_Philox4x32_10 and
+ * *mismatches receives the number of blocks that differ (0 expected).  All arrays host or
+ * device; nsamples >= 1.  Synchronous.  Errors: PT_ERR_ARG for NULL arrays / n < 0. */
+pt_status pt_rng_draws(pt_ctx* ctx, const uint64_t* pid, const uint32_t* block, const uint32_t* stream,
+                       int64_t n, uint64_t rng_seed, uint32_t nsamples, uint32_t* words, uint32_t* samples,
+                       int64_t* mismatches);
 
 /* Roofline micro-benchmark: uniformly random, record-aligned
  * reads of `record_bytes` (8, 16, 32 or 64) from a device buffer of `buffer_bytes`,

@@ -87,7 +87,7 @@ def lib():
             L.oracle_sample_index.restype = ctypes.c_uint32
             L.oracle_track.argtypes = [ctypes.POINTER(_Volume), ctypes.POINTER(_Params), vp, vp,
                                        ctypes.c_int64, ctypes.c_int64, ctypes.c_int64,
-                                       vp, vp, vp, vp, vp, ctypes.c_int32, vp, ctypes.c_int32, vp]
+                                       vp, vp, vp, vp, vp, ctypes.c_int32, vp, ctypes.c_int32, vp, vp]
             L.oracle_track.restype = ctypes.c_int
             L.oracle_mcmc_signal.argtypes = [ctypes.c_int, vp, ctypes.c_int, vp, vp, vp]
             L.oracle_mcmc_signal.restype = None
@@ -144,12 +144,13 @@ def _structs(volume, step, curv_thr, fib_thr, max_steps, rng_seed, P, sample_mod
 
 def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = True,
           want_particles: bool = True, path_stride: int = 0, threads: int = 1,
-          labels: Optional[np.ndarray] = None, ntargets: int = 0) -> dict:
+          labels: Optional[np.ndarray] = None, ntargets: int = 0, want_unique: bool = False) -> dict:
     """Run the oracle on workload ``w`` (a phantom.Workload or duck-typed equivalent).
 
     Returns dict(map=uint64[Z][Y][X] or None, nsteps=int32[n], reason=uint8[n],
     end=float32[n][3], paths=float32[n][path_stride][3] or None, conn=uint64[nseeds][ntargets]
-    or None), particles ordered (seed index, j) -- with ``w.bidir`` two entries per particle
+    or None, umap=uint64[Z][Y][X] streamlines per voxel (R25) with ``want_unique`` else None),
+    particles ordered (seed index, j) -- with ``w.bidir`` two entries per particle
     (seed index, j, half), n = 2 * nseeds * npp.  ``threads`` > 1 runs independent single-threaded oracle calls on
     disjoint seed shards (seed i -> worker i mod threads) and sums their maps.
     """
@@ -176,7 +177,7 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
     lab = None if labels is None else np.ascontiguousarray(labels, np.uint8)
     T = int(ntargets) if lab is not None else 0
 
-    def run(shard: np.ndarray, mp: Optional[np.ndarray]):
+    def run(shard: np.ndarray, mp: Optional[np.ndarray], um: Optional[np.ndarray]):
         sd = np.ascontiguousarray(seeds[shard])
         si = np.ascontiguousarray(ids[shard])
         m = len(shard) * npp * H
@@ -187,19 +188,20 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
         lc = np.zeros((len(shard), T), np.uint64) if T else None
         rc = L.oracle_track(ctypes.byref(vs), ctypes.byref(ps), sd.ctypes.data, si.ctypes.data,
                             len(shard), j_begin, j_end, _ptr(mp), _ptr(ln), _ptr(lr), _ptr(le),
-                            _ptr(lp), path_stride, _ptr(lab), T, _ptr(lc))
+                            _ptr(lp), path_stride, _ptr(lab), T, _ptr(lc), _ptr(um))
         if rc != 0:
             raise ValueError(f"oracle_track rejected its arguments (rc={rc})")
         return ln, lr, le, lp, lc
 
     maps = [np.zeros((v.nz, v.ny, v.nx), np.uint64) if want_map else None for _ in range(threads)]
+    umaps = [np.zeros((v.nz, v.ny, v.nx), np.uint64) if want_unique else None for _ in range(threads)]
     shards = [np.arange(t, ns, threads) for t in range(threads)]
     results = [None] * threads
     if threads == 1:
-        results[0] = run(shards[0], maps[0])
+        results[0] = run(shards[0], maps[0], umaps[0])
     else:
         def worker(t):
-            results[t] = run(shards[t], maps[t])
+            results[t] = run(shards[t], maps[t], umaps[t])
         th = [threading.Thread(target=worker, args=(t,)) for t in range(threads)]
         for t in th:
             t.start()
@@ -226,7 +228,12 @@ def track(w, j_begin: int = 0, j_end: Optional[int] = None, *, want_map: bool = 
         mp = maps[0]
         for m in maps[1:]:
             mp += m
-    return dict(map=mp, nsteps=nsteps, reason=reason, end=end, paths=paths, conn=conn)
+    um = None
+    if want_unique:
+        um = umaps[0]
+        for m in umaps[1:]:
+            um += m
+    return dict(map=mp, nsteps=nsteps, reason=reason, end=end, paths=paths, conn=conn, umap=um)
 
 
 # ----------------------------------------------------------------------------- NEXT-4 MCMC

@@ -15,6 +15,7 @@
 #include <float.h>
 #include <math.h>
 #include <stddef.h>
+#include <stdlib.h>
 #include <string.h>
 
 #if !defined(FLT_EVAL_METHOD) || FLT_EVAL_METHOD != 0
@@ -193,6 +194,8 @@ typedef struct {
     int32_t ntargets;
     float* path;             /* [path_stride][3] or NULL                                 */
     int32_t path_stride;
+    int64_t* entered_vox;    /* R25: voxel of every committed step of the streamline, or NULL */
+    int64_t nentered;
 } half_io;
 
 /* One (half-)streamline: Algorithm 1's inner loop.  Returns n; *why and the
@@ -312,6 +315,7 @@ static int32_t track_half(const oracle_volume* vol, const oracle_params* prm, ha
             if (io->map) io->map[vox] += 1u;
             if (io->entered && io->labels[vox] != 0 && io->labels[vox] <= io->ntargets)
                 io->entered[io->labels[vox] - 1] = 1;     /* R21: committed steps only */
+            if (io->entered_vox) io->entered_vox[io->nentered++] = vox;  /* R25 */
             if (io->path && n < io->path_stride)
                 for (a = 0; a < 3; ++a) io->path[n * 3 + a] = q[a] + c[a];
         }
@@ -321,12 +325,17 @@ static int32_t track_half(const oracle_volume* vol, const oracle_params* prm, ha
     return n;
 }
 
+static int cmp_i64(const void* a, const void* b) {
+    const int64_t x = *(const int64_t*)a, y = *(const int64_t*)b;
+    return (x > y) - (x < y);
+}
+
 int oracle_track(const oracle_volume* vol, const oracle_params* prm,
                  const float* seeds_xyz, const uint64_t* seed_ids, int64_t nseeds,
                  int64_t j_begin, int64_t j_end,
                  uint64_t* map, int32_t* nsteps, uint8_t* reason, float* end_xyz,
                  float* paths, int32_t path_stride,
-                 const uint8_t* labels, int32_t ntargets, uint64_t* conn) {
+                 const uint8_t* labels, int32_t ntargets, uint64_t* conn, uint64_t* umap) {
     const uint64_t P = (uint64_t)prm->particles_per_seed;
     const float c[3] = {(float)(vol->nx / 2), (float)(vol->ny / 2), (float)(vol->nz / 2)};
     const int64_t npp = j_end - j_begin;
@@ -337,10 +346,18 @@ int oracle_track(const oracle_volume* vol, const oracle_params* prm,
     if (nseeds < 0 || j_begin < 0 || j_end < j_begin || (uint64_t)j_end > P) return -2;
     if (paths && path_stride < 1) return -3;
     if (conn && (!labels || ntargets < 1 || ntargets > 64)) return -5;
+    int64_t* entered_vox = NULL;  /* R25: committed-step voxels of one streamline */
+    if (umap) {
+        entered_vox = (int64_t*)malloc(sizeof(int64_t) * (size_t)halves * (size_t)prm->max_steps + 8);
+        if (!entered_vox) return -6;
+    }
 
     for (si = 0; si < nseeds; ++si) {
         const uint64_t sid = seed_ids ? seed_ids[si] : (uint64_t)si;
-        if (sid > (UINT64_MAX - (P - 1)) / P) return -4;       /* pid overflow */
+        if (sid > (UINT64_MAX - (P - 1)) / P) {                  /* pid overflow */
+            free(entered_vox);
+            return -4;
+        }
         for (jj = j_begin; jj < j_end; ++jj) {
             const int64_t out = si * npp + (jj - j_begin);
             unsigned char entered[64];   /* NEXT-2: targets this streamline passed through */
@@ -357,6 +374,8 @@ int oracle_track(const oracle_volume* vol, const oracle_params* prm,
             io.labels = labels;
             io.ntargets = ntargets;
             io.path_stride = path_stride;
+            io.entered_vox = entered_vox;
+            io.nentered = 0;
             for (h = 0; h < halves; ++h) {
                 const int64_t o = out * halves + h;              /* output slot */
                 float qe[3];
@@ -376,7 +395,16 @@ int oracle_track(const oracle_volume* vol, const oracle_params* prm,
                 for (t = 0; t < ntargets; ++t)
                     if (entered[t]) conn[si * ntargets + t] += 1u;
             }
+            /* R25: each voxel the streamline passed through counts once (sort, then count
+             * the distinct values) */
+            if (umap) {
+                int64_t k;
+                qsort(entered_vox, (size_t)io.nentered, sizeof(int64_t), cmp_i64);
+                for (k = 0; k < io.nentered; ++k)
+                    if (k == 0 || entered_vox[k] != entered_vox[k - 1]) umap[entered_vox[k]] += 1u;
+            }
         }
     }
+    free(entered_vox);
     return 0;
 }

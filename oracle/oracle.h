@@ -82,13 +82,17 @@ uint32_t oracle_sample_index(uint32_t w, uint32_t nsamples);
  *   conn      [nseeds][ntargets] uint64, accumulated: number of the seed's particles whose
  *             committed steps enter target t at least once (NEXT-2; R21); may be NULL
  *             (with bidir a streamline is the union of its two halves)
+ *   umap      [Z][Y][X] uint64, accumulated: number of streamlines with at least one
+ *             committed step landing in the voxel -- "counting the number of streamlines
+ *             passing through B" (R25); may be NULL (with bidir a streamline is
+ *             the union of its two halves)
  * Returns 0 on success, <0 on invalid arguments (nothing written). */
 int oracle_track(const oracle_volume* vol, const oracle_params* prm,
                  const float* seeds_xyz, const uint64_t* seed_ids, int64_t nseeds,
                  int64_t j_begin, int64_t j_end,
                  uint64_t* map, int32_t* nsteps, uint8_t* reason, float* end_xyz,
                  float* paths, int32_t path_stride,
-                 const uint8_t* labels, int32_t ntargets, uint64_t* conn);
+                 const uint8_t* labels, int32_t ntargets, uint64_t* conn, uint64_t* umap);
 
 
 /* ---------------------------------------------------------------- NEXT-4: MCMC sampler

@@ -27,9 +27,9 @@ __all__ = [
     "PT_REC_PATHS", "PT_MAP_ACCUMULATE", "PT_KERNEL_SIMPLE", "PT_SEED_ORDER_INPUT",
     "PT_SAMPLE_PER_STREAMLINE", "PT_REC_CONN", "PT_BIDIR", "PT_INTERP", "PT_INIT_RANDOM",
     "PT_INIT_FWEIGHT", "PT_KERNEL_VARIANT", "variant_flags", "pt_mcmc", "pt_get_mcmc_stats",
-    "pt_mcmc_to_volume", "pt_dwi_shape", "pt_mcmc_params", "PT_KERNEL_SEGMENTED", "pt_set_segments", "PT_KERNEL_SPEC",
-    "SEGMENTS_B", "SEGMENTS_C", "pt_load_targets", "pt_get_connectivity", "PT_END_MASK", "PT_END_CURV",
-    "PT_END_MAXLEN", "EXPORTS",
+    "pt_mcmc_to_volume", "pt_dwi_shape", "pt_mcmc_params", "PT_KERNEL_SEGMENTED", "pt_set_segments",
+    "PT_MAP_UNIQUE", "SEGMENTS_B", "SEGMENTS_C", "pt_load_targets", "pt_get_connectivity", "PT_END_MASK",
+    "PT_END_CURV", "PT_END_MAXLEN", "pt_get_load_stats", "pt_rng_draws", "EXPORTS",
 ]
 
 PT_OK, PT_ERR_ARG, PT_ERR_STATE, PT_ERR_OOM, PT_ERR_CUDA, PT_ERR_OVERFLOW = range(6)
@@ -50,7 +50,7 @@ PT_INIT_RANDOM = 1 << 13
 PT_INIT_FWEIGHT = 1 << 14
 PT_KERNEL_VARIANT = 1 << 15
 PT_KERNEL_SEGMENTED = 1 << 16
-PT_KERNEL_SPEC = 1 << 17  # ablation: speculative 2nd-gather kernel (pt_spec.cu)
+PT_MAP_UNIQUE = 1 << 18  # NEXT-2: per-streamline-unique visitation map (R25)
 # the paper's increasing-interval segmentation strategies
 SEGMENTS_B = (1, 2, 5, 10, 20, 50, 100, 200, 500)
 SEGMENTS_C = (1, 1, 2, 2, 5, 5, 10, 10, 20, 20, 50, 50, 100, 100, 200, 200)
@@ -65,7 +65,7 @@ def variant_flags(bidir: int = 0, interp: int = 0, init_fibre: int = 0) -> int:
 EXPORTS = ["pt_create", "pt_destroy", "pt_last_error", "pt_set_stream", "pt_load_samples",
            "pt_track", "pt_get_paths", "pt_get_stats", "pt_gather_bench", "pt_record_bytes",
            "pt_load_targets", "pt_get_connectivity", "pt_mcmc", "pt_get_mcmc_stats",
-           "pt_mcmc_to_volume", "pt_set_segments"]
+           "pt_mcmc_to_volume", "pt_set_segments", "pt_get_load_stats", "pt_rng_draws"]
 
 _STATUS = {1: "PT_ERR_ARG", 2: "PT_ERR_STATE", 3: "PT_ERR_OOM", 4: "PT_ERR_CUDA", 5: "PT_ERR_OVERFLOW"}
 
@@ -99,7 +99,12 @@ class pt_stats(ctypes.Structure):
                 ("lane_active", ctypes.c_uint64), ("lane_slots", ctypes.c_uint64),
                 ("map_sum", ctypes.c_uint64), ("overflow", ctypes.c_int32),
                 ("kernel_ms", ctypes.c_float), ("track_ms", ctypes.c_float),
-                ("spec_hits", ctypes.c_uint64)]
+                ("unique_visits", ctypes.c_uint64)]
+
+
+class pt_load_stats(ctypes.Structure):
+    _fields_ = [("h2d_ms", ctypes.c_float), ("repack_ms", ctypes.c_float), ("h2d_bytes", ctypes.c_uint64),
+                ("record_bytes", ctypes.c_uint64)]
 
 
 class pt_dwi_shape(ctypes.Structure):
@@ -161,6 +166,11 @@ def lib() -> ctypes.CDLL:
     L.pt_mcmc_to_volume.restype = ctypes.c_int
     L.pt_set_segments.argtypes = [vp, vp, ctypes.c_int32]
     L.pt_set_segments.restype = ctypes.c_int
+    L.pt_get_load_stats.argtypes = [vp, P(pt_load_stats)]
+    L.pt_get_load_stats.restype = ctypes.c_int
+    L.pt_rng_draws.argtypes = [vp, vp, vp, vp, ctypes.c_int64, ctypes.c_uint64, ctypes.c_uint32, vp, vp,
+                               P(ctypes.c_int64)]
+    L.pt_rng_draws.restype = ctypes.c_int
     L.pt_record_bytes.argtypes = [ctypes.c_int32, ctypes.c_int32]
     L.pt_record_bytes.restype = ctypes.c_int32
     _lib = L
@@ -250,6 +260,20 @@ def pt_set_segments(ctx, intervals) -> None:
     _check(ctx, lib().pt_set_segments(ctx, arr, len(intervals)))
 
 
+def pt_get_load_stats(ctx) -> pt_load_stats:
+    s = pt_load_stats()
+    _check(ctx, lib().pt_get_load_stats(ctx, ctypes.byref(s)))
+    return s
+
+
+def pt_rng_draws(ctx, pid_ptr, block_ptr, stream_ptr, n: int, rng_seed: int, nsamples: int, words_ptr,
+                 samples_ptr) -> int:
+    mm = ctypes.c_int64()
+    _check(ctx, lib().pt_rng_draws(ctx, pid_ptr, block_ptr, stream_ptr, n, rng_seed, nsamples, words_ptr,
+                                   samples_ptr, ctypes.byref(mm)))
+    return mm.value
+
+
 def pt_gather_bench(ctx, buffer_bytes: int, record_bytes: int) -> float:
     r = ctypes.c_double()
     _check(ctx, lib().pt_gather_bench(ctx, buffer_bytes, record_bytes, ctypes.byref(r)))
@@ -276,6 +300,22 @@ def _contig(a):
     if isinstance(a, np.ndarray):
         return np.ascontiguousarray(a)
     return a.contiguous()
+
+
+def _dt(a) -> str:
+    """dtype name of a numpy array or torch tensor ('float32', 'uint8', ...)."""
+    return str(a.dtype).replace("torch.", "")
+
+
+def _expect(name: str, a, dtypes, shape=None) -> None:
+    """Argument check before a pointer crosses the ABI: the C side reads raw bytes, so a
+    wrong dtype or shape would be silent garbage or an out-of-bounds read."""
+    if _dt(a) not in dtypes:
+        raise TypeError(f"{name}: dtype {_dt(a)}, expected one of {sorted(dtypes)}")
+    if shape is not None:
+        got = tuple(int(d) for d in a.shape)
+        if len(got) != len(shape) or any(e is not None and g != e for g, e in zip(got, shape)):
+            raise ValueError(f"{name}: shape {got}, expected {tuple('*' if e is None else e for e in shape)}")
 
 
 class Tracker:
@@ -305,8 +345,11 @@ class Tracker:
     def load_samples(self, dyads, f, mask, nsamples: int, nfibres: int) -> None:
         """dyads [F][S][Z][Y][X][3], f [F][S][Z][Y][X] (float32 or float16), mask [Z][Y][X]
         uint8; numpy (host) or torch (host or cuda) arrays."""
-        half = str(dyads.dtype).endswith("float16")
-        nz, ny, nx = mask.shape
+        half = _dt(dyads) == "float16"
+        _expect("mask", mask, {"uint8", "bool"}, (None, None, None))
+        nz, ny, nx = (int(d) for d in mask.shape)
+        _expect("dyads", dyads, {"float32", "float16"}, (nfibres, nsamples, nz, ny, nx, 3))
+        _expect("f", f, {_dt(dyads)}, (nfibres, nsamples, nz, ny, nx))
         self._stream()
         pt_load_samples(self.ctx, nx, ny, nz, nsamples, nfibres, PT_F16 if half else PT_F32,
                         _ptr(dyads), _ptr(f), _ptr(mask))
@@ -328,8 +371,13 @@ class Tracker:
         prm = pt_params(step, curv_thr, fib_thr, max_steps, rng_seed, particles_per_seed, flags,
                         path_stride)
         seeds, seed_ids = _contig(seeds), _contig(seed_ids)
-        self._stream()
+        _expect("seeds", seeds, {"float32"}, (None, 3))
         n = int(seeds.shape[0])
+        if seed_ids is not None:
+            _expect("seed_ids", seed_ids, {"uint64", "int64"}, (n,))
+        if want_map and out_map is not None:
+            _expect("out_map", out_map, {"int32", "uint32"}, self.shape)
+        self._stream()
         pt_track(self.ctx, _ptr(seeds), _ptr(seed_ids), n, prm, _ptr(out_map) if want_map else None)
         return out_map if want_map else None
 
@@ -379,6 +427,8 @@ class Tracker:
     def load_targets(self, labels, ntargets: int) -> None:
         """Target regions for the seed x target matrix (uint8 [Z][Y][X], 0 = none, t+1)."""
         labels = _contig(labels)
+        if labels is not None:
+            _expect("labels", labels, {"uint8"}, self.shape)
         self._stream()
         pt_load_targets(self.ctx, _ptr(labels), ntargets)
 
@@ -392,6 +442,27 @@ class Tracker:
     def set_segments(self, intervals) -> None:
         """Schedule of the PT_KERNEL_SEGMENTED ablation (the paper's NumIteration[])."""
         pt_set_segments(self.ctx, intervals)
+
+    def load_stats(self) -> dict:
+        """Timing of the last load_samples: H2D copy and repack (device ms), bytes."""
+        s = pt_get_load_stats(self.ctx)
+        return {k: getattr(s, k) for k, _ in pt_load_stats._fields_}
+
+    def rng_draws(self, pid, block, stream, rng_seed: int, nsamples: int):
+        """Device self-test of the tracking RNG (pt_rng_draws): returns (words uint32 [n][4],
+        sample indices uint32 [n][3], blocks that differ from curand_Philox4x32_10)."""
+        pid = np.ascontiguousarray(pid, np.uint64)
+        block = np.ascontiguousarray(block, np.uint32)
+        stream = np.ascontiguousarray(stream, np.uint32)
+        n = pid.size
+        if block.size != n or stream.size != n:
+            raise ValueError("pid, block and stream must have the same length")
+        words = np.zeros((n, 4), np.uint32)
+        samples = np.zeros((n, 3), np.uint32)
+        self._stream()
+        mm = pt_rng_draws(self.ctx, pid.ctypes.data, block.ctypes.data, stream.ctypes.data, n, rng_seed,
+                          nsamples, words.ctypes.data, samples.ctypes.data)
+        return words, samples, mm
 
     def gather_bench(self, buffer_bytes: int, record_bytes: int) -> float:
         self._stream()
@@ -416,7 +487,16 @@ class Tracker:
             samples = torch.empty((NP, int(d.nsamples), nz, ny, nx), dtype=torch.float64, device=self.device)
         acc = torch.empty((NP, nz, ny, nx), dtype=torch.int32, device=self.device) if accepted else None
         dwi, bv, bc, mask = (_contig(x) for x in (d.dwi, d.bvals, d.bvecs, d.mask))
+        nm = int(shape.nmeas)
+        _expect("dwi", dwi, {"float32"}, (nm, nz, ny, nx))
+        _expect("bvals", bv, {"float32"}, (nm,))
+        _expect("bvecs", bc, {"float32"}, (nm, 3))
+        _expect("mask", mask, {"uint8", "bool"}, (nz, ny, nx))
+        if samples is not None:
+            _expect("samples", samples, {"float64"}, (NP, int(d.nsamples), nz, ny, nx))
         ini = _contig(init)
+        if ini is not None:
+            _expect("init", ini, {"float64"}, (NP, nz, ny, nx))
         self._stream()
         pt_mcmc(self.ctx, shape, _ptr(dwi), _ptr(bv), _ptr(bc), _ptr(mask), prm, _ptr(ini),
                 _ptr(samples), _ptr(acc))

@@ -1,23 +1,30 @@
-"""Build libpt.so in-tree with nvcc for sm_100a (no JIT cache, no torch extension)."""
+"""Build libpt.so in-tree with nvcc for sm_100a (no JIT cache, no torch extension).
+
+Each translation unit is compiled to an object in parallel (the tracking kernel's
+instantiations are split by fibre count into pt_track_f{1,2,3}.cu), then linked."""
 from __future__ import annotations
 
 import os
 import shutil
 import subprocess
+from concurrent.futures import ThreadPoolExecutor
 
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.environ.get("PT_LIB") or os.path.join(PKG, "libpt.so")  # PT_LIB: experiment builds
-SOURCES = ["pt_api.cu", "pt_kernels.cu", "pt_variants.cu", "pt_mcmc.cu", "pt_segmented.cu", "pt_spec.cu"]
-HEADERS = ["pt_device.cuh", "pt_internal.h", "pt_claim.cuh"]
+OBJDIR = os.path.join(PKG, "build")
+SOURCES = ["pt_api.cu", "pt_kernels.cu", "pt_track_f1.cu", "pt_track_f2.cu", "pt_track_f3.cu",
+           "pt_mcmc.cu", "pt_segmented.cu"]
+HEADERS = ["pt_device.cuh", "pt_internal.h", "pt_claim.cuh", "pt_track.cuh"]
 
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC_FLAGS = [
-    "-gencode", "arch=compute_100a,code=sm_100a",
+    *ARCH,
     "-O3", "-lineinfo", "-std=c++17",
     "-fmad=false",          # no FMA contraction anywhere in the library (R15)
-    "-Xcompiler", "-fPIC", "-shared",
+    "-Xcompiler", "-fPIC",
     "-Xptxas", "-warn-spills", "-diag-suppress", "186",
 ]
 
@@ -46,13 +53,29 @@ def stale() -> bool:
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
-    tmp = LIB + f".tmp{os.getpid()}"
     extra = os.environ.get("PT_NVCC_EXTRA", "").split()  # experiment builds: -D overrides
-    cmd = [nvcc(), *NVCC_FLAGS, *extra, "-I", INCLUDE, "-o", tmp, *[os.path.join(CSRC, s) for s in SOURCES]]
+    tag = f"{os.getpid()}"
+    os.makedirs(OBJDIR, exist_ok=True)
+    objs = [os.path.join(OBJDIR, os.path.splitext(s)[0] + f".{tag}.o") for s in SOURCES]
+    cmds = [[nvcc(), *NVCC_FLAGS, *extra, "-I", INCLUDE, "-c", "-o", o, os.path.join(CSRC, s)]
+            for s, o in zip(SOURCES, objs)]
     if verbose:
-        print(" ".join(cmd))
-    subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
+        for c in cmds:
+            print(" ".join(c))
+    try:
+        with ThreadPoolExecutor(max_workers=len(cmds)) as ex:
+            for f in [ex.submit(subprocess.check_call, c) for c in cmds]:
+                f.result()
+        tmp = LIB + f".tmp{tag}"
+        link = [nvcc(), *ARCH, "-shared", "-o", tmp, *objs]
+        if verbose:
+            print(" ".join(link))
+        subprocess.check_call(link)
+        os.replace(tmp, LIB)
+    finally:
+        for o in objs:
+            if os.path.exists(o):
+                os.remove(o)
     return LIB
 
 

@@ -16,9 +16,6 @@
 
 #include "pt_internal.h"
 
-#ifndef PT_MAP_COPIES
-#define PT_MAP_COPIES 1  // private map copies (privatisation; 1 = add into the map directly)
-#endif
 #ifndef PT_SEEDS_PER_CLAIM
 // Whole seeds per CTA claim when every seed fits one claim: a CTA walks 32 consecutive
 // (Morton-adjacent) seeds, so its L1 keeps serving the shared tract voxels (sweep 1..64:
@@ -57,8 +54,12 @@ struct pt_ctx {
     size_t temp_cap = 0;
     uint32_t* d_map = nullptr;   // internal map for host map pointers
     size_t map_cap = 0;
-    uint32_t* d_copies = nullptr;  // private map copies (PT_MAP_COPIES > 1)
-    size_t copies_cap = 0;
+    unsigned long long* d_utab = nullptr;  // NEXT-2 unique map: per-lane hash sets
+    size_t utab_cap = 0;
+    uint8_t* d_stage = nullptr;    // pt_load_samples: staging of host inputs (grow-only)
+    size_t stage_cap = 0;
+    cudaEvent_t lev[3] = {nullptr, nullptr, nullptr};  // load: start, after H2D, after repack
+    uint64_t load_h2d_bytes = 0;
     uint16_t* d_nsteps = nullptr;
     size_t nsteps_cap = 0;
     uint8_t* d_reason = nullptr;
@@ -173,6 +174,46 @@ int rec_bytes_of(int F, int dtype) {
     return raw <= 8 ? 8 : raw <= 16 ? 16 : raw <= 32 ? 32 : 64;
 }
 
+// Device view of a caller buffer: device pointers are used in place; host inputs are
+// copied into a temporary device buffer; host outputs get a temporary device buffer that
+// is copied back by finish().
+struct Staged {
+    void* dev = nullptr;
+    void* tmp = nullptr;
+    void* host_out = nullptr;
+    size_t bytes = 0;
+    ~Staged() {
+        if (tmp) cudaFree(tmp);
+    }
+    cudaError_t in(const void* p, size_t n, cudaStream_t st) {
+        bytes = n;
+        if (!p || is_device_ptr(p)) {
+            dev = const_cast<void*>(p);
+            return cudaSuccess;
+        }
+        cudaError_t e = cudaMalloc(&tmp, n ? n : 1);
+        if (e != cudaSuccess) return e;
+        dev = tmp;
+        return cudaMemcpyAsync(tmp, p, n, cudaMemcpyHostToDevice, st);
+    }
+    cudaError_t out(void* p, size_t n) {
+        bytes = n;
+        if (!p || is_device_ptr(p)) {
+            dev = p;
+            return cudaSuccess;
+        }
+        cudaError_t e = cudaMalloc(&tmp, n ? n : 1);
+        if (e != cudaSuccess) return e;
+        dev = tmp;
+        host_out = p;
+        return cudaSuccess;
+    }
+    cudaError_t finish(cudaStream_t st) {
+        if (!host_out) return cudaSuccess;
+        return cudaMemcpyAsync(host_out, dev, bytes, cudaMemcpyDeviceToHost, st);
+    }
+};
+
 }  // namespace
 
 extern "C" {
@@ -213,6 +254,13 @@ pt_status pt_create(int cuda_device, pt_ctx** out) {
             return fail(nullptr, PT_ERR_CUDA, "pt_create: cudaEventCreate failed");
         }
     }
+    for (auto& ev : c->lev) {
+        if (cudaEventCreate(&ev) != cudaSuccess) {
+            cudaGetLastError();
+            pt_destroy(c);
+            return fail(nullptr, PT_ERR_CUDA, "pt_create: cudaEventCreate failed");
+        }
+    }
     for (auto& ev : c->ev) {
         if (cudaEventCreate(&ev) != cudaSuccess) {
             cudaGetLastError();
@@ -235,14 +283,16 @@ void pt_destroy(pt_ctx* c) {
     DeviceGuard g(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
     else cudaDeviceSynchronize();
-    void* bufs[] = {c->d_rec, c->d_mask, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_copies, c->d_labels, c->d_conn, c->d_nsteps,
-                    c->d_reason, c->d_end, c->d_paths, c->d_stats, c->d_mstats, c->d_mvox, c->d_mflags,
-                    c->d_mtemp, c->d_mcount, c->d_seg};
+    void* bufs[] = {c->d_rec, c->d_mask, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_utab,
+                    c->d_stage, c->d_labels, c->d_conn, c->d_nsteps, c->d_reason, c->d_end, c->d_paths,
+                    c->d_stats, c->d_mstats, c->d_mvox, c->d_mflags, c->d_mtemp, c->d_mcount, c->d_seg};
     for (void* b : bufs)
         if (b) cudaFree(b);
     for (auto& ev : c->ev)
         if (ev) cudaEventDestroy(ev);
     for (auto& ev : c->mev)
+        if (ev) cudaEventDestroy(ev);
+    for (auto& ev : c->lev)
         if (ev) cudaEventDestroy(ev);
     cudaGetLastError();
     delete c;
@@ -286,33 +336,43 @@ pt_status pt_load_samples(pt_ctx* c, const pt_volume* v, const void* dyads, cons
     if (L.nvox() > 0xFFFFFFFFull) return fail(c, PT_ERR_ARG, "pt_load_samples: padded volume exceeds 2^32-1 voxels");
     const size_t rec_size = L.nvox() * S * (size_t)rb;
 
-    // stage host inputs on the device (device inputs are read in place)
-    const void* d_dy = dyads;
-    const void* d_f = f;
-    const uint8_t* d_m = mask;
-    void* tmp[3] = {nullptr, nullptr, nullptr};
-    auto cleanup = [&]() {
-        for (void* t : tmp)
-            if (t) cudaFree(t);
-    };
+    // stage host inputs on the device through one context-owned buffer (grow-only; device
+    // inputs are read in place): one cudaMemcpyAsync per host array, at full speed when the
+    // caller's memory is pinned
     const void* src[3] = {dyads, f, mask};
     const size_t sz[3] = {dy_bytes, f_bytes, m_bytes};
-    const void** dst[3] = {&d_dy, &d_f, reinterpret_cast<const void**>(&d_m)};
+    size_t off[3], need = 0;
+    bool host[3];
     for (int i = 0; i < 3; ++i) {
-        if (!is_device_ptr(src[i])) {
-            cudaError_t e = cudaMalloc(&tmp[i], sz[i]);
-            if (e != cudaSuccess) {
-                cleanup();
-                return cuda_fail(c, e, "pt_load_samples: staging allocation");
-            }
-            e = cudaMemcpyAsync(tmp[i], src[i], sz[i], cudaMemcpyHostToDevice, c->stream);
-            if (e != cudaSuccess) {
-                cleanup();
-                return cuda_fail(c, e, "pt_load_samples: host-to-device copy");
-            }
-            *dst[i] = tmp[i];
+        host[i] = !is_device_ptr(src[i]);
+        off[i] = need;
+        if (host[i]) need += (sz[i] + 255) / 256 * 256;
+    }
+    if (need > c->stage_cap) {
+        cudaStreamSynchronize(c->stream);
+        if (c->d_stage) cudaFree(c->d_stage);
+        c->d_stage = nullptr;
+        c->stage_cap = 0;
+        cudaError_t e = cudaMalloc(&c->d_stage, need);
+        if (e != cudaSuccess) return cuda_fail(c, e, "pt_load_samples: staging allocation");
+        c->stage_cap = need;
+    }
+    CK(cudaEventRecord(c->lev[0], c->stream), "pt_load_samples: event");
+    const void* dsrc[3];
+    c->load_h2d_bytes = 0;
+    for (int i = 0; i < 3; ++i) {
+        dsrc[i] = src[i];
+        if (host[i]) {
+            CK(cudaMemcpyAsync(c->d_stage + off[i], src[i], sz[i], cudaMemcpyHostToDevice, c->stream),
+               "pt_load_samples: host-to-device copy");
+            dsrc[i] = c->d_stage + off[i];
+            c->load_h2d_bytes += sz[i];
         }
     }
+    CK(cudaEventRecord(c->lev[1], c->stream), "pt_load_samples: event");
+    const void* d_dy = dsrc[0];
+    const void* d_f = dsrc[1];
+    const uint8_t* d_m = static_cast<const uint8_t*>(dsrc[2]);
     if (c->d_rec && c->rec_size != rec_size) {
         cudaStreamSynchronize(c->stream);
         cudaFree(c->d_rec);
@@ -322,7 +382,6 @@ pt_status pt_load_samples(pt_ctx* c, const pt_volume* v, const void* dyads, cons
     if (!c->d_rec) {
         cudaError_t e = cudaMalloc(&c->d_rec, rec_size);
         if (e != cudaSuccess) {
-            cleanup();
             c->loaded = false;
             return cuda_fail(c, e, "pt_load_samples: record volume allocation");
         }
@@ -335,11 +394,11 @@ pt_status pt_load_samples(pt_ctx* c, const pt_volume* v, const void* dyads, cons
     if (e == cudaSuccess)
         e = pt::launch_repack(d_dy, d_f, d_m, c->d_rec, v->nx, v->ny, v->nz, L, v->nsamples, v->nfibres,
                               v->dtype == PT_F16, rb, c->d_stats + pt::kStatBadInput, c->stream);
+    if (e == cudaSuccess) e = cudaEventRecord(c->lev[2], c->stream);
     unsigned long long bad = 0;
     if (e == cudaSuccess)
         e = cudaMemcpyAsync(&bad, c->d_stats + pt::kStatBadInput, sizeof bad, cudaMemcpyDeviceToHost, c->stream);
     if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
-    cleanup();
     if (e != cudaSuccess) return cuda_fail(c, e, "pt_load_samples: repack");
     if (bad) return fail(c, PT_ERR_ARG, "pt_load_samples: %llu records inside the mask hold non-finite values", bad);
     c->vol = *v;
@@ -370,26 +429,32 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     const uint64_t P = (uint64_t)p->particles_per_seed;
     if (P > 0xFFFFFFFFull) return fail(c, PT_ERR_ARG, "pt_track: particles_per_seed must be < 2^32");
     const uint64_t N = (uint64_t)nseeds;
+    if (N > 0xFFFFFFFFull) return fail(c, PT_ERR_ARG, "pt_track: more than 2^32-1 seeds");
     if (N && P > UINT64_MAX / N) return fail(c, PT_ERR_ARG, "pt_track: nseeds * P overflows");
     const uint64_t npart = N * P;
+    const uint32_t fl = p->flags;
     const uint32_t kVariantFlags = PT_BIDIR | PT_INTERP | PT_INIT_RANDOM | PT_INIT_FWEIGHT | PT_KERNEL_VARIANT;
-    const bool variant = (p->flags & kVariantFlags) != 0;
-    const bool segmented = (p->flags & PT_KERNEL_SEGMENTED) != 0;
-    if (segmented && (variant || (p->flags & (PT_KERNEL_SIMPLE | PT_REC_PATHS | PT_REC_CONN))))
+    const bool variant = (fl & kVariantFlags) != 0;
+    const bool segmented = (fl & PT_KERNEL_SEGMENTED) != 0;
+    const bool simple = (fl & PT_KERNEL_SIMPLE) != 0;
+    const bool unique = (fl & PT_MAP_UNIQUE) != 0;
+    if (segmented && (variant || unique || (fl & (PT_KERNEL_SIMPLE | PT_REC_PATHS | PT_REC_CONN))))
         return fail(c, PT_ERR_ARG, "pt_track: PT_KERNEL_SEGMENTED runs the base semantics with nsteps/reason/end outputs only");
-    if (variant && (p->flags & PT_KERNEL_SIMPLE))
-        return fail(c, PT_ERR_ARG, "pt_track: PT_KERNEL_SIMPLE cannot run the NEXT-3 variants");
-    if ((p->flags & PT_KERNEL_SPEC) && (variant || segmented || (p->flags & PT_KERNEL_SIMPLE)))
-        return fail(c, PT_ERR_ARG, "pt_track: PT_KERNEL_SPEC runs the base semantics only (no SIMPLE, SEGMENTED or NEXT-3 variants)");
-    if ((p->flags & PT_INIT_RANDOM) && (p->flags & PT_INIT_FWEIGHT))
+    if (simple && (variant || unique))
+        return fail(c, PT_ERR_ARG, "pt_track: PT_KERNEL_SIMPLE runs the base semantics only (no NEXT-3 variants, no PT_MAP_UNIQUE)");
+    if ((fl & PT_INIT_RANDOM) && (fl & PT_INIT_FWEIGHT))
         return fail(c, PT_ERR_ARG, "pt_track: PT_INIT_RANDOM and PT_INIT_FWEIGHT are exclusive");
-    const uint64_t H = (p->flags & PT_BIDIR) ? 2 : 1;   // output entries per particle
+    if (unique && (fl & PT_MAP_ACCUMULATE) == 0 && !map)
+        return fail(c, PT_ERR_ARG, "pt_track: PT_MAP_UNIQUE needs a map");
+    const uint64_t H = (fl & PT_BIDIR) ? 2 : 1;   // output entries per particle
     if (npart > UINT64_MAX / 2) return fail(c, PT_ERR_ARG, "pt_track: too many particles");
     const uint64_t nout = npart * H;
     DeviceGuard g(c->device);
     if (!g.ok) return fail(c, PT_ERR_CUDA, "pt_track: cannot select device %d", c->device);
     cudaStream_t st = c->stream;
 
+    // pid overflow: seed_id * P + (P - 1) must fit in 64 bits
+    const uint64_t max_id = (UINT64_MAX - (P - 1)) / P;
     // inputs: host -> device staging
     const float* d_seeds = seeds_xyz;
     const uint64_t* d_ids = seed_ids;
@@ -399,19 +464,17 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         d_seeds = c->d_seeds;
     }
     if (seed_ids) {
-        // pid overflow: seed_id * P + (P - 1) must fit in 64 bits
-        const uint64_t lim = (UINT64_MAX - (P - 1)) / P;
         if (!is_device_ptr(seed_ids)) {
             for (uint64_t i = 0; i < N; ++i)
-                if (seed_ids[i] > lim) return fail(c, PT_ERR_ARG, "pt_track: seed_id %llu * P overflows 64 bits", (unsigned long long)seed_ids[i]);
+                if (seed_ids[i] > max_id) return fail(c, PT_ERR_ARG, "pt_track: seed_id %llu * P overflows 64 bits", (unsigned long long)seed_ids[i]);
             if (N) {
                 CK(ensure(c->d_ids, c->ids_cap, N), "pt_track: id buffer");
                 CK(cudaMemcpyAsync(c->d_ids, seed_ids, N * sizeof(uint64_t), cudaMemcpyHostToDevice, st), "pt_track: ids H2D");
                 d_ids = c->d_ids;
             }
         }
-        // device-resident ids are not range-checked (the caller guarantees id*P+P-1 < 2^64)
-    } else if (N && N - 1 > (UINT64_MAX - (P - 1)) / P) {
+        // device-resident ids are checked by the kernel (kStatBadId -> PT_ERR_ARG in pt_get_stats)
+    } else if (N && N - 1 > max_id) {
         return fail(c, PT_ERR_ARG, "pt_track: pid overflow");
     }
 
@@ -423,10 +486,9 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         CK(ensure(c->d_map, c->map_cap, V), "pt_track: map buffer");
         d_map = c->d_map;
     }
-    const bool acc = (p->flags & PT_MAP_ACCUMULATE) != 0;
+    const bool acc = (fl & PT_MAP_ACCUMULATE) != 0;
 
     // outputs
-    const uint32_t fl = p->flags;
     if (fl & PT_REC_LEN) CK(ensure(c->d_nsteps, c->nsteps_cap, nout), "pt_track: nsteps buffer");
     if (fl & PT_REC_REASON) CK(ensure(c->d_reason, c->reason_cap, nout), "pt_track: reason buffer");
     if (fl & PT_REC_END) CK(ensure(c->d_end, c->end_cap, 3 * nout), "pt_track: end buffer");
@@ -444,9 +506,10 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         else CK(pt::launch_map_sum(d_map, (int64_t)V, c->d_stats + pt::kStatMapBefore, st), "pt_track: map sum");
     }
 
+    // Z-order (Morton) processing order of the seeds (cub's item count is an int: above
+    // INT_MAX seeds the input order is kept; results are identical either way)
     const uint32_t* d_order = nullptr;
-    if (!(fl & (PT_SEED_ORDER_INPUT | PT_KERNEL_SIMPLE)) && N > 1) {
-        if (N > 0xFFFFFFFFull) return fail(c, PT_ERR_ARG, "pt_track: more than 2^32-1 seeds");
+    if (!(fl & (PT_SEED_ORDER_INPUT | PT_KERNEL_SIMPLE)) && N > 1 && N <= 0x7FFFFFFFull) {
         CK(ensure(c->d_order, c->order_cap, 4 * N), "pt_track: order buffers");
         const size_t tb = pt::seed_order_temp_bytes(N);
         CK(ensure(c->d_temp, c->temp_cap, tb), "pt_track: sort temp storage");
@@ -489,6 +552,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.P = P;
     a.seeds = d_seeds;
     a.seed_ids = d_ids;
+    a.max_seed_id = max_id;
     a.order = d_order;
     a.nseeds = N;
     a.nparticles = npart;
@@ -517,16 +581,6 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         a.total_chunks = a.group_chunks + (N - a.group_chunks * G);
     }
     a.map = d_map;
-    a.map_copies = 1;
-    const bool simple = (fl & PT_KERNEL_SIMPLE) != 0;
-    uint32_t copies = (d_map && !simple && !variant && npart > 0) ? (uint32_t)PT_MAP_COPIES : 1u;
-    if (copies > (uint32_t)c->num_sms) copies = (uint32_t)c->num_sms;
-    if (copies > 1) {
-        CK(ensure(c->d_copies, c->copies_cap, (size_t)copies * V), "pt_track: map copies");
-        CK(cudaMemsetAsync(c->d_copies, 0, (size_t)copies * V * sizeof(uint32_t), st), "pt_track: map copies zero");
-        a.map = c->d_copies;
-        a.map_copies = copies;
-    }
     a.o_nsteps = (fl & PT_REC_LEN) ? c->d_nsteps : nullptr;
     a.o_reason = (fl & PT_REC_REASON) ? c->d_reason : nullptr;
     a.o_end = (fl & PT_REC_END) ? c->d_end : nullptr;
@@ -540,8 +594,35 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.interp = (fl & PT_INTERP) ? 1u : 0u;
     a.init_mode = (fl & PT_INIT_RANDOM) ? 1u : ((fl & PT_INIT_FWEIGHT) ? 2u : 0u);
     a.mask = c->d_mask;
+    pt::TrackMode mode;
+    mode.simple = simple;
+    mode.out = a.o_nsteps || a.o_reason || a.o_end || a.o_paths || a.conn;
+    mode.var = variant;
+    mode.unique = unique;
+    if (unique && npart) {
+        // one hash set per resident lane, >= 2x the most voxels a streamline can enter
+        // (H halves x max_steps committed steps); the buffer is capped (PT_UNIQUE_MB, default
+        // 8192 MB) by launching fewer persistent CTAs
+        uint32_t ulog = 1;
+        while ((1ull << ulog) < 2ull * H * (uint64_t)p->max_steps + 2ull) ++ulog;
+        const uint64_t per_cta = (uint64_t)pt::kThreadsExt << ulog;  // entries (UNQ CTAs are kThreadsExt wide)
+        uint64_t budget = 8192ull << 20;
+        if (const char* e = getenv("PT_UNIQUE_MB")) budget = (uint64_t)atoll(e) << 20;
+        uint64_t ctas = budget / (per_cta * sizeof(unsigned long long));
+        if (ctas < 1) ctas = 1;
+        const uint64_t full = (uint64_t)(c->num_sms > 0 ? c->num_sms : 1);
+        if (ctas > full) ctas = full;
+        const uint64_t need = (npart + pt::kThreadsExt - 1) / pt::kThreadsExt;
+        if (ctas > need) ctas = need;
+        CK(ensure(c->d_utab, c->utab_cap, (size_t)(ctas * per_cta)), "pt_track: unique-map hash sets");
+        CK(cudaMemsetAsync(c->d_utab, 0, (size_t)(ctas * per_cta) * sizeof(unsigned long long), st),
+           "pt_track: unique-map hash sets zero");
+        a.utab = c->d_utab;
+        a.ulog = ulog;
+        a.max_ctas = ctas;
+    }
 
-    if (!segmented) CK(cudaEventRecord(c->ev[1], st), "pt_track: event");
+    CK(cudaEventRecord(c->ev[1], st), "pt_track: event");
     if (segmented) {
         const uint32_t batch = (uint32_t)(npart < (1ull << 26) ? (npart ? npart : 1) : (1ull << 26));
         const size_t tb = pt::seg_select_temp_bytes(batch);
@@ -565,22 +646,14 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         uint32_t* d_count = reinterpret_cast<uint32_t*>(take(16));
         ss.flag = take((size_t)batch);
         void* temp = take(tb);
-        CK(cudaEventRecord(c->ev[1], st), "pt_track: event");
         CK(pt::run_segmented(a, c->vol.nfibres, c->vol.dtype == PT_F16, ss, batch, c->seg_sched, c->seg_n, live_b,
                              d_count, temp, tb, st),
            "pt_track: segmented relaunch");
-    } else if (variant)
-        CK(pt::launch_track_var(a, c->vol.nfibres, c->vol.dtype == PT_F16, c->num_sms, st),
-           "pt_track: variant tracking kernel launch");
-    else if (fl & PT_KERNEL_SPEC)
-        CK(pt::launch_track_spec(a, c->vol.nfibres, c->vol.dtype == PT_F16, c->num_sms, st),
+    } else {
+        CK(pt::launch_track(a, mode, c->vol.nfibres, c->vol.dtype == PT_F16, c->num_sms, st),
            "pt_track: tracking kernel launch");
-    else
-        CK(pt::launch_track(a, c->vol.nfibres, c->vol.dtype == PT_F16, (fl & PT_KERNEL_SIMPLE) != 0, c->num_sms, st),
-           "pt_track: tracking kernel launch");
+    }
     CK(cudaEventRecord(c->ev[2], st), "pt_track: event");
-    if (a.map_copies > 1)
-        CK(pt::launch_map_combine(a.map, a.map_copies, (int64_t)V, d_map, true, st), "pt_track: map combine");
     if (d_map) CK(pt::launch_map_sum(d_map, (int64_t)V, c->d_stats + pt::kStatMapAfter, st), "pt_track: map sum");
     if (host_map) {
         CK(cudaMemcpyAsync(map, d_map, V * sizeof(uint32_t), cudaMemcpyDeviceToHost, st), "pt_track: map D2H");
@@ -621,7 +694,15 @@ pt_status pt_load_targets(pt_ctx* c, const uint8_t* labels, int32_t ntargets) {
     const size_t V = (size_t)c->vol.nx * c->vol.ny * c->vol.nz;
     CK(ensure(c->d_labels, c->labels_cap, V), "pt_load_targets: label buffer");
     CK(cudaMemcpyAsync(c->d_labels, labels, V, cudaMemcpyDefault, c->stream), "pt_load_targets: copy");
+    c->ntargets = 0;
+    CK(cudaMemsetAsync(c->d_stats + pt::kStatLabelMax, 0, sizeof(unsigned long long), c->stream), "pt_load_targets: reset");
+    CK(pt::launch_label_max(c->d_labels, (int64_t)V, c->d_stats + pt::kStatLabelMax, c->stream), "pt_load_targets: scan");
+    unsigned long long lmax = 0;
+    CK(cudaMemcpyAsync(&lmax, c->d_stats + pt::kStatLabelMax, sizeof lmax, cudaMemcpyDeviceToHost, c->stream),
+       "pt_load_targets: scan result");
     CK(cudaStreamSynchronize(c->stream), "pt_load_targets: synchronise");
+    if (lmax > (unsigned long long)ntargets)
+        return fail(c, PT_ERR_ARG, "pt_load_targets: label %llu > ntargets %d", lmax, ntargets);
     c->ntargets = ntargets;
     return PT_OK;
 }
@@ -657,13 +738,17 @@ pt_status pt_get_stats(pt_ctx* c, pt_stats* out) {
     out->lane_active = s[pt::kStatLaneActive];
     out->lane_slots = s[pt::kStatLaneSlots];
     out->map_sum = s[pt::kStatMapAfter];
-    out->spec_hits = s[pt::kStatSpecHits];
-    out->overflow = (c->last_map && s[pt::kStatMapAfter] != s[pt::kStatMapBefore] + s[pt::kStatSteps]) ? 1 : 0;
+    out->unique_visits = s[pt::kStatUnique];
+    // the map gains one count per committed step (R13), or per first entry with PT_MAP_UNIQUE
+    const unsigned long long added = (c->last_flags & PT_MAP_UNIQUE) ? s[pt::kStatUnique] : s[pt::kStatSteps];
+    out->overflow = (c->last_map && s[pt::kStatMapAfter] != s[pt::kStatMapBefore] + added) ? 1 : 0;
     float ms = 0.f;
     CK(cudaEventElapsedTime(&ms, c->ev[1], c->ev[2]), "pt_get_stats: kernel time");
     out->kernel_ms = ms;
     CK(cudaEventElapsedTime(&ms, c->ev[0], c->ev[3]), "pt_get_stats: track time");
     out->track_ms = ms;
+    if (s[pt::kStatBadId])
+        return fail(c, PT_ERR_ARG, "pt_track: a device-resident seed_id * P overflows 64 bits (those particles ran as seed id 0)");
     if (out->overflow) return fail(c, PT_ERR_OVERFLOW, "a uint32 map cell wrapped past 2^32-1");
     return PT_OK;
 }
@@ -696,6 +781,52 @@ pt_status pt_get_paths(pt_ctx* c, pt_paths* out) {
     pt_stats s;
     pt_status rc = pt_get_stats(c, &s);
     return rc;
+}
+
+pt_status pt_get_load_stats(pt_ctx* c, pt_load_stats* out) {
+    if (!c || !out) return PT_ERR_ARG;
+    c->err.clear();
+    if (!c->loaded) return fail(c, PT_ERR_STATE, "pt_get_load_stats: no sample volume loaded");
+    DeviceGuard g(c->device);
+    float a = 0.f, b = 0.f;
+    CK(cudaEventElapsedTime(&a, c->lev[0], c->lev[1]), "pt_get_load_stats: h2d time");
+    CK(cudaEventElapsedTime(&b, c->lev[1], c->lev[2]), "pt_get_load_stats: repack time");
+    out->h2d_ms = a;
+    out->repack_ms = b;
+    out->h2d_bytes = c->load_h2d_bytes;
+    out->record_bytes = c->rec_size;
+    return PT_OK;
+}
+
+pt_status pt_rng_draws(pt_ctx* c, const uint64_t* pid, const uint32_t* block, const uint32_t* stream, int64_t n,
+                       uint64_t rng_seed, uint32_t nsamples, uint32_t* words, uint32_t* samples,
+                       int64_t* mismatches) {
+    if (!c) return PT_ERR_ARG;
+    c->err.clear();
+    if (n < 0 || nsamples < 1 || (n > 0 && (!pid || !block || !stream || !words || !samples)) || !mismatches)
+        return fail(c, PT_ERR_ARG, "pt_rng_draws: NULL array, n < 0 or nsamples < 1");
+    DeviceGuard g(c->device);
+    cudaStream_t st = c->stream;
+    const size_t un = (size_t)n;
+    Staged sp, sb, ss, sw, sm;
+    CK(sp.in(pid, un * 8, st), "pt_rng_draws: pid");
+    CK(sb.in(block, un * 4, st), "pt_rng_draws: block");
+    CK(ss.in(stream, un * 4, st), "pt_rng_draws: stream");
+    CK(sw.out(words, un * 16), "pt_rng_draws: words");
+    CK(sm.out(samples, un * 12), "pt_rng_draws: samples");
+    CK(cudaMemsetAsync(c->d_stats + pt::kStatLabelMax, 0, sizeof(unsigned long long), st), "pt_rng_draws: reset");
+    CK(pt::launch_rng_draws(static_cast<const uint64_t*>(sp.dev), static_cast<const uint32_t*>(sb.dev),
+                            static_cast<const uint32_t*>(ss.dev), n, (uint32_t)rng_seed, (uint32_t)(rng_seed >> 32),
+                            nsamples, static_cast<uint32_t*>(sw.dev), static_cast<uint32_t*>(sm.dev),
+                            c->d_stats + pt::kStatLabelMax, st),
+       "pt_rng_draws: kernel");
+    CK(sw.finish(st), "pt_rng_draws: words D2H");
+    CK(sm.finish(st), "pt_rng_draws: samples D2H");
+    unsigned long long mm = 0;
+    CK(cudaMemcpyAsync(&mm, c->d_stats + pt::kStatLabelMax, sizeof mm, cudaMemcpyDeviceToHost, st), "pt_rng_draws: count");
+    CK(cudaStreamSynchronize(st), "pt_rng_draws: synchronise");
+    *mismatches = (int64_t)mm;
+    return PT_OK;
 }
 
 pt_status pt_gather_bench(pt_ctx* c, int64_t buffer_bytes, int32_t record_bytes, double* sectors_per_s) {
@@ -755,49 +886,6 @@ pt_status pt_gather_bench(pt_ctx* c, int64_t buffer_bytes, int32_t record_bytes,
 
 // ------------------------------------------------------------------------- NEXT-4 MCMC
 
-namespace {
-
-// Device view of a caller buffer: device pointers are used in place; host inputs are
-// copied into a temporary device buffer; host outputs get a temporary device buffer that
-// is copied back by finish().
-struct Staged {
-    void* dev = nullptr;
-    void* tmp = nullptr;
-    void* host_out = nullptr;
-    size_t bytes = 0;
-    ~Staged() {
-        if (tmp) cudaFree(tmp);
-    }
-    cudaError_t in(const void* p, size_t n, cudaStream_t st) {
-        bytes = n;
-        if (!p || is_device_ptr(p)) {
-            dev = const_cast<void*>(p);
-            return cudaSuccess;
-        }
-        cudaError_t e = cudaMalloc(&tmp, n ? n : 1);
-        if (e != cudaSuccess) return e;
-        dev = tmp;
-        return cudaMemcpyAsync(tmp, p, n, cudaMemcpyHostToDevice, st);
-    }
-    cudaError_t out(void* p, size_t n) {
-        bytes = n;
-        if (!p || is_device_ptr(p)) {
-            dev = p;
-            return cudaSuccess;
-        }
-        cudaError_t e = cudaMalloc(&tmp, n ? n : 1);
-        if (e != cudaSuccess) return e;
-        dev = tmp;
-        host_out = p;
-        return cudaSuccess;
-    }
-    cudaError_t finish(cudaStream_t st) {
-        if (!host_out) return cudaSuccess;
-        return cudaMemcpyAsync(host_out, dev, bytes, cudaMemcpyDeviceToHost, st);
-    }
-};
-
-}  // namespace
 
 extern "C" {
 

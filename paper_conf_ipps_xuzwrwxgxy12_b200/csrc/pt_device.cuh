@@ -15,9 +15,12 @@ constexpr uint32_t kFull = 0xFFFFFFFFu;
 
 // ---------------------------------------------------------------------------- RNG (R16)
 // Philox4x32-10 (Salmon et al., SC'11): counter-based, so a particle's draws depend only
-// on (rng_seed, pid, block) and never on scheduling.  One block = 4 words: words 0..2
-// give the sample indices of steps 3b, 3b+1, 3b+2; word 3 of block 0 gives the first
-// step's sign.  Replaces the combined Tausworthe generator of P:L153.
+// on (rng_seed, pid, stream, block) and never on scheduling.  Counter = {block, pid_lo,
+// pid_hi, stream}.  Stream 0 (1 = the reverse half of a bidirectional streamline, R22):
+// words 0..2 of block b give the sample indices of steps 3b, 3b+1, 3b+2; word 3 of block 0
+// gives the first step's sign.  Stream 2 + half, block n: interpolation draws of step n
+// (R23) and the first-fibre draw (word 3 of block 0, R24).  Replaces the combined
+// Tausworthe generator of P:L153 (the frozen contract: DESIGN.md R16).
 __device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint32_t k0, uint32_t k1) {
 #pragma unroll
     for (int r = 0; r < 10; ++r) {
@@ -96,22 +99,6 @@ __device__ __forceinline__ void ldg_record<64>(const void* p, uint32_t* w) {
     ldg_record<32>(static_cast<const char*>(p) + 32, w + 8);
 }
 
-// L2 prefetch size of the record gathers: on an L2 miss the line's neighbourhood (the
-// voxel's adjacent samples) comes along, so siblings drawing other samples of the same
-// voxel hit in L2.  PT_L2_PREFETCH: 0 = none, 64/128/256 bytes.
-#ifndef PT_L2_PREFETCH
-#define PT_L2_PREFETCH 0
-#endif
-#if PT_L2_PREFETCH == 256
-#define PT_LDQ ".L2::256B"
-#elif PT_L2_PREFETCH == 128
-#define PT_LDQ ".L2::128B"
-#elif PT_L2_PREFETCH == 64
-#define PT_LDQ ".L2::64B"
-#else
-#define PT_LDQ ""
-#endif
-
 // Predicated variants for straight-line step code: the load / reduction is issued only by
 // lanes with p != 0; the destination registers of the other lanes keep their values.
 template <int BYTES>
@@ -119,19 +106,19 @@ __device__ __forceinline__ void ldg_record_if(bool p, const void* ptr, uint32_t*
 
 template <>
 __device__ __forceinline__ void ldg_record_if<8>(bool p, const void* ptr, uint32_t* w) {
-    asm("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %3, 0;\n\t@q ld.global.nc" PT_LDQ ".v2.b32 {%0,%1}, [%2];\n\t}"
+    asm("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %3, 0;\n\t@q ld.global.nc" ".v2.b32 {%0,%1}, [%2];\n\t}"
         : "+r"(w[0]), "+r"(w[1])
         : "l"(ptr), "r"((int)p));
 }
 template <>
 __device__ __forceinline__ void ldg_record_if<16>(bool p, const void* ptr, uint32_t* w) {
-    asm("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %5, 0;\n\t@q ld.global.nc" PT_LDQ ".v4.b32 {%0,%1,%2,%3}, [%4];\n\t}"
+    asm("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %5, 0;\n\t@q ld.global.nc" ".v4.b32 {%0,%1,%2,%3}, [%4];\n\t}"
         : "+r"(w[0]), "+r"(w[1]), "+r"(w[2]), "+r"(w[3])
         : "l"(ptr), "r"((int)p));
 }
 template <>
 __device__ __forceinline__ void ldg_record_if<32>(bool p, const void* ptr, uint32_t* w) {
-    asm("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %9, 0;\n\t@q ld.global.nc" PT_LDQ ".v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];\n\t}"
+    asm("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %9, 0;\n\t@q ld.global.nc" ".v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];\n\t}"
         : "+r"(w[0]), "+r"(w[1]), "+r"(w[2]), "+r"(w[3]), "+r"(w[4]), "+r"(w[5]), "+r"(w[6]), "+r"(w[7])
         : "l"(ptr), "r"((int)p));
 }

@@ -15,15 +15,11 @@ namespace pt {
 // tickets), so a seed's particles run on one SM (L1 locality) while the chip as a whole
 // works on a compact set of Morton-adjacent seeds (L2 locality).
 constexpr int kThreads = PT_CTA_THREADS;
-#ifndef PT_CTA_THREADS2
-#define PT_CTA_THREADS2 768
-#endif
-constexpr int kThreads2 = PT_CTA_THREADS2;  // CTA size of the 2-slot kernel (<= 85 registers)
 constexpr int kSimpleThreads = 256;  // no-refill ablation kernel
-#ifndef PT_VAR_THREADS
-#define PT_VAR_THREADS 768
+#ifndef PT_CTA_THREADS_EXT
+#define PT_CTA_THREADS_EXT 768
 #endif
-constexpr int kVarThreads = PT_VAR_THREADS;  // NEXT-3 variant kernel (one CTA per SM)
+constexpr int kThreadsExt = PT_CTA_THREADS_EXT;  // variant / unique-map instantiations
 constexpr uint32_t kSub = 32;
 constexpr uint32_t kMinCtaChunk = 1024;
 
@@ -37,8 +33,10 @@ enum StatIdx {
     kStatMapBefore = 5,  // sum of map cells before the kernel (accumulate mode)
     kStatQueue = 6,      // work-queue counter (chunks claimed)
     kStatBadInput = 7,   // repack: non-finite value inside the mask
-    kStatSpecHits = 8,   // steps taken with the speculative record (pt_spec.cu)
-    kNumStats = 9
+    kStatBadId = 8,      // a device-resident seed id whose pid overflows 64 bits
+    kStatUnique = 9,     // UNQ: first entries counted (= increments of the unique map)
+    kStatLabelMax = 10,  // pt_load_targets: largest label
+    kNumStats = 11
 };
 
 struct TrackArgs {
@@ -63,9 +61,8 @@ struct TrackArgs {
     uint64_t group_chunks;       // ... for claims < group_chunks; later claims are one seed each
     uint32_t chunks_per_seed;    // ceil(P / cta_chunk)
     uint64_t total_chunks;       // nseeds * chunks_per_seed
+    uint64_t max_seed_id;        // largest seed id whose pids fit 64 bits: (2^64-1 - (P-1)) / P
     uint32_t* map;               // [V] or nullptr: the map this launch adds into
-    uint32_t map_copies;         // > 1: map points at map_copies private [V] copies;
-                                 //      CTA b adds into copy b % map_copies
     uint16_t* o_nsteps;          // [nparticles] or nullptr
     uint8_t* o_reason;
     float* o_end;                // [nparticles][3]
@@ -75,11 +72,23 @@ struct TrackArgs {
     uint32_t* conn;              // [nseeds][ntargets] seed x target matrix or nullptr
     int path_stride;
     unsigned long long* stats;   // [kNumStats]
-    // NEXT-3 variants (track_var_kernel only; R22-R24)
+    // NEXT-3 variants (VAR instantiations only; R22-R24)
     uint32_t bidir;              // 1: two halves per particle, outputs at 2*i + half
     uint32_t interp;             // 1: probabilistic interpolation of the sampled voxel
     uint32_t init_mode;          // first fibre: 0 fibre 0, 1 uniform eligible, 2 f-weighted
     const uint8_t* mask;         // [V] tracking mask (interp: candidate test) or nullptr
+    // NEXT-2 per-streamline-unique map (UNQ instantiations only; R25)
+    unsigned long long* utab;    // [lanes][2^ulog] generation-tagged hash sets, zeroed per call
+    uint32_t ulog;               // log2 entries per lane's hash set
+    uint64_t max_ctas;           // CTAs the hash-set buffer covers
+};
+
+// Which instantiation of the tracking kernel a call runs.
+struct TrackMode {
+    bool simple;  // no-refill ablation (i)
+    bool out;     // per-particle outputs / polylines / connectivity recorded
+    bool var;     // NEXT-3 variants (run-time selected by bidir / interp / init_mode)
+    bool unique;  // NEXT-2 per-streamline-unique map
 };
 
 // NEXT-4 MCMC sampler (pt_mcmc.cu): one warp per voxel of the compacted mask list.
@@ -125,15 +134,18 @@ cudaError_t run_segmented(const TrackArgs& a, int F, bool half, const SegState& 
                           const int32_t* schedule, int nsched, uint32_t* live_b, uint32_t* d_count, void* temp,
                           size_t temp_bytes, cudaStream_t st);
 
-// Launchers (return the launch error, if any).
-cudaError_t launch_track(const TrackArgs& a, int nfibres, bool half, bool simple, int num_sms,
+// Launchers (return the launch error, if any).  launch_track dispatches on F to
+// launch_track_f<F> (pt_track_f{1,2,3}.cu, one translation unit per fibre count).
+cudaError_t launch_track(const TrackArgs& a, const TrackMode& m, int nfibres, bool half, int num_sms,
                          cudaStream_t st);
-// Speculative tracking kernel (PT_KERNEL_SPEC ablation): persistent + refill + a second
-// gather at the extrapolated next voxel (pt_spec.cu).
-cudaError_t launch_track_spec(const TrackArgs& a, int nfibres, bool half, int num_sms, cudaStream_t st);
-// NEXT-3 variant kernel (bidirectional / interpolation / first-fibre modes; also runs the
-// default semantics when forced with PT_KERNEL_VARIANT).
-cudaError_t launch_track_var(const TrackArgs& a, int nfibres, bool half, int num_sms, cudaStream_t st);
+template <int F>
+cudaError_t launch_track_f(const TrackArgs& a, const TrackMode& m, bool half, int num_sms, cudaStream_t st);
+// pt_rng_draws: the tracking RNG on explicit counters, cross-checked against curand
+cudaError_t launch_rng_draws(const uint64_t* pid, const uint32_t* block, const uint32_t* stream, int64_t n,
+                             uint32_t k0, uint32_t k1, uint32_t S, uint32_t* words, uint32_t* samples,
+                             unsigned long long* mismatches, cudaStream_t st);
+// max over the target labels (pt_load_targets validation) into *out
+cudaError_t launch_label_max(const uint8_t* labels, int64_t V, unsigned long long* out, cudaStream_t st);
 // Record layout (see rec_vox in pt_device.cuh): b = brick log2 edge, 0 (raster) or
 // kBrickLog (the default; the main tracking kernel is compiled for these two).
 constexpr uint32_t kBrickLog = 4;
@@ -151,9 +163,6 @@ cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask,
 size_t seed_order_temp_bytes(uint64_t nseeds);
 cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint32_t* keys, uint32_t* keys_out,
                               uint32_t* idx, uint32_t* perm, void* temp, size_t temp_bytes, cudaStream_t st);
-// out[v] (+)= sum over c of copies[c * V + v]
-cudaError_t launch_map_combine(const uint32_t* copies, uint32_t ncopies, int64_t V, uint32_t* out,
-                               bool accumulate, cudaStream_t st);
 cudaError_t launch_map_sum(const uint32_t* map, int64_t V, unsigned long long* out,
                            cudaStream_t st);
 cudaError_t launch_gather_bench(const uint8_t* buf, uint64_t nrec, int rec_bytes, uint32_t iters,

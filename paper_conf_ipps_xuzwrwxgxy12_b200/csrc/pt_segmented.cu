@@ -55,7 +55,11 @@ __global__ void seg_init_kernel(const __grid_constant__ TrackArgs a, SegState s,
         const uint64_t g = base + i;                 // processing-order particle index
         const uint64_t k = g / a.P, j = g - k * a.P;
         const uint64_t si = a.order ? a.order[k] : k;
-        const uint64_t sid = a.seed_ids ? a.seed_ids[si] : si;
+        uint64_t sid = a.seed_ids ? a.seed_ids[si] : si;
+        if (sid > a.max_seed_id) {  // pid would overflow 64 bits: reported as PT_ERR_ARG
+            atomicExch(a.stats + kStatBadId, 1ull);
+            sid = 0;
+        }
         s.li[i] = si * a.P + j;
         s.pid[i] = sid * a.P + j;
         const float qx = __fsub_rn(a.seeds[3 * si + 0], a.fcx);
@@ -67,7 +71,9 @@ __global__ void seg_init_kernel(const __grid_constant__ TrackArgs a, SegState s,
         s.p[3 * i] = s.p[3 * i + 1] = s.p[3 * i + 2] = 0.f;
         s.n[i] = 0u;
         uint32_t v;
-        const bool ok = inside_volume(a, qx, qy, qz, v) && a.mask[v] != 0;
+        // non-finite seeds are outside (R12; a NaN would truncate into the volume)
+        const bool fin = isfinite(qx) && isfinite(qy) && isfinite(qz);
+        const bool ok = fin && inside_volume(a, qx, qy, qz, v) && a.mask[v] != 0;
         s.vox[i] = v;
         s.live[i] = i;
         s.flag[i] = ok ? 1 : 0;

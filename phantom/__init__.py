@@ -29,7 +29,7 @@ import numpy as np
 
 __all__ = [
     "Volume", "Workload", "tube", "crossing", "whole_brain", "isotropic", "bent_tube",
-    "t_junction", "fork", "paper_dataset", "mirror_x", "to_half", "config", "CONFIGS", "wm_seeds",
+    "t_junction", "fork", "vortex", "paper_dataset", "mirror_x", "to_half", "config", "CONFIGS", "wm_seeds",
     "DwiWorkload", "gradient_scheme", "dwi_brain", "dwi_uniform", "MCMC_CONFIGS", "mcmc_config",
 ]
 
@@ -391,6 +391,37 @@ def t_junction(x_j=40, nx=64, ny=64, nz=16, y=(24, 40), width=8, nsamples=16,
     return Workload("t_junction", vol, seeds, None, step=step, curv_thr=curv_thr,
                     rng_seed=rng_seed, particles_per_seed=particles_per_seed,
                     recipe=f"T junction at x={x_j}")
+
+
+def vortex(n=48, nz=4, r_in=6.0, r_out=20.0, nsamples=8, sigma=0.0, seed_r=(10, 13, 16), nseeds_per_r=4,
+           particles_per_seed=32, max_steps=600, step=0.5, curv_thr=0.2, gen_seed=31, rng_seed=99) -> Workload:
+    """Closed loops (NEXT-2 pins, R25): an annulus r_in <= r < r_out around the volume's
+    z-axis, F = 1, fibre = the tangent (-dy, dx, 0) / r at the voxel centre (plus a sigma
+    dispersion per sample), f = 1, mask = the annulus (all slices).  Streamlines circle the
+    axis and come back to voxels they have already entered, so a per-streamline-unique map
+    differs from the step map.  Seeds at voxel centres on circles of radius seed_r."""
+    rng = np.random.Generator(np.random.PCG64(gen_seed))
+    F, S = 1, nsamples
+    dy, f, mask = _empty(n, n, nz, S, F)
+    zz, yy, xx = np.meshgrid(np.arange(nz), np.arange(n), np.arange(n), indexing="ij")
+    cx = cy = n / 2.0
+    dxv, dyv = xx + 0.5 - cx, yy + 0.5 - cy
+    r = np.sqrt(dxv ** 2 + dyv ** 2)
+    mask[(r >= r_in) & (r < r_out)] = 1
+    t = np.stack([-dyv, dxv, np.zeros_like(r)], -1) / np.maximum(r, 1e-9)[..., None]
+    t = np.broadcast_to(t.astype(np.float32), (F, S, nz, n, n, 3))
+    dy[...] = _disperse(t, sigma, rng) if sigma > 0 else t
+    f[...] = 1.0
+    vol = Volume(n, n, nz, S, F, np.ascontiguousarray(dy), f, mask)
+    pts = []
+    for rr in seed_r:
+        for k in range(nseeds_per_r):
+            a = 2 * math.pi * k / nseeds_per_r + 0.3
+            pts.append([int(cx + rr * math.cos(a)), int(cy + rr * math.sin(a)), nz // 2])
+    seeds = _centres(np.array(pts))
+    return Workload("vortex", vol, seeds, None, step=step, curv_thr=curv_thr, max_steps=max_steps,
+                    rng_seed=rng_seed, particles_per_seed=particles_per_seed,
+                    recipe=f"vortex annulus [{r_in}, {r_out}) sigma {sigma}")
 
 
 def mirror_x(w: Workload) -> Workload:

@@ -7,7 +7,8 @@
   (iii) fp32 vs fp16 records (c3 vs c4)
   (v)   raster vs Morton seed order (PT_SEED_ORDER_INPUT)
   (vi)  raster vs bricked record layout (PT_BRICK=0 vs the default 16^3 bricks)
-  plus the speculative-gather kernel (PT_KERNEL_SPEC) and the NEXT-3 variant kernel on the default semantics (PT_KERNEL_VARIANT).
+  plus the NEXT-3 variant instantiation on the default semantics (PT_KERNEL_VARIANT), the
+  variants themselves (PT_BIDIR, PT_INTERP) and the NEXT-2 unique map (PT_MAP_UNIQUE).
 
 Every run's total steps must equal the main kernel's (same parity contract: the results
 are identical, only the schedule differs).  Prints one JSON line per variant and a markdown
@@ -50,9 +51,13 @@ def main():
 
     variants = [
         ("main (persistent, lane refill, Morton)", 0, None, w),
-        ("speculative 2nd gather, 2 steps/iteration on a hit (PT_KERNEL_SPEC)", pt.PT_KERNEL_SPEC, None, w),
         ("(v) raster seed order", pt.PT_SEED_ORDER_INPUT, None, w),
-        ("variant kernel, default semantics", pt.PT_KERNEL_VARIANT, None, w),
+        ("variant instantiation, default semantics", pt.PT_KERNEL_VARIANT, None, w),
+        ("NEXT-3 bidirectional", pt.PT_BIDIR, None, w),
+        ("NEXT-3 probabilistic interpolation", pt.PT_INTERP, None, w),
+        ("NEXT-3 bidirectional + interpolation + f-weighted first fibre",
+         pt.PT_BIDIR | pt.PT_INTERP | pt.PT_INIT_FWEIGHT, None, w),
+        ("NEXT-2 per-streamline-unique map", pt.PT_MAP_UNIQUE, None, w),
         ("(i) no refill, one thread per particle (A_MaxStep)", pt.PT_KERNEL_SIMPLE, None, w),
         ("(ii) segmented A_1", pt.PT_KERNEL_SEGMENTED, (1,), w),
         ("(ii) segmented A_10", pt.PT_KERNEL_SEGMENTED, (10,), w),

@@ -71,8 +71,21 @@ def _first_fibre(mode, ff, fthr, word):
 
 def track(w, seed_index: int, j: int, max_points: int = 10**9):
     """Track one particle (half 0); returns (nsteps, reason, positions float32 [n+1][3])."""
-    n, why, pos, _ = _half(w, seed_index, j, 0, None, max_points)
+    n, why, pos, _, _ = _half(w, seed_index, j, 0, None, max_points)
     return n, why, pos
+
+
+def streamline_voxels(w, seed_index: int, j: int) -> set:
+    """The set of voxels (z, y, x) the committed steps of one streamline (all its halves)
+    land in -- what the per-streamline-unique map counts once (R25)."""
+    out = set()
+    d0 = None
+    for h in range(2 if getattr(w, "bidir", 0) else 1):
+        _, _, _, d, vox = _half(w, seed_index, j, h, d0, 1)
+        if h == 0:
+            d0 = d
+        out.update(vox)
+    return out
 
 
 def track_streamline(w, seed_index: int, j: int, max_points: int = 10**9):
@@ -80,7 +93,7 @@ def track_streamline(w, seed_index: int, j: int, max_points: int = 10**9):
     out = []
     d0 = None
     for h in range(2 if getattr(w, "bidir", 0) else 1):
-        n, why, pos, d = _half(w, seed_index, j, h, d0, max_points)
+        n, why, pos, d, _ = _half(w, seed_index, j, h, d0, max_points)
         if h == 0:
             d0 = d
         out.append((n, why, pos))
@@ -116,13 +129,14 @@ def _half(w, seed_index: int, j: int, half: int, d0, max_points: int):
     pos = [[q[a] + c[a] for a in range(3)]]
     vox = lookup(q)
     d_first = None
+    visited = []  # voxel of every committed step
     if vox is None or (half == 1 and d0 is None):
-        return 0, 0, np.array(pos, np.float32), None
+        return 0, 0, np.array(pos, np.float32), None, visited
     n = 0
     p = None if half == 0 else [-d0[a] for a in range(3)]
     while True:
         if n == w.max_steps:
-            return n, 2, np.array(pos, np.float32), d_first
+            return n, 2, np.array(pos, np.float32), d_first, visited
         wd = philox4x32_10([n // 3, pid & _M, pid >> 32, half], key)
         s = (j % S) if getattr(w, "sample_mode", 0) == 1 else (wd[n % 3] * S) >> 32
         first = n == 0 and half == 0
@@ -148,7 +162,7 @@ def _half(w, seed_index: int, j: int, half: int, d0, max_points: int):
             if js is None:
                 js = 0
             if not (abs(dots[js]) > thr):
-                return n, 1, np.array(pos, np.float32), d_first
+                return n, 1, np.array(pos, np.float32), d_first, visited
             sg = np.float32(1.0) if dots[js] > np.float32(0) else np.float32(-1.0)
         d = [sg * vv[js][a] for a in range(3)]
         if first:
@@ -156,8 +170,9 @@ def _half(w, seed_index: int, j: int, half: int, d0, max_points: int):
         qn = [q[a] + h * d[a] for a in range(3)]
         vn = lookup(qn)
         if vn is None:
-            return n, 0, np.array(pos, np.float32), d_first
+            return n, 0, np.array(pos, np.float32), d_first, visited
         q, p, vox = qn, d, vn
         n += 1
+        visited.append(vn)
         if len(pos) < max_points:
             pos.append([q[a] + c[a] for a in range(3)])

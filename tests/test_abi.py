@@ -47,10 +47,11 @@ def test_no_fma_in_stepping_code(ptlib):
     """R15: the library is compiled with -fmad=false; no FFMA may appear in the tracking
     kernels (a contracted a*b+c would change rounding vs the oracle)."""
     sass = subprocess.run(["cuobjdump", "-sass", ptlib.LIB], capture_output=True, text=True).stdout
-    assert "track_kernel" in sass and "track_var_kernel" in sass
+    assert "track_kernel" in sass
     funcs = re.split(r"\n\s*Function : ", sass)
     tracking = [f for f in funcs if f.split("\n", 1)[0].find("track") >= 0]
-    assert len(tracking) >= 24          # 12 main-kernel and 12 variant-kernel instantiations
+    # per (F, precision): 2 bench-path layouts, outputs, 4 variant / unique-map, 2 no-refill
+    assert len(tracking) >= 6 * 11
     for f in tracking:
         assert "FFMA" not in f, f.split("\n", 1)[0]
 

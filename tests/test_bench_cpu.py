@@ -45,3 +45,25 @@ def test_mcmc_reference_arm_json_line():
     d = json.loads(lines[0])
     assert d["impl"] == "reference" and d["unit"] == "voxels/s" and d["value"] > 0
     assert d["cpu_baseline"]["kind"] == "oracle" and d["dtype"] == "f64"
+
+
+def test_bench_self_launches_ranks():
+    """bench.py --gpus 2 without a torch.distributed environment re-launches itself as two
+    ranks (torch.distributed.run); rank 0 prints the one JSON line, rank 1 stays silent."""
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--gpus", "2",
+                          "--config", "c1", "--steps", "1", "--warmup", "1", "--cpu-seconds", "0.3"],
+                         capture_output=True, text=True, timeout=600, cwd=ROOT, env=env)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, out.stdout
+    assert json.loads(lines[0])["n_gpus"] == 2
+    assert "torch.distributed.run" in out.stderr and "--nproc-per-node 2" in out.stderr
+
+
+def test_bench_refuses_world_mismatch():
+    """Our arm must not time fewer ranks than --gpus asks for."""
+    env = dict(os.environ, WORLD_SIZE="1", RANK="0", LOCAL_RANK="0")
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--config", "c1"],
+                         capture_output=True, text=True, timeout=600, cwd=ROOT, env=env)
+    assert out.returncode != 0 and "WORLD_SIZE" in out.stderr

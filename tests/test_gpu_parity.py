@@ -174,15 +174,53 @@ def test_record_layout_rejects_other_bricks(pt, monkeypatch):
 # ----------------------------------------------------------------------------- full size, sampled
 
 @pytest.mark.parametrize("cfg", ["c3", "c4"])
-def test_whole_brain_full_size_sampled(pt, tracker, cfg):
-    """configs[2]/[3] at full size in the launch configuration bench.py times (persistent
-    kernel, all WM seeds x 5000 particles): 3000 sampled particles recomputed one by one
-    by the oracle, plus the global invariants at full size."""
+def test_timed_instantiation_map_vs_oracle(pt, tracker, cfg):
+    """The exact launch bench.py times (flags = 0: no per-particle outputs, compile-time
+    16^3-brick layout, Morton claims) on configs[2] / [3]: every 16th WM seed at the full
+    P = 5000, the FULL uint32 map compared with the oracle's bit for bit, and the kernel's
+    step counter with the oracle's total."""
+    import torch
+    w = phantom.wm_seeds(phantom.config(cfg), every=16)
+    tracker.load_volume(w.volume)
+    m = tracker.track_workload(w, flags=0)
+    torch.cuda.synchronize()
+    st = tracker.stats()
+    gm = m.cpu().numpy().view(np.uint32)
+    r = oracle.track(w, want_particles=False, threads=_threads())
+    assert np.array_equal(gm.astype(np.uint64), r["map"]), \
+        f"{np.count_nonzero(gm.astype(np.uint64) != r['map'])} map cells differ"
+    assert st["total_steps"] == int(r["map"].sum())
+    assert st["particles"] == w.nparticles
+
+
+@pytest.mark.parametrize("cfg", ["c2", "c2_dispersed"])
+def test_timed_instantiation_full_config(pt, tracker, cfg):
+    """configs[1] in the bench launch (flags = 0): the full map bit-exact vs the oracle."""
     import torch
     w = phantom.config(cfg)
     tracker.load_volume(w.volume)
+    m = tracker.track_workload(w, flags=0)
+    torch.cuda.synchronize()
+    r = oracle.track(w, want_particles=False, threads=_threads())
+    assert np.array_equal(m.cpu().numpy().view(np.uint32).astype(np.uint64), r["map"])
+    assert tracker.stats()["total_steps"] == int(r["map"].sum())
+
+
+@pytest.mark.parametrize("cfg", ["c3", "c4"])
+def test_whole_brain_full_size_sampled(pt, tracker, cfg):
+    """configs[2]/[3] at full size (all WM seeds x 5000 particles): the map of the bench
+    launch (flags = 0) equals the map of the outputs instantiation bit for bit, and 3000
+    sampled particles of the latter are recomputed one by one by the oracle, plus the global
+    invariants at full size."""
+    import torch
+    w = phantom.config(cfg)
+    tracker.load_volume(w.volume)
+    m0 = tracker.track_workload(w, flags=0).clone()
+    torch.cuda.synchronize()
+    steps0 = tracker.stats()["total_steps"]
     m = tracker.track_workload(w, flags=REC_ALL)
     torch.cuda.synchronize()
+    assert torch.equal(m0, m) and tracker.stats()["total_steps"] == steps0
     st = tracker.stats()
     out = tracker.get_paths(on_device=True)
     nst = out["nsteps"].to(torch.int64)
@@ -212,6 +250,71 @@ def test_whole_brain_full_size_sampled(pt, tracker, cfg):
         np.any(g["end"].view(np.uint32) != r["end"].view(np.uint32), axis=1)
     assert diverged.sum() == 0, f"{diverged.sum()} of {len(pick)} sampled streamlines diverge"
     assert r["nsteps"].mean() > 10
+
+
+# ----------------------------------------------------------------------------- NEXT-2 unique map
+
+def _unique_run(pt, tr, w, extra=0):
+    import torch
+    tr.load_volume(w.volume)
+    m = tr.track_workload(w, flags=pt.PT_MAP_UNIQUE | extra)
+    torch.cuda.synchronize()
+    return m.cpu().numpy().view(np.uint32), tr.stats()
+
+
+@pytest.mark.parametrize("cfg", ["c2", "c2_dispersed"])
+def test_unique_map_full_config(pt, tracker, cfg):
+    """PT_MAP_UNIQUE (R25): configs[1] at full size, map bit-exact vs the oracle's
+    per-streamline-unique map; the overflow check balances on the unique counts."""
+    w = phantom.config(cfg)
+    gm, st = _unique_run(pt, tracker, w)
+    r = oracle.track(w, want_particles=False, want_unique=True, threads=_threads())
+    assert np.array_equal(gm.astype(np.uint64), r["umap"])
+    assert st["unique_visits"] == int(r["umap"].sum()) and st["total_steps"] == int(r["map"].sum())
+    assert st["overflow"] == 0
+
+
+@pytest.mark.parametrize("rec", [False, True])
+@pytest.mark.parametrize("variant", [0, 1, 2])
+def test_unique_map_loops_and_variants(pt, tracker, variant, rec):
+    """Closed loops (vortex: streamlines revisit their voxels ~3 times), with and without the
+    NEXT-3 variants (bidirectional union of halves, interpolation + f-weighted first fibre)
+    and with per-particle outputs recorded on the side."""
+    w = phantom.vortex(sigma=0.2, particles_per_seed=64, max_steps=700)
+    w = w.replace(bidir=int(variant >= 1), interp=int(variant == 2), init_fibre=2 if variant == 2 else 0)
+    flags = pt.PT_REC_LEN if rec else 0
+    gm, st = _unique_run(pt, tracker, w, flags | pt.variant_flags(w.bidir, w.interp, w.init_fibre))
+    r = oracle.track(w, want_unique=True, threads=_threads())
+    assert np.array_equal(gm.astype(np.uint64), r["umap"])
+    assert r["map"].sum() > 1.5 * r["umap"].sum()
+    if rec:
+        g = tracker.get_paths(nsteps=True, reason=False, end=False)
+        assert np.array_equal(g["nsteps"].astype(np.int64), r["nsteps"].astype(np.int64))
+
+
+def test_unique_map_whole_brain_sampled(pt, tracker):
+    """configs[2] shape: every 64th WM seed at full P, unique map bit-exact vs the oracle;
+    and a small hash-set budget (fewer persistent CTAs) gives the same map."""
+    import os as _os
+    w = phantom.wm_seeds(phantom.config("c3"), every=64)
+    gm, st = _unique_run(pt, tracker, w)
+    r = oracle.track(w, want_particles=False, want_unique=True, threads=_threads())
+    assert np.array_equal(gm.astype(np.uint64), r["umap"])
+    _os.environ["PT_UNIQUE_MB"] = "64"
+    try:
+        gm2, _ = _unique_run(pt, tracker, w)
+    finally:
+        del _os.environ["PT_UNIQUE_MB"]
+    assert np.array_equal(gm2, gm)
+
+
+def test_unique_map_errors(pt, tracker):
+    w = phantom.tube(particles_per_seed=4)
+    tracker.load_volume(w.volume)
+    for bad in (pt.PT_KERNEL_SIMPLE, pt.PT_KERNEL_SEGMENTED):
+        with pytest.raises(pt.PtError) as e:
+            tracker.track_workload(w, flags=pt.PT_MAP_UNIQUE | bad)
+        assert e.value.status == pt.PT_ERR_ARG
 
 
 def test_c5_hcp_scale_sampled(pt, tracker):
@@ -345,6 +448,37 @@ def test_errors(pt):
     with pytest.raises(pt.PtError) as e:
         t.get_paths(paths=True)
     t.close()
+
+
+def test_argument_checks(pt, tracker):
+    """ADVICE r01: wrong dtypes are refused by the binding before a pointer crosses the ABI;
+    labels above ntargets are PT_ERR_ARG (no out-of-bounds connectivity write); a
+    device-resident seed id whose pids overflow 64 bits is reported as PT_ERR_ARG."""
+    import torch
+    w = phantom.crossing(sigma=0.15, nseeds=8, particles_per_seed=8)
+    tracker.load_volume(w.volume)
+    kw = dict(step=w.step, curv_thr=w.curv_thr, fib_thr=w.fib_thr, max_steps=w.max_steps,
+              rng_seed=w.rng_seed, particles_per_seed=w.particles_per_seed)
+    with pytest.raises(TypeError):
+        tracker.track(w.seeds.astype(np.float64), None, **kw)
+    with pytest.raises(TypeError):
+        tracker.track(w.seeds, np.arange(w.nseeds, dtype=np.int32), **kw)
+    with pytest.raises(ValueError):
+        tracker.track(w.seeds[:, :2].copy(), None, **kw)
+    v = w.volume
+    with pytest.raises(TypeError):
+        tracker.load_samples(v.dyads, v.f.astype(np.float16), v.mask, v.nsamples, v.nfibres)
+    lab = np.zeros(v.mask.shape, np.uint8)
+    lab[0, 0, 0] = 9
+    with pytest.raises(pt.PtError) as e:
+        tracker.load_targets(lab, 8)
+    assert e.value.status == pt.PT_ERR_ARG
+    tracker.load_targets(lab, 9)
+    big = torch.full((w.nseeds,), -1, dtype=torch.int64, device="cuda")  # 2^64 - 1
+    tracker.track(torch.as_tensor(w.seeds, device="cuda"), big, **kw)
+    with pytest.raises(pt.PtError) as e:
+        tracker.stats()
+    assert e.value.status == pt.PT_ERR_ARG
 
 
 def test_lane_efficiency_and_gather_bench(pt, tracker):
