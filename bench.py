@@ -54,10 +54,24 @@ MCMC_TEXT = {
 # Table III: valid voxels, CPU time, GPU time (HD 5870), context only
 PAPER_TABLE3 = {"m1": {"voxels": 205082, "cpu_s": 1383, "gpu_s": 41.3, "speedup": 33.6},
                 "m2": {"voxels": 402194, "cpu_s": 2724, "gpu_s": 80.1, "speedup": 34.0}}
-# executed FP64 lane-instructions (DFMA + DMUL + DADD) per voxel-loop of the MCMC kernel for
-# the Table III shape (n = 64, N = 2): ncu SASS count of the current kernel (v5),
-# profiles/r01f_v5_mcmc_ncu.md.  Per-unit figure of the MCMC roofline (bound "alu", FP64 pipe).
-MCMC_FP64_OPS_PER_VOXEL_LOOP = {"m1": 14322, "m2": 14322, "m2_prof": 14322}
+
+
+def mcmc_flops_per_mh_step(n: int, N: int) -> int:
+    """Algorithmic FP64 operations of one Metropolis-Hastings step: Eq. 1
+    evaluated at the proposal for all n measurements, plus the Gaussian log-likelihood.
+    Per measurement i: the ball term e^{-b_i d} (b_i d: 1 mul, exp: 1) weighted by (1 - sum
+    f) (1 mul); per stick j: r_i . v_j (3 mul + 2 add), squared (1), times b_i d (1), exp (1),
+    times f_j (1), added (1) = 10; the sum times S0 (1); the residual y_i - mu_i (1) and its
+    square accumulated (1 mul + 1 add).  Per step: 1 - sum f (N adds) and the log posterior
+    of M2/M3 (ln sigma, the 1/(2 sigma^2) scaling, the sin-theta priors and the
+    accept test: 8).  exp and ln count as one operation each (the FP64 pipe spends ~20
+    instructions on one -- the reason the measured fraction stays well below 1)."""
+    return n * (3 + 10 * N + 1 + 3) + N + 8
+
+
+def mcmc_flops_per_voxel_loop(n: int, N: int) -> int:
+    """One loop = one MH step per parameter (NP = 3 + 3N, Fig. 2 / P:L147)."""
+    return (3 + 3 * N) * mcmc_flops_per_mh_step(n, N)
 
 # Table II (P:L283-291) of the paper, for context beside the NEXT-1 paper-mode workloads:
 # (total fibre length = total steps, longest fibre) on the real CABI datasets, HD 5870.
@@ -248,11 +262,12 @@ def run_reference(args):
 # ----------------------------------------------------------------------------- NEXT-4 MCMC arm
 
 def _fp64_peak():
-    """FP64 FMA lane-instructions/s derived from the unit counts: 148 SMs x 64 FP64 lanes
-    per SM per clock x the measured max SM clock (MEASURED_PEAKS.json, else 1965 MHz)."""
+    """FP64 flop/s derived from the unit counts: 148 SMs x 64 FP64 lanes per SM per clock x
+    2 (an FMA is two operations) x the measured max SM clock (MEASURED_PEAKS.json, else
+    1965 MHz): 37.2 TFLOP/s at 1965 MHz."""
     p = _peaks()
     mhz = (p or {}).get("sm_max_mhz", 1965.0)
-    return 148 * 64 * mhz * 1e6
+    return 148 * 64 * 2 * mhz * 1e6
 
 
 def _mcmc_shard(d, rank, world):
@@ -333,16 +348,15 @@ def run_mcmc(args):
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
 
     kmean = sum(kms) / len(kms)
-    roof = None
     peak = _fp64_peak()
-    ops = MCMC_FP64_OPS_PER_VOXEL_LOOP.get(args.config)
-    if ops:
-        ach = st["voxels"] * d.loops * ops / (kmean * 1e-3)
-        roof = {"bound": "alu", "achieved": ach / 1e12, "peak": peak / 1e12,
-                "unit": "T FP64 lane-instructions/s", "frac": ach / peak, "traffic": None,
-                "kernel_ms": kmean, "fp64_lane_instructions_per_voxel_loop": ops,
-                "per_unit_source": "ncu SASS count (DFMA + DMUL + DADD), profiles/r01f_v5_mcmc_ncu.md",
-                "peak_source": "derived: 148 SMs x 64 FP64 lanes per clock x sm_max_mhz (FMA = 1 instruction)"}
+    ops = mcmc_flops_per_voxel_loop(int(d.nmeas), int(d.nfibres))
+    ach = st["voxels"] * d.loops * ops / (kmean * 1e-3)
+    roof = {"bound": "alu", "achieved": ach / 1e12, "peak": peak / 1e12,
+            "unit": "TFLOP/s (FP64)", "frac": ach / peak, "traffic": None,
+            "kernel_ms": kmean, "flops_per_voxel_loop": ops,
+            "per_unit_source": "algorithmic: Eq. 1 (P:L67-69) at the proposal for all n measurements per MH "
+                               "step, NP = 3 + 3N steps per loop (bench.mcmc_flops_per_mh_step; exp/ln = 1 op)",
+            "peak_source": "derived: 148 SMs x 64 FP64 lanes x 2 (FMA) x sm_max_mhz"}
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         import oracle

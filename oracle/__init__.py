@@ -20,23 +20,26 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "oracle.c")
 _SRC_MCMC = os.path.join(_HERE, "oracle_mcmc.c")
 _HDR = os.path.join(_HERE, "oracle.h")
-_LIB = os.path.join(_HERE, "liboracle.so")
+_LIB = os.environ.get("ORACLE_LIB") or os.path.join(_HERE, "liboracle.so")  # ORACLE_LIB: sanitizer build
 CFLAGS = ["-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared",
           "-Wall", "-Wextra"]
+SANITIZE = ["-fsanitize=address,undefined", "-fno-sanitize-recover=all", "-fno-omit-frame-pointer", "-g"]
 
 END_MASK, END_CURV, END_MAXLEN = 0, 1, 2
 
 
-def build(force: bool = False) -> str:
-    """Compile liboracle.so with gcc (no FMA contraction, no fast-math)."""
+def build(force: bool = False, out: Optional[str] = None, sanitize: bool = False) -> str:
+    """Compile liboracle.so with gcc (no FMA contraction, no fast-math).  ``sanitize``: an
+    ASan + UBSan build (load it with LD_PRELOAD=libasan.so and ORACLE_LIB=<out>)."""
+    lib_path = out or _LIB
     srcs = [_SRC, _SRC_MCMC]
-    stale = (not os.path.exists(_LIB) or
-             os.path.getmtime(_LIB) < max(os.path.getmtime(f) for f in srcs + [_HDR]))
+    stale = (not os.path.exists(lib_path) or
+             os.path.getmtime(lib_path) < max(os.path.getmtime(f) for f in srcs + [_HDR]))
     if force or stale:
-        tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, *srcs, "-lm"])
-        os.replace(tmp, _LIB)
-    return _LIB
+        tmp = lib_path + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", *CFLAGS, *(SANITIZE if sanitize else []), "-o", tmp, *srcs, "-lm"])
+        os.replace(tmp, lib_path)
+    return lib_path
 
 
 class _Volume(ctypes.Structure):
@@ -75,7 +78,7 @@ def lib():
     global _lib
     with _lock:
         if _lib is None:
-            L = ctypes.CDLL(build())
+            L = ctypes.CDLL(_LIB if os.environ.get("ORACLE_LIB") else build())
             vp = ctypes.c_void_p
             L.oracle_philox4x32_10.argtypes = [vp, vp, vp]
             L.oracle_half_to_float.argtypes = [ctypes.c_uint16]

@@ -31,7 +31,7 @@ def main():
     ap.add_argument("--config", default="c3")
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--seed-every", type=int, default=1)
-    ap.add_argument("--only", default="")
+    ap.add_argument("--only", default="", help="comma list of substrings of the variant names to run")
     args = ap.parse_args()
     import numpy as np
     import torch
@@ -75,7 +75,7 @@ def main():
     ref_steps = None
     loaded = None
     for name, flags, sched, wv, brick in variants:
-        if args.only and args.only not in name:
+        if args.only and not any(o and o in name for o in args.only.split(",")):
             continue
         if wv is None:
             wv = phantom.to_half(w)
