@@ -1,7 +1,8 @@
 """Build libpt.so in-tree with nvcc for sm_100a (no JIT cache, no torch extension).
 
 Each translation unit is compiled to an object in parallel (the tracking kernel's
-instantiations are split by fibre count into pt_track_f{1,2,3}.cu), then linked."""
+instantiations are split by fibre count and precision into pt_track_f<F>_<f32|f16>.cu), then
+linked."""
 from __future__ import annotations
 
 import os
@@ -15,8 +16,8 @@ CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.environ.get("PT_LIB") or os.path.join(PKG, "libpt.so")  # PT_LIB: experiment builds
 OBJDIR = os.path.join(PKG, "build")
-SOURCES = ["pt_api.cu", "pt_kernels.cu", "pt_track_f1.cu", "pt_track_f2.cu", "pt_track_f3.cu",
-           "pt_mcmc.cu", "pt_segmented.cu"]
+SOURCES = ["pt_api.cu", "pt_kernels.cu", "pt_mcmc.cu", "pt_segmented.cu"] + \
+    [f"pt_track_f{F}_{p}.cu" for F in (1, 2, 3) for p in ("f32", "f16")]
 HEADERS = ["pt_device.cuh", "pt_internal.h", "pt_claim.cuh", "pt_track.cuh"]
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

@@ -55,6 +55,20 @@ struct Rec {
     __device__ __forceinline__ bool outside() const {
         return HALF ? ((w[1] >> 16) == 0xFFFFu) : (w[3] == 0xFFFFFFFFu);
     }
+    // exchange fibre js (< F) with fibre 0 (straight-line selects, no local memory)
+    __device__ __forceinline__ void swap_to_front(int js) {
+        constexpr int WF = HALF ? 2 : 4;  // words per fibre
+#pragma unroll
+        for (int j = 1; j < F; ++j) {
+            const bool p = js == j;
+#pragma unroll
+            for (int k = 0; k < WF; ++k) {
+                const uint32_t a = w[k], b = w[WF * j + k];
+                w[k] = p ? b : a;
+                w[WF * j + k] = p ? a : b;
+            }
+        }
+    }
     __device__ __forceinline__ void fibre(int j, float& x, float& y, float& z, float& f) const {
         if (HALF) {
             const uint32_t a = w[2 * j], b = w[2 * j + 1];

@@ -62,7 +62,9 @@ struct TrackArgs {
     uint32_t chunks_per_seed;    // ceil(P / cta_chunk)
     uint64_t total_chunks;       // nseeds * chunks_per_seed
     uint64_t max_seed_id;        // largest seed id whose pids fit 64 bits: (2^64-1 - (P-1)) / P
-    uint32_t* map;               // [V] or nullptr: the map this launch adds into
+    uint32_t* map;               // the map this launch adds into, or nullptr: indexed by record
+                                 // position (rec_vox; [V'] bricked) for the stepping kernel, by
+                                 // raster voxel for the segmented ablation
     uint16_t* o_nsteps;          // [nparticles] or nullptr
     uint8_t* o_reason;
     float* o_end;                // [nparticles][3]
@@ -134,12 +136,12 @@ cudaError_t run_segmented(const TrackArgs& a, int F, bool half, const SegState& 
                           const int32_t* schedule, int nsched, uint32_t* live_b, uint32_t* d_count, void* temp,
                           size_t temp_bytes, cudaStream_t st);
 
-// Launchers (return the launch error, if any).  launch_track dispatches on F to
-// launch_track_f<F> (pt_track_f{1,2,3}.cu, one translation unit per fibre count).
+// Launchers (return the launch error, if any).  launch_track dispatches on (F, precision)
+// to launch_track_f<F, HALF> (pt_track_f<F>_<f32|f16>.cu, one translation unit each).
 cudaError_t launch_track(const TrackArgs& a, const TrackMode& m, int nfibres, bool half, int num_sms,
                          cudaStream_t st);
-template <int F>
-cudaError_t launch_track_f(const TrackArgs& a, const TrackMode& m, bool half, int num_sms, cudaStream_t st);
+template <int F, bool HALF>
+cudaError_t launch_track_f(const TrackArgs& a, const TrackMode& m, int num_sms, cudaStream_t st);
 // pt_rng_draws: the tracking RNG on explicit counters, cross-checked against curand
 cudaError_t launch_rng_draws(const uint64_t* pid, const uint32_t* block, const uint32_t* stream, int64_t n,
                              uint32_t k0, uint32_t k1, uint32_t S, uint32_t* words, uint32_t* samples,
@@ -163,6 +165,9 @@ cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask,
 size_t seed_order_temp_bytes(uint64_t nseeds);
 cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint32_t* keys, uint32_t* keys_out,
                               uint32_t* idx, uint32_t* perm, void* temp, size_t temp_bytes, cudaStream_t st);
+// map[v] += bmap[rec_vox(v)] (the kernel's record-ordered counts into the caller's raster map)
+cudaError_t launch_unbrick_add(const uint32_t* bmap, int nx, int ny, int nz, const RecLayout& L, uint32_t* map,
+                               cudaStream_t st);
 cudaError_t launch_map_sum(const uint32_t* map, int64_t V, unsigned long long* out,
                            cudaStream_t st);
 cudaError_t launch_gather_bench(const uint8_t* buf, uint64_t nrec, int rec_bytes, uint32_t iters,

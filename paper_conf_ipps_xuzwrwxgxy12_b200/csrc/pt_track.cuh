@@ -11,12 +11,16 @@
 //   OUT     per-particle outputs / polylines / the seed x target matrix are recorded
 //           (compiled out of the bench path).
 //   BL      record layout, log2 brick edge (0 raster, 4 = 16^3 bricks) as a compile-time
-//           constant, or -1: read from the launch arguments.
-//   VAR     NEXT-3 FSL-fidelity variants, selected at run time by the launch arguments:
-//           R22 bidirectional streamlines (half 1 restarts in the same lane at a round
-//           boundary), R23 probabilistic interpolation of the sampled voxel (one extra Philox
-//           block per step, stream 2 + half, plus a 1-byte mask read of the candidate's
-//           nearest voxel), R24 random / f-weighted first fibre.
+//           constant, or -1: read from the launch arguments.  The compile-time layouts are
+//           the bench path and assume the random-sample mode (R1); paper mode (NEXT-1,
+//           sample_mode = 1) runs the BL = -1 instantiations.
+//   VM      NEXT-3 FSL-fidelity variants compiled in (bit mask; 0 = the north star's
+//           semantics): kVarBidir R22 bidirectional streamlines (half 1 restarts in the same
+//           lane at a round boundary), kVarInterp R23 probabilistic interpolation of the
+//           sampled voxel (one extra Philox block per step, stream 2 + half, plus a 1-byte
+//           mask read of the candidate's nearest voxel), kVarInit R24 random / f-weighted
+//           first fibre.  Each compiled-in variant is still switched by its launch argument
+//           (bidir / interp / init_mode), so VM = kVarAll runs any combination.
 //   UNQ     NEXT-2 per-streamline-unique visitation map (R25): a voxel counts once
 //           per streamline; exact, through a per-lane open-addressing hash set of the
 //           voxels the streamline has entered (global scratch, generation-tagged).
@@ -37,6 +41,12 @@
 
 #ifndef PT_RUNLEN
 #define PT_RUNLEN 1  // merge consecutive visits of a voxel before the RED (0: ablation iv, one RED per step)
+#endif
+#ifndef PT_MAP_TILE
+#define PT_MAP_TILE 0  // experiment: shared-memory count tile over the CTA's current seed brick
+#endif
+#ifndef PT_TILE_EVERY
+#define PT_TILE_EVERY 16  // rounds between the CTA-wide tile flushes / re-targets
 #endif
 #ifndef PT_REFILL_MIN
 #define PT_REFILL_MIN 2  // free lanes a warp waits for before refilling (amortises the refill block)
@@ -59,24 +69,27 @@ __device__ __forceinline__ int interp_axis(float q, int c, uint32_t w) {
 }
 
 // State of the particle a lane owns.
-template <int F, bool HALF, bool VAR, bool UNQ>
+enum { kVarBidir = 1, kVarInterp = 2, kVarInit = 4, kVarAll = 7 };
+
+template <int F, bool HALF, bool UNQ>
 struct Lane {
     bool alive;        // holds a particle (half) in flight
     bool pend;         // the round's last candidate step waits for the next round's gather
     float qx, qy, qz;  // committed position, centred coordinates (R10)
     float px, py, pz;  // direction of the last (candidate) step
-    uint32_t gvox;     // voxel read by the round-start gather (seed or pending candidate)
+    uint32_t gvox;     // raster voxel of the round-start gather (RASTER instantiations only)
     uint32_t grv;      // its position in the record volume (rec_vox)
     int n;             // committed steps (of this half)
     uint64_t pid;      // global particle id = seed_id * P + j (RNG key, R16)
-    uint32_t run_vox, run_cnt;  // run-length merge of consecutive visits (UNQ: current voxel)
+    uint32_t run_vox, run_cnt;  // run-length merge of consecutive visits of the voxel whose
+                                // record position is run_vox (UNQ: the current voxel)
     uint32_t sfix;     // paper mode (NEXT-1): the particle's sample volume, j mod S
     int why;           // >= 0: ended with this reason, outputs pending (finish)
     uint4 W;           // Philox block of the current round (stream = half)
     Rec<F, HALF> rv;   // record of the current step
     uint64_t tmask;    // NEXT-2: targets entered by the streamline so far (bit t-1)
     uint32_t sidx;     // seed index of this call
-    // VAR (R22, R24)
+    // variants (R22, R24)
     uint32_t half;     // 0, or 1 = the reverse half of a bidirectional streamline
     bool have_d0;      // half 0 computed its first direction
     float d0x, d0y, d0z;
@@ -88,28 +101,53 @@ struct Lane {
 
 // CTA size: one CTA per SM; the variant / unique instantiations keep more state per lane
 // and run 768 threads (<= 85 registers) instead of 1024 (<= 64)
-template <bool REFILL, bool VAR, bool UNQ>
+template <bool REFILL, int VM, bool UNQ>
 __host__ __device__ constexpr int track_tpb() {
-    return REFILL ? ((VAR || UNQ) ? kThreadsExt : kThreads) : kSimpleThreads;
+    return REFILL ? (((VM & (kVarInterp | kVarInit)) != 0 || UNQ) ? kThreadsExt : kThreads) : kSimpleThreads;
 }
 
-template <int F, bool HALF, bool REFILL, bool OUT, int BL, bool VAR, bool UNQ>
-__global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel(const __grid_constant__ TrackArgs a) {
+template <int F, bool HALF, bool REFILL, bool OUT, int BL, int VM, bool UNQ>
+__global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(const __grid_constant__ TrackArgs a) {
     using R = Rec<F, HALF>;
-    using L = Lane<F, HALF, VAR, UNQ>;
+    using L = Lane<F, HALF, UNQ>;
     constexpr int RB = R::kBytes;
-    constexpr int TPB = track_tpb<REFILL, VAR, UNQ>();
+    constexpr int TPB = track_tpb<REFILL, VM, UNQ>();
+    constexpr bool VB = (VM & kVarBidir) != 0, VI = (VM & kVarInterp) != 0, VN = (VM & kVarInit) != 0;
     __shared__ unsigned long long s_li[OUT ? TPB : 1];  // particle index (outputs)
     __shared__ uint32_t s_q[TPB / 32][3];               // per-warp sub-chunk
     __shared__ unsigned long long s_work;               // CTA claim + tickets
+    // PT_MAP_TILE: counts of the CTA's current seed brick (16^3 voxels), flushed and re-targeted
+    // every PT_TILE_EVERY rounds at a CTA-wide barrier
+    constexpr bool TILE = PT_MAP_TILE && REFILL && VM == 0 && !UNQ && BL != 0;
+    __shared__ uint32_t s_tile[TILE ? 4096 : 1];
+    __shared__ uint32_t s_tile_br, s_cur_seed;
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t wib = threadIdx.x >> 5;
     const uint32_t lt_mask = (1u << lane) - 1u;
+    // the map this launch adds into is indexed by record position (rec_vox: the bricked
+    // voxel order of the records; pt_track adds it into the caller's raster map afterwards),
+    // so a step needs no raster index unless it reads a raster per-voxel array: the mask
+    // byte of PT_INTERP or the target labels of the connectivity matrix
     uint32_t* const map = a.map;
     const bool has_map = map != nullptr;
-    const uint32_t H = (VAR && a.bidir) ? 2u : 1u;     // output entries per particle
-    const bool interp = VAR && a.interp;
+    constexpr bool RASTER = VI || OUT;
+    const uint32_t H = (VB && a.bidir) ? 2u : 1u;      // output entries per particle
+    const bool interp = VI && a.interp;
+    const uint32_t init_mode = VN ? a.init_mode : 0u;
+    const bool smode = BL < 0 && a.sample_mode != 0u;  // paper mode (NEXT-1): s = j mod S
     if (threadIdx.x == 0) s_work = kNoChunk << 24;
+    if (TILE) {
+        for (int i = threadIdx.x; i < 4096; i += TPB) s_tile[i] = 0u;
+        if (threadIdx.x == 0) {
+            s_tile_br = 0xFFFFFFFFu;
+            s_cur_seed = 0xFFFFFFFFu;
+        }
+    }
+    // brick the tile covers (register copy, CTA-uniform; 0xFFFFFFFF: none, as brick ids are
+    // < 2^20); the tile is used only with a map and the 16^3-brick record layout
+    const bool tile_on = TILE && a.map != nullptr && a.rb_log == kBrickLog;
+    uint32_t tile_br = 0xFFFFFFFFu;
+    uint32_t trounds = 0;
     if (lane == 0) {
         s_q[wib][0] = 0u;
         s_q[wib][1] = 0u;
@@ -164,7 +202,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
     auto philox = [&](uint32_t block, uint32_t stream) -> uint4 {
         return philox4x32_10(make_uint4(block, (uint32_t)x.pid, (uint32_t)(x.pid >> 32), stream), a.key0, a.key1);
     };
-    auto out_index = [&]() -> uint64_t { return OUT ? s_li[threadIdx.x] * H + (VAR ? x.half : 0u) : 0ull; };
+    auto out_index = [&]() -> uint64_t { return OUT ? s_li[threadIdx.x] * H + (VB ? x.half : 0u) : 0ull; };
     // SetEndPoint() of a finished (half-)streamline: outputs, count flush
     auto write_outputs = [&](int n, int why, float qx, float qy, float qz) {
         if (OUT && (a.o_nsteps || a.o_reason || a.o_end)) {
@@ -197,8 +235,19 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
             my_steps = 0u;
         }
     };
+    // a run of visits of one voxel: into the tile if the voxel lies in the tile's brick
+    // (record position >> 12 = brick, & 4095 = voxel in the brick), else a global RED
+    auto red_run = [&](bool p, uint32_t rv, uint32_t cnt) {
+        if (TILE) {
+            const bool in_tile = (rv >> 12) == tile_br;
+            if (p && in_tile) atomicAdd(&s_tile[rv & 4095u], cnt);
+            red_add_if(p && !in_tile, map + rv, cnt);
+        } else {
+            red_add_if(p, map + rv, cnt);
+        }
+    };
     auto flush_run = [&]() {
-        if (!UNQ && has_map && x.run_cnt) atomicAdd(map + x.run_vox, x.run_cnt);  // RED
+        if (!UNQ && has_map) red_run(x.run_cnt != 0u, x.run_vox, x.run_cnt);
         x.run_cnt = 0u;
     };
     // begin half h of the current particle at its seed: centred position, seed voxel.
@@ -223,8 +272,9 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
         // non-finite seeds are outside (a NaN would truncate into the volume)
         const bool fin = isfinite(x.qx) && isfinite(x.qy) && isfinite(x.qz);
         if (fin && (unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny && (unsigned)iz < (unsigned)a.nz) {
-            x.gvox = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
-            x.grv = recv(ix, iy, iz, x.gvox);
+            const uint32_t v = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
+            if (RASTER) x.gvox = v;
+            x.grv = recv(ix, iy, iz, v);
             return true;
         }
         return false;
@@ -234,7 +284,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
         flush_run();
         write_outputs(x.n, x.why, x.qx, x.qy, x.qz);
         x.why = -1;
-        if (VAR && H == 2u && x.half == 0u) {
+        if (VB && H == 2u && x.half == 0u) {
             const bool ok = begin(1u) && x.have_d0;
             if (ok) {  // the reverse half starts against half 0's first direction
                 x.px = -x.d0x;
@@ -257,7 +307,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
             sid = 0;
         }
         x.pid = sid * a.P + j;
-        x.sfix = a.sample_mode ? (uint32_t)(j % a.S) : 0u;
+        x.sfix = smode ? (uint32_t)(j % a.S) : 0u;
         x.tmask = 0ull;
         x.sidx = (uint32_t)si;
         x.have_d0 = false;
@@ -271,14 +321,15 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
             // loop may hand this lane another particle
             x.alive = false;
             write_outputs(0, kEndMask, x.qx, x.qy, x.qz);
-            if (VAR && H == 2u) {
+            if (VB && H == 2u) {
                 begin(1u);  // (outside again) point 0 of half 1's polyline
                 write_outputs(0, kEndMask, x.qx, x.qy, x.qz);
             }
             particle_done();
         }
     };
-    // UNQ (R25): has the streamline entered voxel v before?  Inserts it if not.
+    // UNQ (R25): has the streamline entered the voxel at record position v before?  Inserts
+    // it if not.
     auto first_entry = [&](bool c, uint32_t v) -> bool {
         bool fresh = false;
         bool probe = c && v != x.run_vox && v != x.prev_vox;
@@ -302,26 +353,27 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
     // commit a step (if c): new position, one visit of the new voxel (R13);
     // consecutive visits of the same voxel are merged (run length) and flushed with a
     // predicated RED when the voxel changes.  Straight-line except for the UNQ probe.
-    auto commit_if = [&](bool c, float nx_, float ny_, float nz_, uint32_t v) {
+    // v: raster voxel (RASTER instantiations), vrv: its record position (the map index)
+    auto commit_if = [&](bool c, float nx_, float ny_, float nz_, uint32_t v, uint32_t vrv) {
         x.qx = c ? nx_ : x.qx;
         x.qy = c ? ny_ : x.qy;
         x.qz = c ? nz_ : x.qz;
         x.n += c ? 1 : 0;
         if (UNQ) {
-            const bool fresh = first_entry(c, v);
-            red_add_if(has_map && fresh, map + v, 1u);
+            const bool fresh = first_entry(c, vrv);
+            red_add_if(has_map && fresh, map + vrv, 1u);
             my_unique += fresh ? 1u : 0u;
-            const bool change = c && v != x.run_vox;
+            const bool change = c && vrv != x.run_vox;
             x.prev_vox = change ? x.run_vox : x.prev_vox;
-            x.run_vox = c ? v : x.run_vox;
+            x.run_vox = c ? vrv : x.run_vox;
         } else if (has_map) {
 #if PT_RUNLEN
-            const bool change = v != x.run_vox;
-            red_add_if(c && change && x.run_cnt != 0u, map + x.run_vox, x.run_cnt);
+            const bool change = vrv != x.run_vox;
+            red_run(c && change && x.run_cnt != 0u, x.run_vox, x.run_cnt);
             x.run_cnt = c ? (change ? 1u : x.run_cnt + 1u) : x.run_cnt;
-            x.run_vox = c ? v : x.run_vox;
+            x.run_vox = c ? vrv : x.run_vox;
 #else
-            red_add_if(c, map + v, 1u);  // ablation (iv): one global RED per committed step
+            red_add_if(c, map + vrv, 1u);  // ablation (iv): one global RED per committed step
 #endif
         }
         if (OUT && a.conn && c) {  // NEXT-2: targets entered by committed steps (R21)
@@ -346,8 +398,9 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
             ldg_record_if<RB>(p, rec_at(nrv, s), x.rv.w);
             return p && x.rv.outside();
         }
-        const uint4 I = philox(nn, 2u + x.half);
-        if (nn == 0u && x.half == 0u) x.winit = I.w;
+        const uint32_t hh = VB ? x.half : 0u;
+        const uint4 I = philox(nn, 2u + hh);
+        if (VN && nn == 0u && hh == 0u) x.winit = I.w;
         const int jx = interp_axis(cqx, a.cx, I.x), jy = interp_axis(cqy, a.cy, I.y), jz = interp_axis(cqz, a.cz, I.z);
         const bool jin = (unsigned)jx < (unsigned)a.nx && (unsigned)jy < (unsigned)a.ny && (unsigned)jz < (unsigned)a.nz;
         const uint32_t jv = ((uint32_t)jz * (uint32_t)a.ny + (uint32_t)jy) * (uint32_t)a.nx + (uint32_t)jx;
@@ -372,7 +425,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
         }
         if (ne == 0u) return 0;
         int js = 0;
-        if (a.init_mode == 1u) {  // uniform over E: E[floor(w |E| / 2^32)]
+        if (init_mode == 1u) {  // uniform over E: E[floor(w |E| / 2^32)]
             const uint32_t r = __umulhi(x.winit, ne);
             uint32_t before = 0;  // eligible fibres before j
 #pragma unroll
@@ -406,10 +459,13 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
     // one step of Alg. 1's inner loop; k = position in the round
     auto step = [&](int k) {
         my_active += x.alive ? 1u : 0u;
-        const bool first = x.n == 0 && (!VAR || x.half == 0u);
+        // a streamline's first step is always step 0 of a round (fresh particles start at a
+        // round start; a live lane has n >= 1 after step 0): compile-time false for k > 0
+        const bool first = k == 0 && x.n == 0 && (!VB || x.half == 0u);
         // choose the fibre closest to the previous direction: eligible iff
         // f_j > fib_thr (R7), strict >, lowest j wins (R8); the first step takes fibre 0
-        // (R5) or the R24 draw.  "Interpolation()" of Alg. 1 = this sample's record (R2).
+        // (R5; with R24 the round start moved the drawn fibre to slot 0).  "Interpolation()" of
+        // Alg. 1 = this sample's record (R2).
         float vx, vy, vz, f0;
         x.rv.fibre(0, vx, vy, vz, f0);
         float bc = __fadd_rn(__fadd_rn(__fmul_rn(vx, x.px), __fmul_rn(vy, x.py)), __fmul_rn(vz, x.pz));
@@ -426,24 +482,13 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
             vy = pick ? uy : vy;
             vz = pick ? uz : vz;
         }
-        if (VAR && F > 1 && a.init_mode != 0u && __any_sync(kFull, first && x.alive)) {
-            const int js = first ? initial_fibre() : 0;
-#pragma unroll
-            for (int j = 1; j < F; ++j) {
-                float ux, uy, uz, fu;
-                x.rv.fibre(j, ux, uy, uz, fu);
-                vx = js == j ? ux : vx;
-                vy = js == j ? uy : vy;
-                vz = js == j ? uz : vz;
-            }
-        }
         // maximum angle, measured by the dot product (R4); orientation
         // kept (R9); first step: sign = top bit of word 3 of block 0 (R6, R16)
         const bool curv_ok = first || fabsf(bc) > a.curv_thr;
         const bool neg = first ? (x.W.w >> 31) != 0u : !(bc > 0.f);
         // StepToNextPoint(): q' = q + h * (sign * v), no FMA
         const float dx = neg ? -vx : vx, dy = neg ? -vy : vy, dz = neg ? -vz : vz;
-        if (VAR) {  // R22: half 0's first direction, defined even if the step is not committed
+        if (VB) {  // R22: half 0's first direction, defined even if the step is not committed
             const bool rec0 = first && x.alive;
             x.d0x = rec0 ? dx : x.d0x;
             x.d0y = rec0 ? dy : x.d0y;
@@ -455,7 +500,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
         const float nqz = __fadd_rn(x.qz, __fmul_rn(a.step, dz));
         const int ix = axis_index(nqx, a.cx), iy = axis_index(nqy, a.cy), iz = axis_index(nqz, a.cz);
         const bool inb = (unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny && (unsigned)iz < (unsigned)a.nz;
-        const uint32_t v = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
+        const uint32_t v = RASTER ? ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix : 0u;
         // stop criteria in order: maximum steps (R14), angle, volume (R11)
         const bool maxed = x.n == a.max_steps;
         const bool go = x.alive && !maxed && curv_ok && inb;
@@ -468,17 +513,18 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
             if ((k + 1) % 3 == 0) {
                 // the next step opens the round's next Philox block: a live lane has
                 // committed t0 + k steps, so that block is (n + 1) / 3 (R16)
-                x.W = philox(((uint32_t)x.n + 1u) / 3u, VAR ? x.half : 0u);
+                x.W = philox(((uint32_t)x.n + 1u) / 3u, VB ? x.half : 0u);
             }
             const uint32_t w = ((k + 1) % 3 == 0) ? x.W.x : ((k + 1) % 3 == 1) ? x.W.y : x.W.z;
-            const uint32_t sk = a.sample_mode ? x.sfix : sample_of(w, a.S);
-            const bool outside = gather(go, nqx, nqy, nqz, recv(ix, iy, iz, v), v, (uint32_t)x.n + 1u, sk);
+            const uint32_t sk = smode ? x.sfix : sample_of(w, a.S);
+            const uint32_t vrv = recv(ix, iy, iz, v);
+            const bool outside = gather(go, nqx, nqy, nqz, vrv, v, (uint32_t)x.n + 1u, sk);
             x.why = outside ? kEndMask : x.why;
             x.alive = go && !outside;
-            commit_if(x.alive, nqx, nqy, nqz, v);
+            commit_if(x.alive, nqx, nqy, nqz, v, vrv);
         } else {
             x.pend = go;  // next round's start gathers and tests it
-            x.gvox = go ? v : x.gvox;
+            if (RASTER) x.gvox = go ? v : x.gvox;
             x.grv = go ? recv(ix, iy, iz, v) : x.grv;
         }
     };
@@ -519,6 +565,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
                     const uint32_t avail = cend - cnext;
                     const uint32_t rank = __popc(need & lt_mask);
                     if (!x.alive && rank < avail) start(cseed, (uint64_t)(cnext + rank));
+                    if (TILE && lane == 0) s_cur_seed = cseed;
                     const uint32_t cnt = (uint32_t)__popc(need);
                     cnext += cnt < avail ? cnt : avail;
                     need = __ballot_sync(kFull, !x.alive);
@@ -532,26 +579,68 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
                 __syncwarp();
             }
         }
-        if (!__any_sync(kFull, x.alive)) break;
+        const bool warp_alive = __any_sync(kFull, x.alive);
+        if (TILE) {
+            // every PT_TILE_EVERY iterations all warps of the CTA meet (warps without work
+            // run empty iterations): flush the tile, re-target it at the brick of the seed
+            // the CTA claimed last, or leave when the CTA has nothing left
+            if (++trounds % PT_TILE_EVERY == 0u) {
+                const bool cont = __syncthreads_or(x.alive || !exhausted);
+                if (tile_br != 0xFFFFFFFFu) {
+                    uint32_t* const mb = map + ((size_t)tile_br << 12);  // the brick, contiguous
+                    for (uint32_t i = threadIdx.x; i < 4096u; i += TPB) {
+                        const uint32_t c = s_tile[i];
+                        if (c != 0u) atomicAdd(mb + i, c);
+                        s_tile[i] = 0u;
+                    }
+                }
+                if (threadIdx.x == 0) {
+                    uint32_t br = 0xFFFFFFFFu;
+                    const uint32_t sd = s_cur_seed;
+                    if (tile_on && sd != 0xFFFFFFFFu) {
+                        const float sx = a.seeds[3 * sd], sy = a.seeds[3 * sd + 1], sz = a.seeds[3 * sd + 2];
+                        if (sx >= 0.f && sy >= 0.f && sz >= 0.f && sx < (float)a.nx && sy < (float)a.ny &&
+                            sz < (float)a.nz)
+                            br = (((uint32_t)sz >> 4) * a.rb_nby + ((uint32_t)sy >> 4)) * a.rb_nbx + ((uint32_t)sx >> 4);
+                    }
+                    s_tile_br = br;
+                }
+                __syncthreads();
+                tile_br = s_tile_br;
+                if (!cont) break;
+            }
+            if (!warp_alive) continue;
+        } else if (!warp_alive) {
+            break;
+        }
         rounds += 1u;
 
         // ------------------------------------------------ round start: one Philox block,
         // gather of (pending candidate | seed) voxel = mask test + first step's record
         {
             const uint32_t t0 = (uint32_t)x.n + (x.pend ? 1u : 0u);  // a multiple of 3
-            x.W = philox(t0 / 3u, VAR ? x.half : 0u);
-            const uint32_t s0 = a.sample_mode ? x.sfix : sample_of(x.W.x, a.S);
+            x.W = philox(t0 / 3u, VB ? x.half : 0u);
+            const uint32_t s0 = smode ? x.sfix : sample_of(x.W.x, a.S);
             // the pending candidate, recomputed bit-identically from (q, d) instead of kept
             const float cqx = x.pend ? __fadd_rn(x.qx, __fmul_rn(a.step, x.px)) : x.qx;
             const float cqy = x.pend ? __fadd_rn(x.qy, __fmul_rn(a.step, x.py)) : x.qy;
             const float cqz = x.pend ? __fadd_rn(x.qz, __fmul_rn(a.step, x.pz)) : x.qz;
-            if (VAR && a.init_mode != 0u && !interp && t0 == 0u && x.half == 0u && x.alive)
+            if (VN && init_mode != 0u && !interp && t0 == 0u && (!VB || x.half == 0u) && x.alive)
                 x.winit = philox(0u, 2u).w;  // R24 draw (with PT_INTERP the gather computes it)
             // seed outside the mask (R12) or pending candidate rejected (R11)
             const bool outside = gather(x.alive, cqx, cqy, cqz, x.grv, x.gvox, t0, s0);
             x.why = outside ? kEndMask : x.why;
             x.alive = x.alive && !outside;
-            commit_if(x.pend && !outside, cqx, cqy, cqz, x.gvox);
+            commit_if(x.pend && !outside, cqx, cqy, cqz, x.gvox, x.grv);
+            // R24: the first step of half 0 takes the drawn fibre: move it to slot 0 of the
+            // record (the first step uses only the chosen fibre's vector)
+            if (VN && F > 1 && init_mode != 0u) {
+                const bool fresh = x.alive && t0 == 0u && (!VB || x.half == 0u);
+                if (__any_sync(kFull, fresh)) {
+                    const int js = fresh ? initial_fibre() : 0;
+                    x.rv.swap_to_front(js);
+                }
+            }
             x.pend = false;
         }
 
@@ -580,10 +669,10 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VAR, UNQ>(), 1) track_kernel
 
 // grid of one launch: persistent (at most #SMs x resident CTAs, or fewer when the job or the
 // UNQ hash sets are smaller) or one thread per particle
-template <int F, bool HALF, bool REFILL, bool OUT, int BL, bool VAR, bool UNQ>
+template <int F, bool HALF, bool REFILL, bool OUT, int BL, int VM, bool UNQ>
 cudaError_t launch_track_kernel(const TrackArgs& a, int num_sms, cudaStream_t st) {
-    auto k = track_kernel<F, HALF, REFILL, OUT, BL, VAR, UNQ>;
-    constexpr int TPB = track_tpb<REFILL, VAR, UNQ>();
+    auto k = track_kernel<F, HALF, REFILL, OUT, BL, VM, UNQ>;
+    constexpr int TPB = track_tpb<REFILL, VM, UNQ>();
     if (a.nparticles == 0) return cudaSuccess;
     unsigned grid;
     if (REFILL) {
@@ -602,27 +691,43 @@ cudaError_t launch_track_kernel(const TrackArgs& a, int num_sms, cudaStream_t st
     return cudaGetLastError();
 }
 
-// All instantiations for one (F, HALF); pt_track_f{1,2,3}.cu define launch_track_f<F>.
+// All instantiations for one (F, HALF); pt_track_f<F>_<h|f>.cu define launch_track_f<F>.
+template <int F, bool HALF, int VM>
+cudaError_t launch_track_var(const TrackArgs& a, const TrackMode& m, int num_sms, cudaStream_t st) {
+    return m.out ? launch_track_kernel<F, HALF, true, true, -1, VM, false>(a, num_sms, st)
+                 : launch_track_kernel<F, HALF, true, false, -1, VM, false>(a, num_sms, st);
+}
+
 template <int F, bool HALF>
 cudaError_t launch_track_fh(const TrackArgs& a, const TrackMode& m, int num_sms, cudaStream_t st) {
     if (m.simple) {  // ablation (i): default semantics only
-        return m.out ? launch_track_kernel<F, HALF, false, true, -1, false, false>(a, num_sms, st)
-                     : launch_track_kernel<F, HALF, false, false, -1, false, false>(a, num_sms, st);
+        return m.out ? launch_track_kernel<F, HALF, false, true, -1, 0, false>(a, num_sms, st)
+                     : launch_track_kernel<F, HALF, false, false, -1, 0, false>(a, num_sms, st);
     }
-    if (m.unique) {
+    if (m.unique) {  // NEXT-2: default semantics, or every variant switched at run time
         if (m.var)
-            return m.out ? launch_track_kernel<F, HALF, true, true, -1, true, true>(a, num_sms, st)
-                         : launch_track_kernel<F, HALF, true, false, -1, true, true>(a, num_sms, st);
-        return m.out ? launch_track_kernel<F, HALF, true, true, -1, false, true>(a, num_sms, st)
-                     : launch_track_kernel<F, HALF, true, false, -1, false, true>(a, num_sms, st);
+            return m.out ? launch_track_kernel<F, HALF, true, true, -1, kVarAll, true>(a, num_sms, st)
+                         : launch_track_kernel<F, HALF, true, false, -1, kVarAll, true>(a, num_sms, st);
+        return m.out ? launch_track_kernel<F, HALF, true, true, -1, 0, true>(a, num_sms, st)
+                     : launch_track_kernel<F, HALF, true, false, -1, 0, true>(a, num_sms, st);
     }
-    if (m.var)
-        return m.out ? launch_track_kernel<F, HALF, true, true, -1, true, false>(a, num_sms, st)
-                     : launch_track_kernel<F, HALF, true, false, -1, true, false>(a, num_sms, st);
-    if (m.out) return launch_track_kernel<F, HALF, true, true, -1, false, false>(a, num_sms, st);
-    // the bench path: record layout as a compile-time constant
-    if (a.rb_log == 0) return launch_track_kernel<F, HALF, true, false, 0, false, false>(a, num_sms, st);
-    if (a.rb_log == kBrickLog) return launch_track_kernel<F, HALF, true, false, (int)kBrickLog, false, false>(a, num_sms, st);
+    if (m.var) {  // the compiled-in variants are exactly the requested ones (forced: all)
+        const int vm = (a.bidir ? kVarBidir : 0) | (a.interp ? kVarInterp : 0) | (a.init_mode ? kVarInit : 0);
+        switch (vm) {
+            case 1: return launch_track_var<F, HALF, 1>(a, m, num_sms, st);
+            case 2: return launch_track_var<F, HALF, 2>(a, m, num_sms, st);
+            case 3: return launch_track_var<F, HALF, 3>(a, m, num_sms, st);
+            case 4: return launch_track_var<F, HALF, 4>(a, m, num_sms, st);
+            case 5: return launch_track_var<F, HALF, 5>(a, m, num_sms, st);
+            case 6: return launch_track_var<F, HALF, 6>(a, m, num_sms, st);
+            default: return launch_track_var<F, HALF, kVarAll>(a, m, num_sms, st);  // 7, or PT_KERNEL_VARIANT alone
+        }
+    }
+    if (m.out) return launch_track_kernel<F, HALF, true, true, -1, 0, false>(a, num_sms, st);
+    if (a.sample_mode) return launch_track_kernel<F, HALF, true, false, -1, 0, false>(a, num_sms, st);
+    // the bench path: record layout as a compile-time constant, random sample per step
+    if (a.rb_log == 0) return launch_track_kernel<F, HALF, true, false, 0, 0, false>(a, num_sms, st);
+    if (a.rb_log == kBrickLog) return launch_track_kernel<F, HALF, true, false, (int)kBrickLog, 0, false>(a, num_sms, st);
     return cudaErrorInvalidValue;
 }
 
