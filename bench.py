@@ -754,8 +754,9 @@ def run_ours(args):
             "e2e_with_load": {"value": e2e_vals[True], "unit": "steps/s",
                               "h2d_bytes_per_step": int(seeds_h.numel() * 4 + ids_h.numel() * 8 + ls["h2d_bytes"]),
                               "d2h_bytes_per_step": int(map_h.numel() * 4)},
-            # per pt_track: seed_keys + cub radix sort (upsweep/scan/downsweep x passes), the
-            # tracking kernel, map_sum; counted from the ncu launch list (profiles/)
+            # per pt_track: seed_keys, cub radix sort (histogram, exclusive sum, 4 onesweep
+            # passes), the tracking kernel, map_sum -- the ncu launch list
+            # (profiles/r02b_c3_launches.md); the L2 flush is torch's fill kernel, not counted
             "gpu_launches": 9 * args.steps,
             "clocks": ck,
         }

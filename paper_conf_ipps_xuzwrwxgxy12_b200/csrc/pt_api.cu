@@ -54,8 +54,6 @@ struct pt_ctx {
     size_t temp_cap = 0;
     uint32_t* d_map = nullptr;   // internal map for host map pointers
     size_t map_cap = 0;
-    uint32_t* d_bmap = nullptr;    // the stepping kernel's map in record (bricked) order
-    size_t bmap_cap = 0;
     unsigned long long* d_utab = nullptr;  // NEXT-2 unique map: per-lane hash sets
     size_t utab_cap = 0;
     uint8_t* d_stage = nullptr;    // pt_load_samples: staging of host inputs (grow-only)
@@ -285,7 +283,7 @@ void pt_destroy(pt_ctx* c) {
     DeviceGuard g(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
     else cudaDeviceSynchronize();
-    void* bufs[] = {c->d_rec, c->d_mask, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_bmap, c->d_utab,
+    void* bufs[] = {c->d_rec, c->d_mask, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_utab,
                     c->d_stage, c->d_labels, c->d_conn, c->d_nsteps, c->d_reason, c->d_end, c->d_paths,
                     c->d_stats, c->d_mstats, c->d_mvox, c->d_mflags, c->d_mtemp, c->d_mcount, c->d_seg};
     for (void* b : bufs)
@@ -582,15 +580,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         a.group_chunks = N > tail ? (N - tail) / G : 0;
         a.total_chunks = a.group_chunks + (N - a.group_chunks * G);
     }
-    // the stepping kernel counts in record order (bricked); unbricked into d_map after it
-    const bool bricked_map = d_map && !segmented && c->layout.b != 0;
     a.map = d_map;
-    if (bricked_map) {
-        const size_t nb = (size_t)c->layout.nvox();
-        CK(ensure(c->d_bmap, c->bmap_cap, nb), "pt_track: bricked map");
-        CK(cudaMemsetAsync(c->d_bmap, 0, nb * sizeof(uint32_t), st), "pt_track: bricked map zero");
-        a.map = c->d_bmap;
-    }
     a.o_nsteps = (fl & PT_REC_LEN) ? c->d_nsteps : nullptr;
     a.o_reason = (fl & PT_REC_REASON) ? c->d_reason : nullptr;
     a.o_end = (fl & PT_REC_END) ? c->d_end : nullptr;
@@ -664,8 +654,6 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
            "pt_track: tracking kernel launch");
     }
     CK(cudaEventRecord(c->ev[2], st), "pt_track: event");
-    if (bricked_map)
-        CK(pt::launch_unbrick_add(c->d_bmap, nxv, nyv, nzv, c->layout, d_map, st), "pt_track: unbrick map");
     if (d_map) CK(pt::launch_map_sum(d_map, (int64_t)V, c->d_stats + pt::kStatMapAfter, st), "pt_track: map sum");
     if (host_map) {
         CK(cudaMemcpyAsync(map, d_map, V * sizeof(uint32_t), cudaMemcpyDeviceToHost, st), "pt_track: map D2H");

@@ -62,9 +62,7 @@ struct TrackArgs {
     uint32_t chunks_per_seed;    // ceil(P / cta_chunk)
     uint64_t total_chunks;       // nseeds * chunks_per_seed
     uint64_t max_seed_id;        // largest seed id whose pids fit 64 bits: (2^64-1 - (P-1)) / P
-    uint32_t* map;               // the map this launch adds into, or nullptr: indexed by record
-                                 // position (rec_vox; [V'] bricked) for the stepping kernel, by
-                                 // raster voxel for the segmented ablation
+    uint32_t* map;               // [V] raster map this launch adds into, or nullptr
     uint16_t* o_nsteps;          // [nparticles] or nullptr
     uint8_t* o_reason;
     float* o_end;                // [nparticles][3]
@@ -165,9 +163,6 @@ cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask,
 size_t seed_order_temp_bytes(uint64_t nseeds);
 cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint32_t* keys, uint32_t* keys_out,
                               uint32_t* idx, uint32_t* perm, void* temp, size_t temp_bytes, cudaStream_t st);
-// map[v] += bmap[rec_vox(v)] (the kernel's record-ordered counts into the caller's raster map)
-cudaError_t launch_unbrick_add(const uint32_t* bmap, int nx, int ny, int nz, const RecLayout& L, uint32_t* map,
-                               cudaStream_t st);
 cudaError_t launch_map_sum(const uint32_t* map, int64_t V, unsigned long long* out,
                            cudaStream_t st);
 cudaError_t launch_gather_bench(const uint8_t* buf, uint64_t nrec, int rec_bytes, uint32_t iters,

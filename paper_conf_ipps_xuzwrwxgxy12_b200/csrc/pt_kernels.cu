@@ -119,27 +119,6 @@ cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint32_t* key
     return cub::DeviceRadixSort::SortPairs(temp, temp_bytes, keys, keys_out, idx, perm, (int)nseeds, 0, 30, st);
 }
 
-// ------------------------------------------------------------------------- unbrick
-// map[v] += bmap[rec_vox(v)] for every raster voxel v: the tracking kernel counts visits in
-// record order (bricked), the caller's map is raster (one pass, 5 MB for c3)
-__global__ void unbrick_add_kernel(const uint32_t* __restrict__ bmap, int nx, int ny, int64_t V, RecLayout L,
-                                   uint32_t* __restrict__ map) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < V; i += (int64_t)gridDim.x * blockDim.x) {
-        const uint32_t rv = rec_vox_raster((uint32_t)i, (uint32_t)nx, (uint32_t)ny, L.b, L.nbx, L.nby);
-        map[i] += bmap[rv];
-    }
-}
-
-cudaError_t launch_unbrick_add(const uint32_t* bmap, int nx, int ny, int nz, const RecLayout& L, uint32_t* map,
-                               cudaStream_t st) {
-    const int64_t V = (int64_t)nx * ny * nz;
-    int64_t blocks = (V + 255) / 256;
-    if (blocks > 148 * 16) blocks = 148 * 16;
-    if (blocks < 1) blocks = 1;
-    unbrick_add_kernel<<<(unsigned)blocks, 256, 0, st>>>(bmap, nx, ny, V, L, map);
-    return cudaGetLastError();
-}
-
 // ------------------------------------------------------------------------- map sum
 __global__ void map_sum_kernel(const uint32_t* __restrict__ map, int64_t V, unsigned long long* out) {
     unsigned long long s = 0;

@@ -42,12 +42,6 @@
 #ifndef PT_RUNLEN
 #define PT_RUNLEN 1  // merge consecutive visits of a voxel before the RED (0: ablation iv, one RED per step)
 #endif
-#ifndef PT_MAP_TILE
-#define PT_MAP_TILE 0  // experiment: shared-memory count tile over the CTA's current seed brick
-#endif
-#ifndef PT_TILE_EVERY
-#define PT_TILE_EVERY 16  // rounds between the CTA-wide tile flushes / re-targets
-#endif
 #ifndef PT_REFILL_MIN
 #define PT_REFILL_MIN 2  // free lanes a warp waits for before refilling (amortises the refill block)
 #endif
@@ -77,12 +71,11 @@ struct Lane {
     bool pend;         // the round's last candidate step waits for the next round's gather
     float qx, qy, qz;  // committed position, centred coordinates (R10)
     float px, py, pz;  // direction of the last (candidate) step
-    uint32_t gvox;     // raster voxel of the round-start gather (RASTER instantiations only)
+    uint32_t gvox;     // raster voxel of the round-start gather (seed or pending candidate)
     uint32_t grv;      // its position in the record volume (rec_vox)
     int n;             // committed steps (of this half)
     uint64_t pid;      // global particle id = seed_id * P + j (RNG key, R16)
-    uint32_t run_vox, run_cnt;  // run-length merge of consecutive visits of the voxel whose
-                                // record position is run_vox (UNQ: the current voxel)
+    uint32_t run_vox, run_cnt;  // run-length merge of consecutive visits (UNQ: current voxel)
     uint32_t sfix;     // paper mode (NEXT-1): the particle's sample volume, j mod S
     int why;           // >= 0: ended with this reason, outputs pending (finish)
     uint4 W;           // Philox block of the current round (stream = half)
@@ -116,38 +109,17 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     __shared__ unsigned long long s_li[OUT ? TPB : 1];  // particle index (outputs)
     __shared__ uint32_t s_q[TPB / 32][3];               // per-warp sub-chunk
     __shared__ unsigned long long s_work;               // CTA claim + tickets
-    // PT_MAP_TILE: counts of the CTA's current seed brick (16^3 voxels), flushed and re-targeted
-    // every PT_TILE_EVERY rounds at a CTA-wide barrier
-    constexpr bool TILE = PT_MAP_TILE && REFILL && VM == 0 && !UNQ && BL != 0;
-    __shared__ uint32_t s_tile[TILE ? 4096 : 1];
-    __shared__ uint32_t s_tile_br, s_cur_seed;
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t wib = threadIdx.x >> 5;
     const uint32_t lt_mask = (1u << lane) - 1u;
-    // the map this launch adds into is indexed by record position (rec_vox: the bricked
-    // voxel order of the records; pt_track adds it into the caller's raster map afterwards),
-    // so a step needs no raster index unless it reads a raster per-voxel array: the mask
-    // byte of PT_INTERP or the target labels of the connectivity matrix
+    // the map is raster-ordered (a record-ordered map was measured 6 % slower)
     uint32_t* const map = a.map;
     const bool has_map = map != nullptr;
-    constexpr bool RASTER = VI || OUT;
     const uint32_t H = (VB && a.bidir) ? 2u : 1u;      // output entries per particle
     const bool interp = VI && a.interp;
     const uint32_t init_mode = VN ? a.init_mode : 0u;
     const bool smode = BL < 0 && a.sample_mode != 0u;  // paper mode (NEXT-1): s = j mod S
     if (threadIdx.x == 0) s_work = kNoChunk << 24;
-    if (TILE) {
-        for (int i = threadIdx.x; i < 4096; i += TPB) s_tile[i] = 0u;
-        if (threadIdx.x == 0) {
-            s_tile_br = 0xFFFFFFFFu;
-            s_cur_seed = 0xFFFFFFFFu;
-        }
-    }
-    // brick the tile covers (register copy, CTA-uniform; 0xFFFFFFFF: none, as brick ids are
-    // < 2^20); the tile is used only with a map and the 16^3-brick record layout
-    const bool tile_on = TILE && a.map != nullptr && a.rb_log == kBrickLog;
-    uint32_t tile_br = 0xFFFFFFFFu;
-    uint32_t trounds = 0;
     if (lane == 0) {
         s_q[wib][0] = 0u;
         s_q[wib][1] = 0u;
@@ -235,17 +207,8 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
             my_steps = 0u;
         }
     };
-    // a run of visits of one voxel: into the tile if the voxel lies in the tile's brick
-    // (record position >> 12 = brick, & 4095 = voxel in the brick), else a global RED
-    auto red_run = [&](bool p, uint32_t rv, uint32_t cnt) {
-        if (TILE) {
-            const bool in_tile = (rv >> 12) == tile_br;
-            if (p && in_tile) atomicAdd(&s_tile[rv & 4095u], cnt);
-            red_add_if(p && !in_tile, map + rv, cnt);
-        } else {
-            red_add_if(p, map + rv, cnt);
-        }
-    };
+    // a run of visits of one voxel: one predicated RED
+    auto red_run = [&](bool p, uint32_t vox, uint32_t cnt) { red_add_if(p, map + vox, cnt); };
     auto flush_run = [&]() {
         if (!UNQ && has_map) red_run(x.run_cnt != 0u, x.run_vox, x.run_cnt);
         x.run_cnt = 0u;
@@ -272,9 +235,8 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         // non-finite seeds are outside (a NaN would truncate into the volume)
         const bool fin = isfinite(x.qx) && isfinite(x.qy) && isfinite(x.qz);
         if (fin && (unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny && (unsigned)iz < (unsigned)a.nz) {
-            const uint32_t v = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
-            if (RASTER) x.gvox = v;
-            x.grv = recv(ix, iy, iz, v);
+            x.gvox = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
+            x.grv = recv(ix, iy, iz, x.gvox);
             return true;
         }
         return false;
@@ -328,8 +290,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
             particle_done();
         }
     };
-    // UNQ (R25): has the streamline entered the voxel at record position v before?  Inserts
-    // it if not.
+    // UNQ (R25): has the streamline entered voxel v before?  Inserts it if not.
     auto first_entry = [&](bool c, uint32_t v) -> bool {
         bool fresh = false;
         bool probe = c && v != x.run_vox && v != x.prev_vox;
@@ -353,27 +314,26 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     // commit a step (if c): new position, one visit of the new voxel (R13);
     // consecutive visits of the same voxel are merged (run length) and flushed with a
     // predicated RED when the voxel changes.  Straight-line except for the UNQ probe.
-    // v: raster voxel (RASTER instantiations), vrv: its record position (the map index)
-    auto commit_if = [&](bool c, float nx_, float ny_, float nz_, uint32_t v, uint32_t vrv) {
+    auto commit_if = [&](bool c, float nx_, float ny_, float nz_, uint32_t v) {
         x.qx = c ? nx_ : x.qx;
         x.qy = c ? ny_ : x.qy;
         x.qz = c ? nz_ : x.qz;
         x.n += c ? 1 : 0;
         if (UNQ) {
-            const bool fresh = first_entry(c, vrv);
-            red_add_if(has_map && fresh, map + vrv, 1u);
+            const bool fresh = first_entry(c, v);
+            red_add_if(has_map && fresh, map + v, 1u);
             my_unique += fresh ? 1u : 0u;
-            const bool change = c && vrv != x.run_vox;
+            const bool change = c && v != x.run_vox;
             x.prev_vox = change ? x.run_vox : x.prev_vox;
-            x.run_vox = c ? vrv : x.run_vox;
+            x.run_vox = c ? v : x.run_vox;
         } else if (has_map) {
 #if PT_RUNLEN
-            const bool change = vrv != x.run_vox;
+            const bool change = v != x.run_vox;
             red_run(c && change && x.run_cnt != 0u, x.run_vox, x.run_cnt);
             x.run_cnt = c ? (change ? 1u : x.run_cnt + 1u) : x.run_cnt;
-            x.run_vox = c ? vrv : x.run_vox;
+            x.run_vox = c ? v : x.run_vox;
 #else
-            red_add_if(c, map + vrv, 1u);  // ablation (iv): one global RED per committed step
+            red_add_if(c, map + v, 1u);  // ablation (iv): one global RED per committed step
 #endif
         }
         if (OUT && a.conn && c) {  // NEXT-2: targets entered by committed steps (R21)
@@ -500,7 +460,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         const float nqz = __fadd_rn(x.qz, __fmul_rn(a.step, dz));
         const int ix = axis_index(nqx, a.cx), iy = axis_index(nqy, a.cy), iz = axis_index(nqz, a.cz);
         const bool inb = (unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny && (unsigned)iz < (unsigned)a.nz;
-        const uint32_t v = RASTER ? ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix : 0u;
+        const uint32_t v = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
         // stop criteria in order: maximum steps (R14), angle, volume (R11)
         const bool maxed = x.n == a.max_steps;
         const bool go = x.alive && !maxed && curv_ok && inb;
@@ -517,14 +477,13 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
             }
             const uint32_t w = ((k + 1) % 3 == 0) ? x.W.x : ((k + 1) % 3 == 1) ? x.W.y : x.W.z;
             const uint32_t sk = smode ? x.sfix : sample_of(w, a.S);
-            const uint32_t vrv = recv(ix, iy, iz, v);
-            const bool outside = gather(go, nqx, nqy, nqz, vrv, v, (uint32_t)x.n + 1u, sk);
+            const bool outside = gather(go, nqx, nqy, nqz, recv(ix, iy, iz, v), v, (uint32_t)x.n + 1u, sk);
             x.why = outside ? kEndMask : x.why;
             x.alive = go && !outside;
-            commit_if(x.alive, nqx, nqy, nqz, v, vrv);
+            commit_if(x.alive, nqx, nqy, nqz, v);
         } else {
             x.pend = go;  // next round's start gathers and tests it
-            if (RASTER) x.gvox = go ? v : x.gvox;
+            x.gvox = go ? v : x.gvox;
             x.grv = go ? recv(ix, iy, iz, v) : x.grv;
         }
     };
@@ -565,7 +524,6 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
                     const uint32_t avail = cend - cnext;
                     const uint32_t rank = __popc(need & lt_mask);
                     if (!x.alive && rank < avail) start(cseed, (uint64_t)(cnext + rank));
-                    if (TILE && lane == 0) s_cur_seed = cseed;
                     const uint32_t cnt = (uint32_t)__popc(need);
                     cnext += cnt < avail ? cnt : avail;
                     need = __ballot_sync(kFull, !x.alive);
@@ -579,40 +537,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
                 __syncwarp();
             }
         }
-        const bool warp_alive = __any_sync(kFull, x.alive);
-        if (TILE) {
-            // every PT_TILE_EVERY iterations all warps of the CTA meet (warps without work
-            // run empty iterations): flush the tile, re-target it at the brick of the seed
-            // the CTA claimed last, or leave when the CTA has nothing left
-            if (++trounds % PT_TILE_EVERY == 0u) {
-                const bool cont = __syncthreads_or(x.alive || !exhausted);
-                if (tile_br != 0xFFFFFFFFu) {
-                    uint32_t* const mb = map + ((size_t)tile_br << 12);  // the brick, contiguous
-                    for (uint32_t i = threadIdx.x; i < 4096u; i += TPB) {
-                        const uint32_t c = s_tile[i];
-                        if (c != 0u) atomicAdd(mb + i, c);
-                        s_tile[i] = 0u;
-                    }
-                }
-                if (threadIdx.x == 0) {
-                    uint32_t br = 0xFFFFFFFFu;
-                    const uint32_t sd = s_cur_seed;
-                    if (tile_on && sd != 0xFFFFFFFFu) {
-                        const float sx = a.seeds[3 * sd], sy = a.seeds[3 * sd + 1], sz = a.seeds[3 * sd + 2];
-                        if (sx >= 0.f && sy >= 0.f && sz >= 0.f && sx < (float)a.nx && sy < (float)a.ny &&
-                            sz < (float)a.nz)
-                            br = (((uint32_t)sz >> 4) * a.rb_nby + ((uint32_t)sy >> 4)) * a.rb_nbx + ((uint32_t)sx >> 4);
-                    }
-                    s_tile_br = br;
-                }
-                __syncthreads();
-                tile_br = s_tile_br;
-                if (!cont) break;
-            }
-            if (!warp_alive) continue;
-        } else if (!warp_alive) {
-            break;
-        }
+        if (!__any_sync(kFull, x.alive)) break;
         rounds += 1u;
 
         // ------------------------------------------------ round start: one Philox block,
@@ -631,7 +556,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
             const bool outside = gather(x.alive, cqx, cqy, cqz, x.grv, x.gvox, t0, s0);
             x.why = outside ? kEndMask : x.why;
             x.alive = x.alive && !outside;
-            commit_if(x.pend && !outside, cqx, cqy, cqz, x.gvox, x.grv);
+            commit_if(x.pend && !outside, cqx, cqy, cqz, x.gvox);
             // R24: the first step of half 0 takes the drawn fibre: move it to slot 0 of the
             // record (the first step uses only the chosen fibre's vector)
             if (VN && F > 1 && init_mode != 0u) {

@@ -28,6 +28,13 @@ KEYS = [
     ("lts__t_sector_hit_rate.pct", "L2 sector hit rate"),
     ("lts__t_sectors_srcunit_tex_op_read.sum", "L2 read sectors (from L1/tex)"),
     ("lts__t_sectors_srcunit_tex_op_red.sum", "L2 reduction sectors (map RED)"),
+    ("lts__t_sectors_srcunit_tex_op_read_lookup_hit.sum", "L2 read sectors that hit"),
+    ("lts__t_sectors_srcunit_tex_op_red_lookup_miss.sum", "L2 RED sectors that missed"),
+    ("lts__t_requests_srcunit_tex_op_read.sum", "L2 read requests (from L1/tex)"),
+    ("l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum", "L1 global load sectors requested"),
+    ("l1tex__t_sectors_pipe_lsu_mem_global_op_ld_lookup_hit.sum", "L1 global load sectors that hit"),
+    ("l1tex__m_xbar2l1tex_read_sectors_mem_lg_op_ld.sum", "sectors L2 -> L1 (global loads)"),
+    ("dram__sectors_read.sum", "DRAM sectors read"),
     ("lts__throughput.avg.pct_of_peak_sustained_elapsed", "L2 throughput % of peak"),
     ("l1tex__t_sector_hit_rate.pct", "L1 sector hit rate"),
     ("l1tex__throughput.avg.pct_of_peak_sustained_elapsed", "L1 throughput % of peak"),
