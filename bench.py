@@ -213,10 +213,10 @@ def _cpu_sample(w, target_s: float, threads: int):
     return sub, P, every
 
 
-def _run_oracle_sample(sub, J, threads, keep=False):
+def _run_oracle_sample(sub, J, threads, keep=False, unique=False):
     import oracle
     t = time.perf_counter()
-    r = oracle.track(sub, 0, J, want_map=True, threads=threads)
+    r = oracle.track(sub, 0, J, want_map=True, threads=threads, want_unique=unique)
     dt = time.perf_counter() - t
     if keep:
         return int(r["nsteps"].sum()), dt, r
@@ -476,6 +476,12 @@ def run_ours(args):
     if args.seed_every > 1:
         import phantom
         w = phantom.wm_seeds(w, every=args.seed_every)
+    # NEXT-3 variants requested through --track-flags: the workload (and so the oracle of the
+    # cpu_baseline / parity leg) carries the same semantics
+    tf = args.track_flags
+    w = w.replace(bidir=int(bool(tf & pt.PT_BIDIR)), interp=int(bool(tf & pt.PT_INTERP)),
+                  init_fibre=1 if tf & pt.PT_INIT_RANDOM else (2 if tf & pt.PT_INIT_FWEIGHT else 0))
+    unique = bool(tf & pt.PT_MAP_UNIQUE)
     mine = _shard(w, rank, world)
     tr = pt.Tracker(local)
     # load through the C ABI from pinned host memory: the paper's Copy3DImagesToGPU (P:L165,
@@ -604,15 +610,15 @@ def run_ours(args):
     # ---- roofline (dominant kernel = the tracking kernel)
     kms = sum(kern_ms) / len(kern_ms)
     # SURVEY §8(d) algorithmic bytes per committed step: one record read + one 4-B map
-    # atomic (read-modify-write: 8 B); per particle 12 B of seed + 8 B of id, amortised
-    alg_bytes = my_steps * (rb + 8) + mine.nseeds * (12 + 8)
+    # atomic (counted as its 4 B, as §8(d) lists it); per seed 12 B of seed + 8 B of id
+    alg_bytes = my_steps * (rb + 4) + mine.nseeds * (12 + 8)
     achieved = alg_bytes / (kms * 1e-3) / 1e9
     peaks = _peaks()
     peak = peaks["hbm_gbs"] if peaks else 6650.0
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": achieved / peak, "traffic": _ncu_traffic(args.config),
             "peak_source": "measured (MEASURED_PEAKS.json hbm_gbs)" if peaks else "fallback 6.65 TB/s",
-            "bytes_per_step": rb + 8, "kernel_ms": kms,
+            "bytes_per_step": rb + 4, "kernel_ms": kms,
             "kernel_ms_steps": kern_ms, "track_ms_steps": track_ms}
     gather = None
     if rank == 0 and not args.no_gather_bench:
@@ -635,7 +641,7 @@ def run_ours(args):
         oracle.build()
         threads = len(os.sched_getaffinity(0))
         sub, J, every = _cpu_sample(w, args.cpu_seconds, threads)
-        s, dt, r = _run_oracle_sample(sub, J, threads, keep=True)
+        s, dt, r = _run_oracle_sample(sub, J, threads, keep=True, unique=unique)
         cpu = {"value": s / dt, "unit": "steps/s", "cores": threads, "kind": "oracle", "cpu_model": _cpu_model(),
                "sample": f"every {every}th WM seed ({sub.nseeds} seeds) x all {J} particles: "
                          f"{s} steps in {dt:.1f} s"}
@@ -647,16 +653,17 @@ def run_ours(args):
             gm = tr.track(sd, si, flags=base_flags, **tparams)
             torch.cuda.synchronize()
             gmap = gm.cpu().numpy().view(np.uint32).astype(np.uint64)
+            rmap = r["umap"] if unique else r["map"]  # PT_MAP_UNIQUE: streamlines per voxel (R25)
             rec = pt.PT_REC_LEN | pt.PT_REC_REASON | pt.PT_REC_END
             tr.track(sd, si, flags=base_flags | rec, want_map=False, **tparams)
             torch.cuda.synchronize()
             g = tr.get_paths()
             div = ((g["nsteps"].astype(np.int64) != r["nsteps"]) | (g["reason"] != r["reason"]) |
                    np.any(g["end"].view(np.uint32) != r["end"].view(np.uint32), axis=1))
-            l1 = float(np.abs(gmap.astype(np.int64) - r["map"].astype(np.int64)).sum()) / max(1, int(r["map"].sum()))
+            l1 = float(np.abs(gmap.astype(np.int64) - rmap.astype(np.int64)).sum()) / max(1, int(rmap.sum()))
             parity = {"sample": cpu["sample"], "streamlines": int(div.size), "divergent": int(div.sum()),
                       "divergent_fraction": float(div.mean()), "map_l1_rel": l1,
-                      "map_bit_exact": bool(np.array_equal(gmap, r["map"])),
+                      "map_bit_exact": bool(np.array_equal(gmap, rmap)),
                       "kernel": "map: the timed launch (flags as benched); per-streamline: the outputs instantiation",
                       "bar": "divergent <= 1e-4, map L1 rel <= 1e-4 (north_star); expected 0 / 0"}
 

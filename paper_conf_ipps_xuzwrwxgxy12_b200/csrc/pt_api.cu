@@ -25,6 +25,9 @@
 #ifndef PT_TAIL_SEEDS_PER_SM
 #define PT_TAIL_SEEDS_PER_SM 4  // single-seed claims at the end of the queue, per SM
 #endif
+#ifndef PT_L2_FETCH_DEFAULT
+#define PT_L2_FETCH_DEFAULT 0  // experiment: cudaLimitMaxL2FetchGranularity set by pt_create (0: leave)
+#endif
 #ifndef PT_BRICK_DEFAULT
 #define PT_BRICK_DEFAULT 4  // record layout brick log2 edge (0 = raster, 4 = 16^3 bricks, measured best)
 #endif
@@ -247,6 +250,13 @@ pt_status pt_create(int cuda_device, pt_ctx** out) {
         return fail(nullptr, PT_ERR_CUDA, "pt_create: %s", cudaGetErrorString(e));
     }
     c->num_sms = prop.multiProcessorCount;
+    {
+        // L2 fetch granularity for the random 32-B record gathers (env PT_L2_FETCH overrides)
+        int gran = PT_L2_FETCH_DEFAULT;
+        if (const char* ev = getenv("PT_L2_FETCH")) gran = atoi(ev);
+        if (gran > 0) cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)gran);
+        cudaGetLastError();
+    }
     for (auto& ev : c->mev) {
         if (cudaEventCreate(&ev) != cudaSuccess) {
             cudaGetLastError();

@@ -90,6 +90,9 @@ struct Lane {
     // UNQ (R25)
     uint32_t gen;      // generation tag of the streamline in the lane's hash set
     uint32_t prev_vox; // the voxel entered before run_vox (recent-voxel filter)
+    bool upend;        // a probe of the hash set is in flight for voxel ukey ...
+    uint32_t ukey, uh; // ... at slot uh,
+    unsigned long long ue;  // whose entry the in-flight load returns
 };
 
 // CTA size: one CTA per SM; the variant / unique instantiations keep more state per lane
@@ -152,6 +155,9 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     x.winit = 0u;
     x.gen = 0u;
     x.prev_vox = 0xFFFFFFFFu;
+    x.upend = false;
+    x.ukey = x.uh = 0u;
+    x.ue = 0ull;
 #pragma unroll
     for (int k = 0; k < R::kWords; ++k) x.rv.w[k] = 0u;
 
@@ -213,6 +219,44 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         if (!UNQ && has_map) red_run(x.run_cnt != 0u, x.run_vox, x.run_cnt);
         x.run_cnt = 0u;
     };
+    // UNQ (R25): has the streamline entered voxel v before?  The lane's hash set answers;
+    // the first probe of a voxel entry is only ISSUED when the voxel is entered (its load
+    // is in flight while the next step computes and gathers) and RESOLVED at the lane's
+    // next voxel entry, or when the half ends -- always before the next probe is issued,
+    // so the set seen by every probe is exact.  Collisions continue synchronously.
+    auto unq_resolve = [&]() {
+        bool fresh = false;
+        bool open = x.upend;
+        unsigned long long e = x.ue;
+        uint32_t h = x.uh;
+        const uint32_t mask = (1u << a.ulog) - 1u;
+        while (open) {
+            if ((uint32_t)(e >> 32) != x.gen) {  // empty or a stale streamline's entry
+                utab[h] = ((unsigned long long)x.gen << 32) | x.ukey;
+                fresh = true;
+                open = false;
+            } else if ((uint32_t)e == x.ukey) {
+                open = false;
+            } else {
+                h = (h + 1u) & mask;
+                e = utab[h];
+            }
+        }
+        x.upend = false;
+        red_add_if(has_map && fresh, map + x.ukey, 1u);
+        my_unique += fresh ? 1u : 0u;
+    };
+    auto unq_issue = [&](bool c, uint32_t v) {
+        // the current and the previous voxel are known to be in the set (recent-voxel filter)
+        const bool probe = c && v != x.run_vox && v != x.prev_vox;
+        if (probe) {
+            unq_resolve();
+            x.ukey = v;
+            x.uh = (v * 0x9E3779B1u) >> (32u - a.ulog);
+            x.ue = utab[x.uh];
+            x.upend = true;
+        }
+    };
     // begin half h of the current particle at its seed: centred position, seed voxel.
     // Returns false if the seed is outside the volume (R12).
     auto begin = [&](uint32_t h) -> bool {
@@ -244,6 +288,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     // a half that ended: outputs; a bidirectional half 0 restarts as half 1 in this lane (R22)
     auto finish = [&]() {
         flush_run();
+        if (UNQ) unq_resolve();  // the half's last voxel entry
         write_outputs(x.n, x.why, x.qx, x.qy, x.qz);
         x.why = -1;
         if (VB && H == 2u && x.half == 0u) {
@@ -290,27 +335,6 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
             particle_done();
         }
     };
-    // UNQ (R25): has the streamline entered voxel v before?  Inserts it if not.
-    auto first_entry = [&](bool c, uint32_t v) -> bool {
-        bool fresh = false;
-        bool probe = c && v != x.run_vox && v != x.prev_vox;
-        const unsigned long long key = ((unsigned long long)x.gen << 32) | v;
-        const uint32_t mask = (1u << a.ulog) - 1u;
-        uint32_t h = (v * 0x9E3779B1u) >> (32u - a.ulog);
-        while (probe) {
-            const unsigned long long e = utab[h];
-            if ((uint32_t)(e >> 32) != x.gen) {  // empty or a stale streamline's entry
-                utab[h] = key;
-                fresh = true;
-                probe = false;
-            } else if ((uint32_t)e == v) {
-                probe = false;
-            } else {
-                h = (h + 1u) & mask;
-            }
-        }
-        return fresh;
-    };
     // commit a step (if c): new position, one visit of the new voxel (R13);
     // consecutive visits of the same voxel are merged (run length) and flushed with a
     // predicated RED when the voxel changes.  Straight-line except for the UNQ probe.
@@ -320,9 +344,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         x.qz = c ? nz_ : x.qz;
         x.n += c ? 1 : 0;
         if (UNQ) {
-            const bool fresh = first_entry(c, v);
-            red_add_if(has_map && fresh, map + v, 1u);
-            my_unique += fresh ? 1u : 0u;
+            unq_issue(c, v);
             const bool change = c && v != x.run_vox;
             x.prev_vox = change ? x.run_vox : x.prev_vox;
             x.run_vox = c ? v : x.run_vox;
