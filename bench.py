@@ -167,14 +167,16 @@ def _peaks():
         return None
 
 
-def _ncu_traffic(cfg):
-    """dram bytes per launch of the tracking kernel from the committed ncu --set full
-    summary (profiles/), or None."""
+def _ncu_traffic(cfg, steps):
+    """DRAM bytes (read + write) per launch of the tracking kernel from the committed ncu
+    --set full capture (profiles/ncu_track_summary.json): bytes per committed step of that
+    capture x this launch's steps (a capture may cover a seed subset, e.g. c5), or None."""
     p = os.path.join(ROOT, "profiles", "ncu_track_summary.json")
     try:
         d = json.load(open(p))
         e = d.get("per_config", {}).get(cfg) or {}
-        return e.get("dram_bytes_per_launch")
+        b = e.get("dram_bytes_per_step")
+        return None if b is None else b * steps
     except (OSError, ValueError):
         return None
 
@@ -592,9 +594,10 @@ def run_ours(args):
             if rank == 0:
                 map_h.copy_(mt)
 
-    e2e_step(False)  # warm
-    e2e_vals = {}
-    for with_load in (False, True):
+    e2e_vals = {False: None, True: None}
+    if not args.no_e2e:
+        e2e_step(False)  # warm
+    for with_load in (() if args.no_e2e else (False, True)):
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
@@ -616,7 +619,8 @@ def run_ours(args):
     peaks = _peaks()
     peak = peaks["hbm_gbs"] if peaks else 6650.0
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-            "frac": achieved / peak, "traffic": _ncu_traffic(args.config),
+            "frac": achieved / peak,
+            "traffic": _ncu_traffic(args.config, my_steps) if not args.track_flags else None,
             "peak_source": "measured (MEASURED_PEAKS.json hbm_gbs)" if peaks else "fallback 6.65 TB/s",
             "bytes_per_step": rb + 4, "kernel_ms": kms,
             "kernel_ms_steps": kern_ms, "track_ms_steps": track_ms}
@@ -812,6 +816,7 @@ def main(argv=None):
                     help="skip the streamline-length statistics (untimed extra pass with PT_REC_LEN)")
     ap.add_argument("--no-parity", action="store_true",
                     help="skip the GPU run of the cpu_baseline sample (the parity report)")
+    ap.add_argument("--no-e2e", action="store_true", help="experiments: skip the e2e legs")
     ap.add_argument("--dump-map", default="", help="rank 0 saves the (reduced) map of the last step (.npy)")
     ap.add_argument("--tag", default="", help="free-form label echoed by experiment scripts")
     ap.add_argument("--seed-every", type=int, default=1,

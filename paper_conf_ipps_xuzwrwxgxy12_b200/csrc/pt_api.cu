@@ -25,9 +25,6 @@
 #ifndef PT_TAIL_SEEDS_PER_SM
 #define PT_TAIL_SEEDS_PER_SM 4  // single-seed claims at the end of the queue, per SM
 #endif
-#ifndef PT_L2_FETCH_DEFAULT
-#define PT_L2_FETCH_DEFAULT 0  // experiment: cudaLimitMaxL2FetchGranularity set by pt_create (0: leave)
-#endif
 #ifndef PT_BRICK_DEFAULT
 #define PT_BRICK_DEFAULT 4  // record layout brick log2 edge (0 = raster, 4 = 16^3 bricks, measured best)
 #endif
@@ -250,13 +247,6 @@ pt_status pt_create(int cuda_device, pt_ctx** out) {
         return fail(nullptr, PT_ERR_CUDA, "pt_create: %s", cudaGetErrorString(e));
     }
     c->num_sms = prop.multiProcessorCount;
-    {
-        // L2 fetch granularity for the random 32-B record gathers (env PT_L2_FETCH overrides)
-        int gran = PT_L2_FETCH_DEFAULT;
-        if (const char* ev = getenv("PT_L2_FETCH")) gran = atoi(ev);
-        if (gran > 0) cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)gran);
-        cudaGetLastError();
-    }
     for (auto& ev : c->mev) {
         if (cudaEventCreate(&ev) != cudaSuccess) {
             cudaGetLastError();
@@ -573,15 +563,22 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         ch = (ch + pt::kSub - 1) / pt::kSub * pt::kSub;
         if (ch < pt::kMinCtaChunk) ch = pt::kMinCtaChunk;
         if (ch > P32) ch = P32;
+        if (const char* e = getenv("PT_CTA_CHUNK")) {  // experiments: particles per CTA claim
+            const uint64_t v = (uint64_t)atoll(e);
+            if (v >= pt::kSub) ch = (v + pt::kSub - 1) / pt::kSub * pt::kSub;
+        }
+        if (ch > P32) ch = P32;
         if (ch > (1ull << 27)) ch = 1ull << 27;  // keeps tickets per chunk < 2^22 (cta_take)
         a.cta_chunk = (uint32_t)ch;
     }
     a.chunks_per_seed = (uint32_t)((P + a.cta_chunk - 1) / a.cta_chunk);
     a.total_chunks = N * (uint64_t)a.chunks_per_seed;
     a.seeds_per_claim = 1;
-    if (a.chunks_per_seed == 1 && PT_SEEDS_PER_CLAIM > 1) {
+    uint64_t spc = PT_SEEDS_PER_CLAIM;
+    if (const char* e = getenv("PT_SEEDS_PER_CLAIM")) spc = (uint64_t)atoll(e);  // experiments
+    if (a.chunks_per_seed == 1 && spc > 1) {
         // whole seeds per claim: G consecutive seeds (tickets per claim must stay < 2^22)
-        uint64_t G = PT_SEEDS_PER_CLAIM;
+        uint64_t G = spc;
         const uint64_t sps = (P + pt::kSub - 1) / pt::kSub;
         while (G > 1 && (G * sps >= (1ull << 22) || N / G < 8ull * (uint64_t)c->num_sms)) G >>= 1;
         // the last PT_TAIL_SEEDS_PER_SM x SMs seeds are claimed one by one (guided tail)

@@ -3,8 +3,9 @@
 #   scripts/gpu.sh test [pytest -k expr]     GPU suite (+ smoke) -> gpurun_out/${TAG}_pytest_gpu.log
 #   scripts/gpu.sh bench CFG [bench args]    one bench.py line   -> gpurun_out/${TAG}_bench_${CFG}.json
 #   scripts/gpu.sh ab "LIBS" "CFGS" REPS     interleaved same-box A/B of experiment builds
-#                                            (LIBS: default or names of scripts/libpt_<name>.so,
-#                                            built here with scripts/build_variant.py)
+#                                            (LIBS: default, names of scripts/libpt_<name>.so
+#                                            built with scripts/build_variant.py, or
+#                                            env:VAR=v,VAR2=w = the default build under that env)
 #   scripts/gpu.sh ncu CFG [KREGEX] [args]   launch list (gpu__time_duration) + one --set full capture
 # TAG (env, default r02) prefixes every output file.
 set -u
@@ -25,9 +26,12 @@ bench)
 ab)
     LIBS=$1; CFGS=$2; REPS=${3:-2}; shift 3 || true
     for rep in $(seq $REPS); do for lib in $LIBS; do for cfg in $CFGS; do
-        if [ "$lib" = default ]; then L=$PWD/paper_conf_ipps_xuzwrwxgxy12_b200/libpt.so; else L=$PWD/scripts/libpt_$lib.so; fi
-        PT_LIB=$L timeout 600 python bench.py --config $cfg --steps 3 --warmup 3 --no-cpu-baseline --no-gather-bench \
-            --no-parity --no-lengths "$@" 2>/dev/null | tail -1 | python -c "
+        ENVS=""
+        if [ "$lib" = default ]; then L=$PWD/paper_conf_ipps_xuzwrwxgxy12_b200/libpt.so
+        elif [[ "$lib" == env:* ]]; then L=$PWD/paper_conf_ipps_xuzwrwxgxy12_b200/libpt.so; ENVS=${lib#env:}; ENVS=${ENVS//,/ }
+        else L=$PWD/scripts/libpt_$lib.so; fi
+        env $ENVS PT_LIB=$L timeout 900 python bench.py --config $cfg --steps 3 --warmup 3 --no-cpu-baseline --no-gather-bench \
+            --no-parity --no-lengths --no-e2e "$@" 2>/dev/null | tail -1 | python -c "
 import json, sys
 d = json.loads(sys.stdin.read())
 print('$lib', '$cfg', round(d['value'] / 1e9, 2), 'G steps/s', round(d['roofline']['kernel_ms'], 2), 'ms',
