@@ -1,8 +1,6 @@
 # The command list of the current gpurun session (overwritten per session; earlier ones are
-# in git history).  r02g: claim granularity on the DRAM-bound c5 (and c3): whole seeds in
-# groups of 32 (default) vs one seed per claim vs seeds split over several CTAs (chunks of
-# 2048 / 1024 particles) -- fewer seeds in flight chip-wide = a smaller L2 working set.
+# in git history).  r02h: c5 seeds-per-claim sweep (whole seeds per CTA claim: 1, 4, 8, 32),
+# interleaved x2 (r02g: 1 seed per claim 94.4 G vs 88.6 G default, but at different clocks).
 set -x
-export TAG=r02g
-scripts/gpu.sh ab "default env:PT_SEEDS_PER_CLAIM=1 env:PT_CTA_CHUNK=2048 env:PT_CTA_CHUNK=1024" "c5" 1
-scripts/gpu.sh ab "default env:PT_SEEDS_PER_CLAIM=1 env:PT_CTA_CHUNK=2048 env:PT_CTA_CHUNK=1024" "c3 c4" 1
+export TAG=r02h
+scripts/gpu.sh ab "env:PT_SEEDS_PER_CLAIM=1 env:PT_SEEDS_PER_CLAIM=4 env:PT_SEEDS_PER_CLAIM=8 default" "c5" 2
