@@ -17,10 +17,19 @@
 #include "pt_internal.h"
 
 #ifndef PT_SEEDS_PER_CLAIM
-// Whole seeds per CTA claim when every seed fits one claim: a CTA walks 32 consecutive
+// Whole seeds per CTA claim when every seed fits one claim: a CTA walks G consecutive
 // (Morton-adjacent) seeds, so its L1 keeps serving the shared tract voxels (sweep 1..64:
-// c3 74.6/75.3/76.0/76.4/77.0/77.2/76.9 G steps/s; 32 is the default).
+// c3 74.6/75.3/76.0/76.4/77.0/77.2/76.9 G steps/s; G = 32 for c3 / c4).  With a record volume
+// far beyond L2 (c5: 7.2 GB) the chip-wide span of in-flight seeds (#SMs x G) decides the
+// L2 working set instead: G = 1 / 4 / 8 / 32 give c5 94.3 / 96.8 / 94.8 / 88.5 G
+// (profiles/r02h_c5_claims_ab.log), so above PT_BIG_VOLUME bytes of records G is 4.
 #define PT_SEEDS_PER_CLAIM 32
+#endif
+#ifndef PT_SEEDS_PER_CLAIM_BIG
+#define PT_SEEDS_PER_CLAIM_BIG 4
+#endif
+#ifndef PT_BIG_VOLUME
+#define PT_BIG_VOLUME (4ull << 30)
 #endif
 #ifndef PT_TAIL_SEEDS_PER_SM
 #define PT_TAIL_SEEDS_PER_SM 4  // single-seed claims at the end of the queue, per SM
@@ -574,7 +583,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.chunks_per_seed = (uint32_t)((P + a.cta_chunk - 1) / a.cta_chunk);
     a.total_chunks = N * (uint64_t)a.chunks_per_seed;
     a.seeds_per_claim = 1;
-    uint64_t spc = PT_SEEDS_PER_CLAIM;
+    uint64_t spc = c->rec_size > PT_BIG_VOLUME ? PT_SEEDS_PER_CLAIM_BIG : PT_SEEDS_PER_CLAIM;
     if (const char* e = getenv("PT_SEEDS_PER_CLAIM")) spc = (uint64_t)atoll(e);  // experiments
     if (a.chunks_per_seed == 1 && spc > 1) {
         // whole seeds per claim: G consecutive seeds (tickets per claim must stay < 2^22)
@@ -629,6 +638,19 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         a.max_ctas = ctas;
     }
 
+    // experiment (env PT_MAP_PERSIST=1): the map as a persisting L2 access-policy window
+    const bool persist = d_map && getenv("PT_MAP_PERSIST") && atoi(getenv("PT_MAP_PERSIST")) > 0;
+    if (persist) {
+        cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)V * sizeof(uint32_t));
+        cudaStreamAttrValue av{};
+        av.accessPolicyWindow.base_ptr = d_map;
+        av.accessPolicyWindow.num_bytes = (size_t)V * sizeof(uint32_t);
+        av.accessPolicyWindow.hitRatio = 1.0f;
+        av.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        av.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &av);
+        cudaGetLastError();
+    }
     CK(cudaEventRecord(c->ev[1], st), "pt_track: event");
     if (segmented) {
         const uint32_t batch = (uint32_t)(npart < (1ull << 26) ? (npart ? npart : 1) : (1ull << 26));
@@ -661,6 +683,13 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
            "pt_track: tracking kernel launch");
     }
     CK(cudaEventRecord(c->ev[2], st), "pt_track: event");
+    if (persist) {
+        cudaStreamAttrValue av{};
+        av.accessPolicyWindow.num_bytes = 0;
+        cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &av);
+        cudaCtxResetPersistingL2Cache();
+        cudaGetLastError();
+    }
     if (d_map) CK(pt::launch_map_sum(d_map, (int64_t)V, c->d_stats + pt::kStatMapAfter, st), "pt_track: map sum");
     if (host_map) {
         CK(cudaMemcpyAsync(map, d_map, V * sizeof(uint32_t), cudaMemcpyDeviceToHost, st), "pt_track: map D2H");

@@ -142,9 +142,18 @@ __device__ __forceinline__ void ldg_record_if<64>(bool p, const void* ptr, uint3
     ldg_record_if<32>(p, static_cast<const char*>(ptr) + 32, w + 8);
 }
 
+#ifndef PT_RED_EVICT_LAST
+#define PT_RED_EVICT_LAST 0  // experiment: map REDs with an L2 evict_last cache policy
+#endif
 __device__ __forceinline__ void red_add_if(bool p, uint32_t* addr, uint32_t v) {
+#if PT_RED_EVICT_LAST
+    asm volatile("{\n\t.reg .pred q;\n\t.reg .b64 pol;\n\tcreatepolicy.fractional.L2::evict_last.b64 pol, 1.0;\n\t"
+                 "setp.ne.b32 q, %2, 0;\n\t@q red.global.add.L2::cache_hint.u32 [%0], %1, pol;\n\t}"
+                 :: "l"(addr), "r"(v), "r"((int)p) : "memory");
+#else
     asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q red.global.add.u32 [%0], %1;\n\t}"
                  :: "l"(addr), "r"(v), "r"((int)p) : "memory");
+#endif
 }
 
 // ---------------------------------------------------------------------------- lookup (R10)

@@ -1,6 +1,8 @@
 # The command list of the current gpurun session (overwritten per session; earlier ones are
-# in git history).  r02h: c5 seeds-per-claim sweep (whole seeds per CTA claim: 1, 4, 8, 32),
-# interleaved x2 (r02g: 1 seed per claim 94.4 G vs 88.6 G default, but at different clocks).
+# in git history).  r02i: keep the map in L2 -- map REDs with an L2 evict_last policy (redel)
+# and the map as a persisting access-policy window (env PT_MAP_PERSIST) vs the default, on
+# c3 / c4 and c5 (c5 now claims 4 seeds at a time: record volume > 4 GB).
 set -x
-export TAG=r02h
-scripts/gpu.sh ab "env:PT_SEEDS_PER_CLAIM=1 env:PT_SEEDS_PER_CLAIM=4 env:PT_SEEDS_PER_CLAIM=8 default" "c5" 2
+export TAG=r02i
+scripts/gpu.sh ab "default redel env:PT_MAP_PERSIST=1" "c3 c4" 2
+scripts/gpu.sh ab "default redel env:PT_MAP_PERSIST=1" "c5" 1
