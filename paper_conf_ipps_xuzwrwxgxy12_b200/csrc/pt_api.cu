@@ -610,6 +610,17 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.interp = (fl & PT_INTERP) ? 1u : 0u;
     a.init_mode = (fl & PT_INIT_RANDOM) ? 1u : ((fl & PT_INIT_FWEIGHT) ? 2u : 0u);
     a.mask = c->d_mask;
+    a.rec_n = c->layout.nvox() * (uint64_t)c->vol.nsamples;
+    a.V = V;
+    a.out_n = nout;
+#if PT_CHECK_BOUNDS
+    // negative control of the bounds-checked build: pretend the map / mask / record buffers
+    // are half their size, so in-range accesses to the upper half must be reported
+    if (getenv("PT_CHECK_BOUNDS_SHRINK")) {
+        a.V /= 2;
+        a.rec_n /= 2;
+    }
+#endif
     pt::TrackMode mode;
     mode.simple = simple;
     mode.out = a.o_nsteps || a.o_reason || a.o_end || a.o_paths || a.conn;
@@ -636,6 +647,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         a.utab = c->d_utab;
         a.ulog = ulog;
         a.max_ctas = ctas;
+        a.utab_lanes = (uint32_t)(ctas * (uint64_t)pt::kThreadsExt);
     }
 
     // experiment (env PT_MAP_PERSIST=1): the map as a persisting L2 access-policy window
@@ -783,6 +795,8 @@ pt_status pt_get_stats(pt_ctx* c, pt_stats* out) {
     out->kernel_ms = ms;
     CK(cudaEventElapsedTime(&ms, c->ev[0], c->ev[3]), "pt_get_stats: track time");
     out->track_ms = ms;
+    if (s[pt::kStatBadAccess])
+        return fail(c, PT_ERR_CUDA, "bounds check (PT_CHECK_BOUNDS build): a tracking kernel accessed outside a buffer");
     if (s[pt::kStatBadId])
         return fail(c, PT_ERR_ARG, "pt_track: a device-resident seed_id * P overflows 64 bits (those particles ran as seed id 0)");
     if (out->overflow) return fail(c, PT_ERR_OVERFLOW, "a uint32 map cell wrapped past 2^32-1");
@@ -1019,6 +1033,8 @@ pt_status pt_get_mcmc_stats(pt_ctx* c, pt_mcmc_stats* out) {
     float ms = 0.f;
     CK(cudaEventElapsedTime(&ms, c->mev[0], c->mev[1]), "pt_get_mcmc_stats: kernel time");
     out->kernel_ms = ms;
+    if (s[pt::kMcmcStatBadAccess])
+        return fail(c, PT_ERR_CUDA, "bounds check (PT_CHECK_BOUNDS build): the MCMC kernel accessed outside a buffer");
     return PT_OK;
 }
 

@@ -47,6 +47,7 @@ __device__ __forceinline__ unsigned long long chunk_sub(unsigned long long chunk
         k = chunk / a.chunks_per_seed;
         j = (chunk - k * a.chunks_per_seed) * (uint64_t)a.cta_chunk + (uint64_t)t * kSub;
     }
+    PT_BOUND(a, k < a.nseeds);
     const uint32_t seed = a.order ? a.order[k] : (uint32_t)k;
     return ((unsigned long long)seed << 32) | j;
 }

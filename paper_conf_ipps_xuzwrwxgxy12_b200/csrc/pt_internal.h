@@ -36,8 +36,27 @@ enum StatIdx {
     kStatBadId = 8,      // a device-resident seed id whose pid overflows 64 bits
     kStatUnique = 9,     // UNQ: first entries counted (= increments of the unique map)
     kStatLabelMax = 10,  // pt_load_targets: largest label
-    kNumStats = 11
+    kStatBadAccess = 11, // PT_CHECK_BOUNDS builds: a device access outside its buffer
+    kNumStats = 12
 };
+
+// Bounds-checked build (-DPT_CHECK_BOUNDS=1, tests/test_gpu_bounds.py): every record gather,
+// map / hash-set / mask / label / output access of the tracking kernels is checked against
+// the size of its buffer (TrackArgs::*_n); a violation sets stats[kStatBadAccess] and
+// pt_get_stats fails.  Replaces compute-sanitizer memcheck, which this GPU pool does not run.
+#ifndef PT_CHECK_BOUNDS
+#define PT_CHECK_BOUNDS 0
+#endif
+#if PT_CHECK_BOUNDS
+#define PT_BOUND(a, cond)                                                                          \
+    do {                                                                                         \
+        if (!(cond)) atomicOr((a).stats + ::pt::kStatBadAccess, 1ull);                           \
+    } while (0)
+#else
+#define PT_BOUND(a, cond) \
+    do {                  \
+    } while (0)
+#endif
 
 struct TrackArgs {
     const uint8_t* rec;          // [V'][S] records of rec_bytes, voxel order rec_vox() (bricked)
@@ -81,6 +100,11 @@ struct TrackArgs {
     unsigned long long* utab;    // [lanes][2^ulog] generation-tagged hash sets, zeroed per call
     uint32_t ulog;               // log2 entries per lane's hash set
     uint64_t max_ctas;           // CTAs the hash-set buffer covers
+    // buffer sizes, read only by PT_CHECK_BOUNDS builds
+    uint64_t rec_n;              // records in rec (allocated voxels x S)
+    uint64_t V;                  // voxels of map / mask / labels (nx ny nz)
+    uint64_t out_n;              // entries of o_nsteps / o_reason / o_end (particles x halves)
+    uint32_t utab_lanes;         // lanes (hash sets) in utab
 };
 
 // Which instantiation of the tracking kernel a call runs.
@@ -92,7 +116,7 @@ struct TrackMode {
 };
 
 // NEXT-4 MCMC sampler (pt_mcmc.cu): one warp per voxel of the compacted mask list.
-enum McmcStatIdx { kMcmcStatAccepted = 0, kMcmcNumStats = 2 };
+enum McmcStatIdx { kMcmcStatAccepted = 0, kMcmcStatBadAccess = 1, kMcmcNumStats = 2 };  // 1: PT_CHECK_BOUNDS
 struct McmcArgs {
     const float* dwi;            // [nmeas][V]
     const float* bvals;          // [nmeas]

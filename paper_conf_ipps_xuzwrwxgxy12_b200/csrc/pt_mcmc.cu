@@ -144,6 +144,11 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
         const bool gact = slot < a.nvox;  // a group without a voxel computes on base's, writes nothing
         const uint32_t v = a.vox[gact ? slot : base];
         const uint64_t V = a.V;
+#if PT_CHECK_BOUNDS
+        bool bad = !(v < V) || (gact && !(slot < a.nvox));
+        for (int m = 0; m < MPL; ++m) bad = bad || (valid[m] && !((int)gl + LPV * m < a.nmeas));
+        if (bad) atomicOr(a.stats + kMcmcStatBadAccess, 1ull);
+#endif
 #pragma unroll
         for (int m = 0; m < MPL; ++m) {
             yf[m] = valid[m] ? a.dwi[(uint64_t)(gl + LPV * m) * V + v] : 0.f;
@@ -498,6 +503,9 @@ __global__ void __launch_bounds__(kMcmcThreads, PT_MCMC_MIN_BLOCKS) mcmc_kernel(
             // samples after the burn-in, every L loops; lane k writes omega_k
             if (t >= a.burnin && (t - a.burnin + 1u) % a.interval == 0u) {
                 const uint32_t s = (t - a.burnin + 1u) / a.interval - 1u;
+#if PT_CHECK_BOUNDS
+                if (s >= a.nsamples) atomicOr(a.stats + kMcmcStatBadAccess, 1ull);
+#endif
                 if (gact && gl < (uint32_t)NP) a.samples[((uint64_t)gl * a.nsamples + s) * V + v] = my_w;
             }
         }

@@ -37,6 +37,7 @@ __device__ __forceinline__ void seg_finish(const TrackArgs& a, const SegState& s
                                            float qy, float qz) {
     if (OUT) {
         const uint64_t li = s.li[i];
+        PT_BOUND(a, li < a.out_n);
         if (a.o_nsteps) a.o_nsteps[li] = (uint16_t)n;
         if (a.o_reason) a.o_reason[li] = (uint8_t)why;
         if (a.o_end) {
@@ -54,7 +55,9 @@ __global__ void seg_init_kernel(const __grid_constant__ TrackArgs a, SegState s,
     for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < count; i += gridDim.x * blockDim.x) {
         const uint64_t g = base + i;                 // processing-order particle index
         const uint64_t k = g / a.P, j = g - k * a.P;
+        PT_BOUND(a, k < a.nseeds);
         const uint64_t si = a.order ? a.order[k] : k;
+        PT_BOUND(a, si < a.nseeds);
         uint64_t sid = a.seed_ids ? a.seed_ids[si] : si;
         if (sid > a.max_seed_id) {  // pid would overflow 64 bits: reported as PT_ERR_ARG
             atomicExch(a.stats + kStatBadId, 1ull);
@@ -73,7 +76,9 @@ __global__ void seg_init_kernel(const __grid_constant__ TrackArgs a, SegState s,
         uint32_t v;
         // non-finite seeds are outside (R12; a NaN would truncate into the volume)
         const bool fin = isfinite(qx) && isfinite(qy) && isfinite(qz);
-        const bool ok = fin && inside_volume(a, qx, qy, qz, v) && a.mask[v] != 0;
+        const bool inv = fin && inside_volume(a, qx, qy, qz, v);
+        if (inv) PT_BOUND(a, v < a.V);
+        const bool ok = inv && a.mask[v] != 0;
         s.vox[i] = v;
         s.live[i] = i;
         s.flag[i] = ok ? 1 : 0;
@@ -113,6 +118,7 @@ __global__ void __launch_bounds__(256) seg_kernel(const __grid_constant__ TrackA
             const uint32_t smp = a.sample_mode ? (uint32_t)((s.li[i] % a.P) % a.S) : sample_of(wn, a.S);
             R rv;
             const uint32_t rvx = rec_vox_raster(vox, (uint32_t)a.nx, (uint32_t)a.ny, a.rb_log, a.rb_nbx, a.rb_nby);
+            PT_BOUND(a, (uint64_t)rvx * a.S + smp < a.rec_n && smp < a.S);
             ldg_record<RB>(a.rec + ((uint64_t)rvx * a.S + smp) * RB, rv.w);
             float vx, vy, vz, f0;
             rv.fibre(0, vx, vy, vz, f0);
@@ -146,7 +152,9 @@ __global__ void __launch_bounds__(256) seg_kernel(const __grid_constant__ TrackA
             const float nqy = __fadd_rn(qy, __fmul_rn(a.step, dy));
             const float nqz = __fadd_rn(qz, __fmul_rn(a.step, dz));
             uint32_t v;
-            if (!inside_volume(a, nqx, nqy, nqz, v) || a.mask[v] == 0) {  // P:L177, R11
+            const bool inv = inside_volume(a, nqx, nqy, nqz, v);
+            if (inv) PT_BOUND(a, v < a.V);
+            if (!inv || a.mask[v] == 0) {  // P:L177, R11
                 why = kSMask;
                 break;
             }

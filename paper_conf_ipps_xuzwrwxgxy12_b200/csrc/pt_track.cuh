@@ -132,6 +132,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     // UNQ: this lane's hash set (2^ulog generation-tagged entries, zeroed by pt_track)
     unsigned long long* const utab =
         UNQ ? a.utab + (((uint64_t)blockIdx.x * TPB + threadIdx.x) << a.ulog) : nullptr;
+    if (UNQ) PT_BOUND(a, (uint64_t)blockIdx.x * TPB + threadIdx.x < a.utab_lanes);
 
     L x;
     x.alive = false;
@@ -185,6 +186,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     auto write_outputs = [&](int n, int why, float qx, float qy, float qz) {
         if (OUT && (a.o_nsteps || a.o_reason || a.o_end)) {
             const uint64_t e = out_index();
+            PT_BOUND(a, e < a.out_n);
             if (a.o_nsteps) a.o_nsteps[e] = (uint16_t)n;
             if (a.o_reason) a.o_reason[e] = (uint8_t)why;
             if (a.o_end) {
@@ -202,6 +204,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
             uint64_t m = x.tmask;
             while (m) {
                 const int t = __ffsll((long long)m) - 1;
+                PT_BOUND(a, x.sidx < a.nseeds && (uint32_t)t < a.ntargets);
                 atomicAdd(a.conn + (uint64_t)x.sidx * a.ntargets + (uint32_t)t, 1u);
                 m &= m - 1ull;
             }
@@ -214,7 +217,10 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         }
     };
     // a run of visits of one voxel: one predicated RED
-    auto red_run = [&](bool p, uint32_t vox, uint32_t cnt) { red_add_if(p, map + vox, cnt); };
+    auto red_run = [&](bool p, uint32_t vox, uint32_t cnt) {
+        if (p) PT_BOUND(a, vox < a.V);
+        red_add_if(p, map + vox, cnt);
+    };
     auto flush_run = [&]() {
         if (!UNQ && has_map) red_run(x.run_cnt != 0u, x.run_vox, x.run_cnt);
         x.run_cnt = 0u;
@@ -231,6 +237,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         uint32_t h = x.uh;
         const uint32_t mask = (1u << a.ulog) - 1u;
         while (open) {
+            PT_BOUND(a, h < (1u << a.ulog));
             if ((uint32_t)(e >> 32) != x.gen) {  // empty or a stale streamline's entry
                 utab[h] = ((unsigned long long)x.gen << 32) | x.ukey;
                 fresh = true;
@@ -243,6 +250,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
             }
         }
         x.upend = false;
+        if (has_map && fresh) PT_BOUND(a, x.ukey < a.V);
         red_add_if(has_map && fresh, map + x.ukey, 1u);
         my_unique += fresh ? 1u : 0u;
     };
@@ -261,6 +269,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     // Returns false if the seed is outside the volume (R12).
     auto begin = [&](uint32_t h) -> bool {
         x.half = h;
+        PT_BOUND(a, x.sidx < a.nseeds);
         x.qx = __fsub_rn(a.seeds[3 * x.sidx + 0], a.fcx);
         x.qy = __fsub_rn(a.seeds[3 * x.sidx + 1], a.fcy);
         x.qz = __fsub_rn(a.seeds[3 * x.sidx + 2], a.fcz);
@@ -270,6 +279,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         x.run_vox = 0xFFFFFFFFu;
         x.prev_vox = 0xFFFFFFFFu;
         if (OUT && a.o_paths) {
+            PT_BOUND(a, out_index() < a.out_n && a.path_stride > 0);
             float* pp = a.o_paths + out_index() * (uint64_t)a.path_stride * 3u;
             pp[0] = __fadd_rn(x.qx, a.fcx);
             pp[1] = __fadd_rn(x.qy, a.fcy);
@@ -307,6 +317,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     // GetStartPoint(): a new particle (seed index si, particle j of the seed)
     auto start = [&](uint64_t si, uint64_t j) {
         const uint64_t li = si * a.P + j;
+        PT_BOUND(a, si < a.nseeds && j < a.P);
         if (OUT) s_li[threadIdx.x] = li;
         uint64_t sid = a.seed_ids ? a.seed_ids[si] : si;
         if (sid > a.max_seed_id) {  // pid would overflow 64 bits: reported as PT_ERR_ARG
@@ -359,10 +370,12 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
 #endif
         }
         if (OUT && a.conn && c) {  // NEXT-2: targets entered by committed steps (R21)
+            PT_BOUND(a, v < a.V);
             const uint32_t lbl = __ldg(a.labels + v);
             x.tmask |= (lbl != 0u && lbl <= a.ntargets) ? (1ull << (lbl - 1u)) : 0ull;
         }
         if (OUT && a.o_paths && c && x.n < a.path_stride) {
+            PT_BOUND(a, out_index() < a.out_n);
             float* pp = a.o_paths + (out_index() * (uint64_t)a.path_stride + (uint64_t)x.n) * 3u;
             pp[0] = __fadd_rn(x.qx, a.fcx);
             pp[1] = __fadd_rn(x.qy, a.fcy);
@@ -377,6 +390,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     auto gather = [&](bool p, float cqx, float cqy, float cqz, uint32_t nrv, uint32_t v, uint32_t nn,
                       uint32_t s) -> bool {
         if (!interp) {
+            if (p) PT_BOUND(a, (uint64_t)nrv * a.S + s < a.rec_n && s < a.S);
             ldg_record_if<RB>(p, rec_at(nrv, s), x.rv.w);
             return p && x.rv.outside();
         }
@@ -386,6 +400,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         const int jx = interp_axis(cqx, a.cx, I.x), jy = interp_axis(cqy, a.cy, I.y), jz = interp_axis(cqz, a.cz, I.z);
         const bool jin = (unsigned)jx < (unsigned)a.nx && (unsigned)jy < (unsigned)a.ny && (unsigned)jz < (unsigned)a.nz;
         const uint32_t jv = ((uint32_t)jz * (uint32_t)a.ny + (uint32_t)jy) * (uint32_t)a.nx + (uint32_t)jx;
+        if (p) PT_BOUND(a, (uint64_t)(jin ? recv(jx, jy, jz, jv) : nrv) * a.S + s < a.rec_n && s < a.S && v < a.V);
         ldg_record_if<RB>(p, rec_at(jin ? recv(jx, jy, jz, jv) : nrv, s), x.rv.w);
         const uint32_t mb = p ? (uint32_t)__ldg(a.mask + v) : 1u;
         const bool outside = p && mb == 0u;
