@@ -181,6 +181,24 @@ def _ncu_traffic(cfg, steps):
         return None
 
 
+def _ncu_counters(cfg):
+    """Counters of the committed ncu --set full capture of this config's tracking kernel
+    (north star: achieved L2 / HBM sector throughput, warp execution efficiency), or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_track_summary.json")
+    try:
+        e = json.load(open(p)).get("per_config", {}).get(cfg)
+    except (OSError, ValueError):
+        return None
+    if not e:
+        return None
+    keys = ("tag", "warp_exec_efficiency", "issue_active_pct", "l1_hit_rate_pct", "l2_hit_rate_pct",
+            "lts_throughput_pct", "l2_read_sectors_per_step", "l2_red_sectors_per_step", "dram_bytes_per_step",
+            "warp_inst_per_32_steps")
+    out = {k: e[k] for k in keys if k in e}
+    out["source"] = "profiles/ncu_track_summary.json (ncu --set full capture, profiles/<tag>_" + cfg + "_track_ncu.md)"
+    return out
+
+
 def _workload(cfg):
     import phantom
     return phantom.config(cfg)
@@ -758,6 +776,7 @@ def run_ours(args):
             "emulated_scaling": emulated,
             "roofline": roof,
             "gather_roofline": gather,
+            "ncu": _ncu_counters(args.config) if not args.track_flags else None,
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_vals[False], "unit": "steps/s",
                     "h2d_bytes_per_step": int(seeds_h.numel() * 4 + ids_h.numel() * 8),

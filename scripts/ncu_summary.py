@@ -88,6 +88,8 @@ def main():
     ap.add_argument("--launches")
     ap.add_argument("--rep")
     ap.add_argument("--note", default="")
+    ap.add_argument("--bench-log", help="stdout of the captured bench.py run (its JSON line gives the steps per launch)")
+    ap.add_argument("--steps", type=float, help="committed steps of the captured launch (else from --bench-log)")
     a = ap.parse_args()
     os.makedirs(PROF, exist_ok=True)
     if a.launches:
@@ -115,12 +117,34 @@ def main():
             v = float(v.replace(",", ""))
             mult = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}.get(u, 1)
             return v * mult
-        d["per_config"][a.cfg] = {
+        steps = a.steps
+        if steps is None and a.bench_log:
+            for ln in open(a.bench_log, errors="replace"):
+                if ln.startswith("{") and '"steps_per_pass"' in ln:
+                    cfgd = json.loads(ln)["config"]
+                    steps = float(cfgd["steps_per_pass"])
+        dram = num("dram__bytes_read.sum") + num("dram__bytes_write.sum")
+        e = {
             "tag": a.tag,
-            "dram_bytes_per_launch": num("dram__bytes_read.sum") + num("dram__bytes_write.sum"),
+            "dram_bytes_per_launch": dram,
             "l2_hit_rate_pct": float(r["lts__t_sector_hit_rate.pct"][0]),
+            "l1_hit_rate_pct": float(r["l1tex__t_sector_hit_rate.pct"][0]),
             "kernel_s_under_ncu": float(r["gpu__time_duration.sum"][0]),
+            "issue_active_pct": float(r["smsp__issue_active.avg.pct_of_peak_sustained_active"][0]),
+            # warp execution efficiency: active threads per executed warp instruction / 32
+            "warp_exec_efficiency": float(r["smsp__thread_inst_executed_per_inst_executed.ratio"][0]) / 32.0,
+            "lts_throughput_pct": float(r["lts__throughput.avg.pct_of_peak_sustained_elapsed"][0]),
         }
+        if steps:
+            e["steps_per_launch_captured"] = steps
+            e["dram_bytes_per_step"] = dram / steps
+            # warp instructions per 32 committed steps (= per fully active warp-step)
+            e["warp_inst_per_32_steps"] = 32.0 * num("smsp__inst_executed.sum") / steps
+            e["l2_read_sectors_per_step"] = num("lts__t_sectors_srcunit_tex_op_read.sum") / steps
+            e["l2_red_sectors_per_step"] = num("lts__t_sectors_srcunit_tex_op_red.sum") / steps
+        if a.note:
+            e["note"] = a.note
+        d["per_config"][a.cfg] = e
         json.dump(d, open(sp, "w"), indent=1)
     print("ok")
 
