@@ -63,6 +63,8 @@ struct pt_ctx {
     size_t temp_cap = 0;
     uint32_t* d_map = nullptr;   // internal map for host map pointers
     size_t map_cap = 0;
+    uint32_t* d_pmap = nullptr;  // PT_MAP_PERM: permuted scratch map
+    size_t pmap_cap = 0;
     unsigned long long* d_utab = nullptr;  // NEXT-2 unique map: per-lane hash sets
     size_t utab_cap = 0;
     uint8_t* d_stage = nullptr;    // pt_load_samples: staging of host inputs (grow-only)
@@ -292,7 +294,7 @@ void pt_destroy(pt_ctx* c) {
     DeviceGuard g(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
     else cudaDeviceSynchronize();
-    void* bufs[] = {c->d_rec, c->d_mask, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_utab,
+    void* bufs[] = {c->d_rec, c->d_mask, c->d_seeds, c->d_ids, c->d_order, c->d_temp, c->d_map, c->d_pmap, c->d_utab,
                     c->d_stage, c->d_labels, c->d_conn, c->d_nsteps, c->d_reason, c->d_end, c->d_paths,
                     c->d_stats, c->d_mstats, c->d_mvox, c->d_mflags, c->d_mtemp, c->d_mcount, c->d_seg};
     for (void* b : bufs)
@@ -597,6 +599,21 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         a.total_chunks = a.group_chunks + (N - a.group_chunks * G);
     }
     a.map = d_map;
+    uint32_t pmask = 0u;
+    // the kernels count into a permuted scratch map (pt_internal.h) unless the
+    // record volume is large (c5: its L2 is thrashed by the records and the raster map's line
+    // locality matters more than spreading the REDs over the slices)
+    int perm = PT_MAP_PERM;
+    if (const char* e = getenv("PT_MAP_PERM")) perm = atoi(e);  // experiments
+    if (d_map && (perm == 2 || (perm == 1 && c->rec_size <= PT_BIG_VOLUME))) {
+        uint64_t cells = 1ull << PT_MAP_GRAN;
+        while (cells < V) cells <<= 1;
+        CK(ensure(c->d_pmap, c->pmap_cap, cells), "pt_track: scratch map");
+        CK(cudaMemsetAsync(c->d_pmap, 0, cells * sizeof(uint32_t), st), "pt_track: scratch map zero");
+        a.map = c->d_pmap;
+        pmask = (uint32_t)((cells >> PT_MAP_GRAN) - 1);
+    }
+    a.map_mask = pmask;
     a.o_nsteps = (fl & PT_REC_LEN) ? c->d_nsteps : nullptr;
     a.o_reason = (fl & PT_REC_REASON) ? c->d_reason : nullptr;
     a.o_end = (fl & PT_REC_END) ? c->d_end : nullptr;
@@ -702,6 +719,8 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         cudaCtxResetPersistingL2Cache();
         cudaGetLastError();
     }
+    if (pmask)
+        CK(pt::launch_map_unpermute(c->d_pmap, pmask, d_map, (int64_t)V, true, st), "pt_track: scratch map add");
     if (d_map) CK(pt::launch_map_sum(d_map, (int64_t)V, c->d_stats + pt::kStatMapAfter, st), "pt_track: map sum");
     if (host_map) {
         CK(cudaMemcpyAsync(map, d_map, V * sizeof(uint32_t), cudaMemcpyDeviceToHost, st), "pt_track: map D2H");

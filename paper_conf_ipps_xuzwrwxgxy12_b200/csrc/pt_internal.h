@@ -20,6 +20,22 @@ constexpr int kSimpleThreads = 256;  // no-refill ablation kernel
 #define PT_CTA_THREADS_EXT 768
 #endif
 constexpr int kThreadsExt = PT_CTA_THREADS_EXT;  // variant / unique-map instantiations
+// Permuted scratch map (map_mask != 0): the kernels count into a scratch map whose cell of
+// voxel v keeps the low PT_MAP_GRAN bits of v and multiplies the rest by an odd constant
+// mod 2^k (a bijection on [0, 2^(k+g)) >= V), so the RED bursts of the compact neighbourhood
+// the CTAs work on spread over all L2 slices instead of a few; pt_track then adds the
+// scratch into the caller's raster map (map_unpermute).
+#ifndef PT_MAP_PERM
+#define PT_MAP_PERM 1  // 0: never permute; 1: permute when the record volume is <= PT_BIG_VOLUME; 2: always
+#endif
+#ifndef PT_MAP_GRAN
+#define PT_MAP_GRAN 0  // log2 voxels kept together per permuted unit
+#endif
+constexpr uint32_t kMapMul = 0x9E3779B1u;
+__host__ __device__ __forceinline__ uint32_t map_perm(uint32_t v, uint32_t mask) {
+    constexpr uint32_t g = PT_MAP_GRAN, lo = (1u << g) - 1u;
+    return ((((v >> g) * kMapMul) & mask) << g) | (v & lo);
+}
 constexpr uint32_t kSub = 32;
 constexpr uint32_t kMinCtaChunk = 1024;
 
@@ -105,7 +121,12 @@ struct TrackArgs {
     uint64_t V;                  // voxels of map / mask / labels (nx ny nz)
     uint64_t out_n;              // entries of o_nsteps / o_reason / o_end (particles x halves)
     uint32_t utab_lanes;         // lanes (hash sets) in utab
+    uint32_t map_mask;           // 0: raster map; else permuted units of the scratch map - 1
 };
+// cell of voxel v in the map the kernels add into
+__host__ __device__ __forceinline__ uint32_t map_cell(const TrackArgs& a, uint32_t v) {
+    return a.map_mask ? map_perm(v, a.map_mask) : v;
+}
 
 // Which instantiation of the tracking kernel a call runs.
 struct TrackMode {
@@ -189,6 +210,9 @@ cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint32_t* key
                               uint32_t* idx, uint32_t* perm, void* temp, size_t temp_bytes, cudaStream_t st);
 cudaError_t launch_map_sum(const uint32_t* map, int64_t V, unsigned long long* out,
                            cudaStream_t st);
+// PT_MAP_PERM: map[v] (+)= scratch[(v * kMapMul) & mask]
+cudaError_t launch_map_unpermute(const uint32_t* scratch, uint32_t mask, uint32_t* map, int64_t V, bool accumulate,
+                                 cudaStream_t st);
 cudaError_t launch_gather_bench(const uint8_t* buf, uint64_t nrec, int rec_bytes, uint32_t iters,
                                 int blocks, uint32_t seed, uint32_t* sink, cudaStream_t st);
 int gather_bench_blocks_per_sm(int rec_bytes);

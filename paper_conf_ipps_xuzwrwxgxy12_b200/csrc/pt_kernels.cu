@@ -63,7 +63,7 @@ __global__ void repack_kernel(const void* __restrict__ dyads, const void* __rest
             atomicAdd(bad, 1ull);
         }
         const uint64_t rv = rec_vox_raster((uint32_t)vox, (uint32_t)nx, (uint32_t)ny, L.b, L.nbx, L.nby);
-        uint8_t* out = rec + (rv * (uint64_t)S + (uint64_t)s) * RB;
+        uint8_t* out = rec + rec_slot((uint32_t)rv, (uint32_t)s, (uint32_t)S, L.b) * RB;
         if (RB == 8) {
             *reinterpret_cast<uint2*>(out) = make_uint2(w[0], w[1]);
         } else {
@@ -127,6 +127,14 @@ __global__ void map_sum_kernel(const uint32_t* __restrict__ map, int64_t V, unsi
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(kFull, s, o);
     if ((threadIdx.x & 31) == 0 && s) atomicAdd(out, s);
+}
+
+__global__ void map_unpermute_kernel(const uint32_t* __restrict__ pm, uint32_t mask, uint32_t* __restrict__ map,
+                                     int64_t V, bool acc) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < V; i += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t c = pm[map_perm((uint32_t)i, mask)];
+        map[i] = acc ? map[i] + c : c;
+    }
 }
 
 // ------------------------------------------------------------------------- RNG self-test
@@ -245,6 +253,14 @@ cudaError_t launch_map_sum(const uint32_t* map, int64_t V, unsigned long long* o
     if (blocks > 148 * 8) blocks = 148 * 8;
     if (blocks < 1) blocks = 1;
     map_sum_kernel<<<(unsigned)blocks, 256, 0, st>>>(map, V, out);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_map_unpermute(const uint32_t* scratch, uint32_t mask, uint32_t* map, int64_t V, bool accumulate,
+                                 cudaStream_t st) {
+    if (V <= 0) return cudaSuccess;
+    const int64_t blocks = (V + 255) / 256 < 4096 ? (V + 255) / 256 : 4096;
+    map_unpermute_kernel<<<(unsigned)blocks, 256, 0, st>>>(scratch, mask, map, V, accumulate);
     return cudaGetLastError();
 }
 

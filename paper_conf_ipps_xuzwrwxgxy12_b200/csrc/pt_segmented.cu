@@ -119,7 +119,7 @@ __global__ void __launch_bounds__(256) seg_kernel(const __grid_constant__ TrackA
             R rv;
             const uint32_t rvx = rec_vox_raster(vox, (uint32_t)a.nx, (uint32_t)a.ny, a.rb_log, a.rb_nbx, a.rb_nby);
             PT_BOUND(a, (uint64_t)rvx * a.S + smp < a.rec_n && smp < a.S);
-            ldg_record<RB>(a.rec + ((uint64_t)rvx * a.S + smp) * RB, rv.w);
+            ldg_record<RB>(a.rec + rec_slot(rvx, smp, a.S, a.rb_log) * RB, rv.w);
             float vx, vy, vz, f0;
             rv.fibre(0, vx, vy, vz, f0);
             bool neg;
@@ -166,7 +166,7 @@ __global__ void __launch_bounds__(256) seg_kernel(const __grid_constant__ TrackA
             pz = dz;
             vox = v;
             n += 1;
-            if (a.map) atomicAdd(a.map + v, 1u);  // P:L109, R13 (plain global RED per step)
+            if (a.map) atomicAdd(a.map + map_cell(a, v), 1u);  // P:L109, R13 (plain global RED per step)
             my_steps += 1;
         }
         s.flag[t] = why >= 0 ? 0 : 1;  // by list position: the compaction's flags

@@ -42,15 +42,6 @@
 #ifndef PT_RUNLEN
 #define PT_RUNLEN 1  // merge consecutive visits of a voxel before the RED (0: ablation iv, one RED per step)
 #endif
-#ifndef PT_MAP_AGG
-#define PT_MAP_AGG 0  // experiment: per-CTA shared-memory aggregation of the map REDs (see track_kernel)
-#endif
-#ifndef PT_AGG_LOG
-#define PT_AGG_LOG 10  // log2 slots per aggregation table
-#endif
-#ifndef PT_AGG_ROUNDS
-#define PT_AGG_ROUNDS 2  // rounds per aggregation epoch
-#endif
 #ifndef PT_REFILL_MIN
 #define PT_REFILL_MIN 2  // free lanes a warp waits for before refilling (amortises the refill block)
 #endif
@@ -123,19 +114,6 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     __shared__ unsigned long long s_li[OUT ? TPB : 1];  // particle index (outputs)
     __shared__ uint32_t s_q[TPB / 32][3];               // per-warp sub-chunk
     __shared__ unsigned long long s_work;               // CTA claim + tickets
-    // Map aggregation (PT_MAP_AGG): two direct-mapped tables of (voxel, count) in shared
-    // memory, one per epoch parity.  A warp adds a run to the slot of its voxel in the table
-    // of its current epoch (claiming an empty slot with one CAS; a slot held by another
-    // voxel sends the run to the global map), and moves to the next epoch every
-    // PT_AGG_ROUNDS rounds.  The last warp to leave an epoch (or to exit) adds the table to
-    // the map with one RED per used slot, clears it and releases it for epoch + 2; a warp
-    // entering an epoch waits until its table is released.  No CTA barrier: the warps of a
-    // CTA drift at most one epoch apart.
-    constexpr bool AGG = PT_MAP_AGG && REFILL && !UNQ;
-    constexpr int AM = AGG ? (1 << PT_AGG_LOG) : 1;
-    constexpr uint32_t kEmpty = 0xFFFFFFFFu;
-    __shared__ uint32_t s_akey[2][AM], s_acnt[2][AM];
-    __shared__ uint32_t s_aw[2], s_aready[2];  // (exited << 16 | left) per table; released epoch
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t wib = threadIdx.x >> 5;
     const uint32_t lt_mask = (1u << lane) - 1u;
@@ -147,17 +125,6 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     const uint32_t init_mode = VN ? a.init_mode : 0u;
     const bool smode = BL < 0 && a.sample_mode != 0u;  // paper mode (NEXT-1): s = j mod S
     if (threadIdx.x == 0) s_work = kNoChunk << 24;
-    if (AGG) {
-        for (int i = threadIdx.x; i < 2 * AM; i += TPB) {
-            (&s_akey[0][0])[i] = kEmpty;
-            (&s_acnt[0][0])[i] = 0u;
-        }
-        if (threadIdx.x == 0) {
-            s_aw[0] = s_aw[1] = 0u;
-            s_aready[0] = 0u;
-            s_aready[1] = 1u;
-        }
-    }
     if (lane == 0) {
         s_q[wib][0] = 0u;
         s_q[wib][1] = 0u;
@@ -211,7 +178,9 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         const uint32_t br = ((uz >> b) * a.rb_nby + (uy >> b)) * a.rb_nbx + (ux >> b);
         return (br << (3 * b)) | ((uz & m) << (2 * b)) | ((uy & m) << b) | (ux & m);
     };
-    auto rec_at = [&](uint32_t rv, uint32_t s) -> const uint8_t* { return a.rec + ((uint64_t)rv * a.S + s) * RB; };
+    auto rec_at = [&](uint32_t rv, uint32_t s) -> const uint8_t* {
+        return a.rec + rec_slot(rv, s, a.S, BL < 0 ? a.rb_log : (uint32_t)BL) * RB;
+    };
     // Philox block of the lane's stream (R16: ctr = {block, pid_lo, pid_hi, stream})
     auto philox = [&](uint32_t block, uint32_t stream) -> uint4 {
         return philox4x32_10(make_uint4(block, (uint32_t)x.pid, (uint32_t)(x.pid >> 32), stream), a.key0, a.key1);
@@ -252,61 +221,9 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         }
     };
     // a run of visits of one voxel: one predicated RED
-    uint32_t a_ep = 0u, a_er = 0u;  // AGG: the warp's epoch and rounds in it (warp-uniform)
     auto red_run = [&](bool p, uint32_t vox, uint32_t cnt) {
         if (p) PT_BOUND(a, vox < a.V);
-        if (AGG) {
-            // one predicated CAS claims the slot or returns its voxel; straight-line code
-            const uint32_t h = (vox * 0x9E3779B1u) >> (32 - PT_AGG_LOG);
-            const uint32_t ka = (uint32_t)__cvta_generic_to_shared(&s_akey[a_ep & 1u][h]);
-            const uint32_t ca = (uint32_t)__cvta_generic_to_shared(&s_acnt[a_ep & 1u][h]);
-            uint32_t prev = 0u;
-            asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %4, 0;\n\t@q atom.shared.cas.b32 %0, [%1], %2, %3;\n\t}"
-                         : "+r"(prev) : "r"(ka), "r"(kEmpty), "r"(vox), "r"((int)p) : "memory");
-            const bool hit = p && (prev == kEmpty || prev == vox);
-            asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q red.shared.add.u32 [%0], %1;\n\t}"
-                         :: "r"(ca), "r"(cnt), "r"((int)hit) : "memory");
-            red_add_if(p && !hit, map + vox, cnt);
-        } else {
-            red_add_if(p, map + vox, cnt);
-        }
-    };
-    // AGG epochs: all warps have left table b's epoch: add it to the map, clear, release
-    auto agg_flush = [&](uint32_t b, uint32_t release) {
-        __threadfence_block();
-        for (uint32_t i = lane; i < (uint32_t)AM; i += 32u) {
-            const uint32_t k = s_akey[b][i];
-            if (k != kEmpty) {
-                red_add_if(true, map + k, s_acnt[b][i]);
-                s_akey[b][i] = kEmpty;
-                s_acnt[b][i] = 0u;
-            }
-        }
-        __syncwarp();
-        if (lane == 0) {
-            atomicAnd(&s_aw[b], 0xFFFF0000u);
-            __threadfence_block();
-            *(volatile uint32_t*)&s_aready[b] = release;
-        }
-        __syncwarp();
-    };
-    // leave epoch e (inc 1) or exit in it (inc 1 << 16: counted as gone in every later epoch)
-    auto agg_leave = [&](uint32_t e, uint32_t inc) {
-        const uint32_t b = e & 1u;
-        uint32_t now = 0u;
-        __syncwarp();
-        if (lane == 0) {
-            __threadfence_block();
-            now = atomicAdd(&s_aw[b], inc) + inc;
-        }
-        now = __shfl_sync(kFull, now, 0);
-        if ((now & 0xFFFFu) + (now >> 16) == (uint32_t)(TPB / 32)) agg_flush(b, e + 2u);
-    };
-    auto agg_enter = [&](uint32_t e) {
-        if (lane == 0)
-            while (*(volatile uint32_t*)&s_aready[e & 1u] != e) __nanosleep(32);
-        __syncwarp();
-        __threadfence_block();
+        red_add_if(p, map + map_cell(a, vox), cnt);
     };
     auto flush_run = [&]() {
         if (!UNQ && has_map) red_run(x.run_cnt != 0u, x.run_vox, x.run_cnt);
@@ -338,7 +255,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         }
         x.upend = false;
         if (has_map && fresh) PT_BOUND(a, x.ukey < a.V);
-        red_add_if(has_map && fresh, map + x.ukey, 1u);
+        red_add_if(has_map && fresh, map + map_cell(a, x.ukey), 1u);
         my_unique += fresh ? 1u : 0u;
     };
     auto unq_issue = [&](bool c, uint32_t v) {
@@ -665,12 +582,6 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         }
         if (!__any_sync(kFull, x.alive)) break;
         rounds += 1u;
-        if (AGG && has_map && ++a_er == (uint32_t)PT_AGG_ROUNDS) {
-            a_er = 0u;
-            agg_leave(a_ep, 1u);
-            a_ep += 1u;
-            agg_enter(a_ep);
-        }
 
         // ------------------------------------------------ round start: one Philox block,
         // gather of (pending candidate | seed) voxel = mask test + first step's record
@@ -706,11 +617,6 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         for (int k = 0; k < kRoundSteps; ++k) step(k);
     }
 
-    if (AGG && has_map) {  // gone from this epoch and the next (the tables stay consistent)
-        agg_leave(a_ep, 1u << 16);
-        agg_enter(a_ep + 1u);
-        agg_leave(a_ep + 1u, 1u << 16);
-    }
     // ---- counters: one atomic per warp (64-bit sums of the per-lane counters)
     unsigned long long s_steps = my_steps, s_parts = my_particles, s_act = my_active, s_uq = my_unique;
 #pragma unroll
