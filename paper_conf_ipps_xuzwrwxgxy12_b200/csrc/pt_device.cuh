@@ -177,20 +177,10 @@ __device__ __forceinline__ uint32_t rec_vox(int ix, int iy, int iz, uint32_t b, 
     const uint32_t br = ((z >> b) * nby + (y >> b)) * nbx + (x >> b);
     return (br << (3u * b)) | ((z & m) << (2u * b)) | ((y & m) << b) | (x & m);
 }
-// Index of record (voxel rv of the record order, sample s).  Voxel-major: rv * S + s (a
-// voxel's S samples contiguous).  PT_REC_SMAJOR (experiment, bricked layouts only): sample-
-// major inside a brick, ((brick * S + s) << 3b) | local, so a voxel's samples lie 2^3b
-// records apart (on different L2 slices) and a 128-B line holds x-neighbours of one sample.
-#ifndef PT_REC_SMAJOR
-#define PT_REC_SMAJOR 0
-#endif
+// Index of record (voxel rv of the record order, sample s): voxel-major, a voxel's S samples
+// contiguous (a sample-major order inside each brick, which puts a voxel's samples on
+// different L2 slices, measured 3.7-6 % slower: DESIGN §11).
 __host__ __device__ __forceinline__ uint64_t rec_slot(uint32_t rv, uint32_t s, uint32_t S, uint32_t b) {
-#if PT_REC_SMAJOR
-    if (b) {
-        const uint32_t lb = 3u * b;
-        return (((uint64_t)(rv >> lb) * S + s) << lb) | (rv & ((1u << lb) - 1u));
-    }
-#endif
     (void)b;
     return (uint64_t)rv * S + s;
 }
