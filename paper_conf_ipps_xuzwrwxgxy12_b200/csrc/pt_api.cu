@@ -176,6 +176,16 @@ cudaError_t ensure(T*& ptr, size_t& cap, size_t n) {
     return e;
 }
 
+// value of a binary16 bit pattern (exact; host side of the fp16 eligibility threshold)
+static float half_bits_to_float(uint32_t h) {
+    const uint32_t e = (h >> 10) & 0x1Fu, m = h & 0x3FFu;
+    float v;
+    if (e == 0u) v = std::ldexp((float)m, -24);
+    else if (e == 31u) v = m ? NAN : INFINITY;
+    else v = std::ldexp((float)(m | 0x400u), (int)e - 25);
+    return (h & 0x8000u) ? -v : v;
+}
+
 int rec_bytes_of(int F, int dtype) {
     if (F < 1 || F > 3) return 0;
     int raw;
@@ -599,21 +609,18 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         a.total_chunks = a.group_chunks + (N - a.group_chunks * G);
     }
     a.map = d_map;
-    uint32_t pmask = 0u;
-    // the kernels count into a permuted scratch map (pt_internal.h) unless the
-    // record volume is large (c5: its L2 is thrashed by the records and the raster map's line
-    // locality matters more than spreading the REDs over the slices)
-    int perm = PT_MAP_PERM;
-    if (const char* e = getenv("PT_MAP_PERM")) perm = atoi(e);  // experiments
-    if (d_map && (perm == 2 || (perm == 1 && c->rec_size <= PT_BIG_VOLUME))) {
-        uint64_t cells = 1ull << PT_MAP_GRAN;
-        while (cells < V) cells <<= 1;
-        CK(ensure(c->d_pmap, c->pmap_cap, cells), "pt_track: scratch map");
-        CK(cudaMemsetAsync(c->d_pmap, 0, cells * sizeof(uint32_t), st), "pt_track: scratch map zero");
-        a.map = c->d_pmap;
-        pmask = (uint32_t)((cells >> PT_MAP_GRAN) - 1);
+    {   // smallest binary16 pattern whose value exceeds fib_thr (fp16 records, fib_thr >= 0;
+        // the finite non-negative patterns 0 .. 0x7BFF are ordered like their values)
+        uint32_t lo = 0u, hi = 0x7C00u;  // 0x7C00 (+inf): no finite f is eligible
+        if (p->fib_thr >= 0.f) {
+            while (lo < hi) {
+                const uint32_t mid = (lo + hi) / 2u;
+                if (half_bits_to_float(mid) > p->fib_thr) hi = mid;
+                else lo = mid + 1u;
+            }
+        }
+        a.fib_h = (int32_t)(hi << 16);
     }
-    a.map_mask = pmask;
     a.o_nsteps = (fl & PT_REC_LEN) ? c->d_nsteps : nullptr;
     a.o_reason = (fl & PT_REC_REASON) ? c->d_reason : nullptr;
     a.o_end = (fl & PT_REC_END) ? c->d_end : nullptr;
@@ -667,6 +674,31 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         a.utab_lanes = (uint32_t)(ctas * (uint64_t)pt::kThreadsExt);
     }
 
+    // The kernels count into a context-owned scratch map, added into the caller's raster map
+    // after the kernel (map_unpermute_kernel), when (a) the map is permuted -- cell of key k =
+    // map_perm(k): the RED bursts of the compact neighbourhood the CTAs work on spread over
+    // all L2 slices; used unless the record volume is large (c5: its records thrash L2 and
+    // the map's line locality matters more) -- or (b) the launch keys the map by record voxel
+    // (track_rv_keys: the bench instantiations, which then need no raster index per step).
+    const bool rvk = !segmented && pt::track_rv_keys(a, mode, c->vol.dtype == PT_F16);
+    a.map_keys = rvk ? c->layout.nvox() : V;
+    int perm = PT_MAP_PERM;
+    if (const char* e = getenv("PT_MAP_PERM")) perm = atoi(e);  // experiments
+    const bool permuted = d_map && (perm == 2 || (perm == 1 && c->rec_size <= PT_BIG_VOLUME));
+    const bool scratch = d_map && (permuted || rvk);
+    uint32_t pmask = 0u;
+    if (scratch) {
+        uint64_t cells = a.map_keys;
+        if (permuted) {
+            cells = 1ull << PT_MAP_GRAN;
+            while (cells < a.map_keys) cells <<= 1;
+            pmask = (uint32_t)((cells >> PT_MAP_GRAN) - 1);
+        }
+        CK(ensure(c->d_pmap, c->pmap_cap, cells), "pt_track: scratch map");
+        CK(cudaMemsetAsync(c->d_pmap, 0, cells * sizeof(uint32_t), st), "pt_track: scratch map zero");
+        a.map = c->d_pmap;
+    }
+    a.map_mask = pmask;
     // experiment (env PT_MAP_PERSIST=1): the map as a persisting L2 access-policy window
     const bool persist = d_map && getenv("PT_MAP_PERSIST") && atoi(getenv("PT_MAP_PERSIST")) > 0;
     if (persist) {
@@ -719,8 +751,9 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         cudaCtxResetPersistingL2Cache();
         cudaGetLastError();
     }
-    if (pmask)
-        CK(pt::launch_map_unpermute(c->d_pmap, pmask, d_map, (int64_t)V, true, st), "pt_track: scratch map add");
+    if (scratch)
+        CK(pt::launch_map_unpermute(c->d_pmap, pmask, rvk, nxv, nyv, c->layout, d_map, (int64_t)V, true, st),
+           "pt_track: scratch map add");
     if (d_map) CK(pt::launch_map_sum(d_map, (int64_t)V, c->d_stats + pt::kStatMapAfter, st), "pt_track: map sum");
     if (host_map) {
         CK(cudaMemcpyAsync(map, d_map, V * sizeof(uint32_t), cudaMemcpyDeviceToHost, st), "pt_track: map D2H");

@@ -85,6 +85,33 @@ struct Rec {
     }
 };
 
+// ---------------------------------------------------------------------------- direction
+// Direction of the last step, d = sign * (a record's unit vector).  fp32 records: three
+// floats.  fp16 records: d is a sign-flipped binary16 vector, kept packed (xy = x | y << 16,
+// z in the low half of zw) and never decoded for the dot products of the fibre choice:
+// they run as mixed-precision FMAs (FHFMA: f32 = f16 * f16 + f32).  The product of two
+// binary16 values is exact in binary32 (22 significand bits, exponents within range), so
+// fma(a, b, c) = round(a*b + c) is bit-identical to the contract's round(round(a*b) + c)
+// (R15); the first product is added to -0, which returns it unchanged, signed zero included.
+__device__ __forceinline__ float hfma_lo(uint32_t a, uint32_t b, float c) {
+    float d;
+    asm("{.reg .f16 ha, hb;\n\tmov.b32 {ha, _}, %1;\n\tmov.b32 {hb, _}, %2;\n\tfma.rn.f32.f16 %0, ha, hb, %3;\n\t}"
+        : "=f"(d) : "r"(a), "r"(b), "f"(c));
+    return d;
+}
+__device__ __forceinline__ float hfma_hi(uint32_t a, uint32_t b, float c) {
+    float d;
+    asm("{.reg .f16 ha, hb;\n\tmov.b32 {_, ha}, %1;\n\tmov.b32 {_, hb}, %2;\n\tfma.rn.f32.f16 %0, ha, hb, %3;\n\t}"
+        : "=f"(d) : "r"(a), "r"(b), "f"(c));
+    return d;
+}
+// ((vx * dx + vy * dy) + vz * dz) of a packed fp16 vector (w_xy, w_z) and a packed direction
+__device__ __forceinline__ float hdot(uint32_t wxy, uint32_t wz, uint32_t dxy, uint32_t dz) {
+    return hfma_lo(wz, dz, hfma_hi(wxy, dxy, hfma_lo(wxy, dxy, -0.f)));
+}
+__device__ __forceinline__ float half_lo(uint32_t w) { return __half2float(__ushort_as_half((unsigned short)(w & 0xFFFFu))); }
+__device__ __forceinline__ float half_hi(uint32_t w) { return __half2float(__ushort_as_half((unsigned short)(w >> 16))); }
+
 // Random gather of one record through the read-only (texture/L1) path: one LDG of 8, 16
 // or 32 bytes (two 32-B LDGs for a 64-B record).
 template <int BYTES>

@@ -122,6 +122,8 @@ struct TrackArgs {
     uint64_t out_n;              // entries of o_nsteps / o_reason / o_end (particles x halves)
     uint32_t utab_lanes;         // lanes (hash sets) in utab
     uint32_t map_mask;           // 0: raster map; else permuted units of the scratch map - 1
+    int32_t fib_h;               // fp16 records, fib_thr >= 0: (smallest binary16 > fib_thr) << 16
+    uint64_t map_keys;           // map keys: V (raster voxel) or the padded record voxels (rv keys)
 };
 // cell of voxel v in the map the kernels add into
 __host__ __device__ __forceinline__ uint32_t map_cell(const TrackArgs& a, uint32_t v) {
@@ -135,6 +137,7 @@ struct TrackMode {
     bool var;     // NEXT-3 variants (run-time selected by bidir / interp / init_mode)
     bool unique;  // NEXT-2 per-streamline-unique map
 };
+
 
 // NEXT-4 MCMC sampler (pt_mcmc.cu): one warp per voxel of the compacted mask list.
 enum McmcStatIdx { kMcmcStatAccepted = 0, kMcmcStatBadAccess = 1, kMcmcNumStats = 2 };  // 1: PT_CHECK_BOUNDS
@@ -210,11 +213,24 @@ cudaError_t launch_seed_order(const float* seeds, uint64_t nseeds, uint32_t* key
                               uint32_t* idx, uint32_t* perm, void* temp, size_t temp_bytes, cudaStream_t st);
 cudaError_t launch_map_sum(const uint32_t* map, int64_t V, unsigned long long* out,
                            cudaStream_t st);
-// PT_MAP_PERM: map[v] (+)= scratch[(v * kMapMul) & mask]
-cudaError_t launch_map_unpermute(const uint32_t* scratch, uint32_t mask, uint32_t* map, int64_t V, bool accumulate,
-                                 cudaStream_t st);
+// map[v] (+)= scratch[cell(key(v))]: key = v or its record voxel rv (RecLayout L), cell =
+// map_perm(key, mask) or key (mask 0)
+cudaError_t launch_map_unpermute(const uint32_t* scratch, uint32_t mask, bool rv_keys, int nx, int ny,
+                                 const RecLayout& L, uint32_t* map, int64_t V, bool accumulate, cudaStream_t st);
 cudaError_t launch_gather_bench(const uint8_t* buf, uint64_t nrec, int rec_bytes, uint32_t iters,
                                 int blocks, uint32_t seed, uint32_t* sink, cudaStream_t st);
 int gather_bench_blocks_per_sm(int rec_bytes);
+
+// The bench instantiations (compile-time bricked record layout, no outputs, default
+// semantics) key the map by the record voxel rv their gathers already computed (no raster
+// index per step); every other instantiation by the raster voxel.  pt_track sizes and
+// reads back the scratch map accordingly; launch_track_fh takes the same decision.
+#ifndef PT_RVKEYS
+#define PT_RVKEYS 1  // 0: every instantiation keys the map by raster voxel (A/B switch)
+#endif
+inline bool track_rv_keys(const TrackArgs& a, const TrackMode& m, bool half) {
+    return PT_RVKEYS && !m.simple && !m.unique && !m.var && !m.out && !a.sample_mode &&
+           !(half && !(a.fib_thr >= 0.f)) && a.rb_log == kBrickLog;
+}
 
 }  // namespace pt

@@ -129,10 +129,11 @@ __global__ void map_sum_kernel(const uint32_t* __restrict__ map, int64_t V, unsi
     if ((threadIdx.x & 31) == 0 && s) atomicAdd(out, s);
 }
 
-__global__ void map_unpermute_kernel(const uint32_t* __restrict__ pm, uint32_t mask, uint32_t* __restrict__ map,
-                                     int64_t V, bool acc) {
+__global__ void map_unpermute_kernel(const uint32_t* __restrict__ pm, uint32_t mask, bool rvk, uint32_t nx,
+                                     uint32_t ny, RecLayout L, uint32_t* __restrict__ map, int64_t V, bool acc) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < V; i += (int64_t)gridDim.x * blockDim.x) {
-        const uint32_t c = pm[map_perm((uint32_t)i, mask)];
+        const uint32_t key = rvk ? rec_vox_raster((uint32_t)i, nx, ny, L.b, L.nbx, L.nby) : (uint32_t)i;
+        const uint32_t c = pm[mask ? map_perm(key, mask) : key];
         map[i] = acc ? map[i] + c : c;
     }
 }
@@ -256,11 +257,12 @@ cudaError_t launch_map_sum(const uint32_t* map, int64_t V, unsigned long long* o
     return cudaGetLastError();
 }
 
-cudaError_t launch_map_unpermute(const uint32_t* scratch, uint32_t mask, uint32_t* map, int64_t V, bool accumulate,
-                                 cudaStream_t st) {
+cudaError_t launch_map_unpermute(const uint32_t* scratch, uint32_t mask, bool rv_keys, int nx, int ny,
+                                 const RecLayout& L, uint32_t* map, int64_t V, bool accumulate, cudaStream_t st) {
     if (V <= 0) return cudaSuccess;
     const int64_t blocks = (V + 255) / 256 < 4096 ? (V + 255) / 256 : 4096;
-    map_unpermute_kernel<<<(unsigned)blocks, 256, 0, st>>>(scratch, mask, map, V, accumulate);
+    map_unpermute_kernel<<<(unsigned)blocks, 256, 0, st>>>(scratch, mask, rv_keys, (uint32_t)nx, (uint32_t)ny, L, map,
+                                                            V, accumulate);
     return cudaGetLastError();
 }
 

@@ -70,7 +70,8 @@ struct Lane {
     bool alive;        // holds a particle (half) in flight
     bool pend;         // the round's last candidate step waits for the next round's gather
     float qx, qy, qz;  // committed position, centred coordinates (R10)
-    float px, py, pz;  // direction of the last (candidate) step
+    float px, py, pz;  // direction of the last (candidate) step (fp32 records)
+    uint32_t pxy, pzw; // the same as packed halves (fp16 records, see hdot)
     uint32_t gvox;     // raster voxel of the round-start gather (seed or pending candidate)
     uint32_t grv;      // its position in the record volume (rec_vox)
     int n;             // committed steps (of this half)
@@ -86,6 +87,7 @@ struct Lane {
     uint32_t half;     // 0, or 1 = the reverse half of a bidirectional streamline
     bool have_d0;      // half 0 computed its first direction
     float d0x, d0y, d0z;
+    uint32_t d0xy, d0zw;  // (fp16 records)
     uint32_t winit;    // word 3 of Philox(stream 2, block 0): the first fibre (R24)
     // UNQ (R25)
     uint32_t gen;      // generation tag of the streamline in the lane's hash set
@@ -111,6 +113,9 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     constexpr bool VB = (VM & kVarBidir) != 0, VI = (VM & kVarInterp) != 0, VN = (VM & kVarInit) != 0;
     // q and d of a particle that ends are read again only for its outputs (end point, path)
     constexpr bool KEEPQ = OUT;
+    // the bench instantiations key the map by the record voxel (track_rv_keys): no raster
+    // voxel index on their path
+    constexpr bool RVKEY = PT_RVKEYS && BL > 0 && !OUT && !UNQ && VM == 0 && REFILL;
     __shared__ unsigned long long s_li[OUT ? TPB : 1];  // particle index (outputs)
     __shared__ uint32_t s_q[TPB / 32][3];               // per-warp sub-chunk
     __shared__ unsigned long long s_work;               // CTA claim + tickets
@@ -141,6 +146,8 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     x.pend = false;
     x.qx = x.qy = x.qz = 0.f;
     x.px = x.py = x.pz = 0.f;
+    x.pxy = x.pzw = 0u;
+    x.d0xy = x.d0zw = 0u;
     x.gvox = 0u;
     x.grv = 0u;
     x.n = 0;
@@ -222,7 +229,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     };
     // a run of visits of one voxel: one predicated RED
     auto red_run = [&](bool p, uint32_t vox, uint32_t cnt) {
-        if (p) PT_BOUND(a, vox < a.V);
+        if (p) PT_BOUND(a, vox < a.map_keys);
         red_add_if(p, map + map_cell(a, vox), cnt);
     };
     auto flush_run = [&]() {
@@ -311,6 +318,8 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
                 x.px = -x.d0x;
                 x.py = -x.d0y;
                 x.pz = -x.d0z;
+                x.pxy = x.d0xy ^ 0x80008000u;
+                x.pzw = x.d0zw ^ 0x00008000u;
                 x.alive = true;
                 return;
             }
@@ -334,6 +343,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         x.sidx = (uint32_t)si;
         x.have_d0 = false;
         x.px = x.py = x.pz = 0.f;
+        x.pxy = x.pzw = 0u;
         x.why = -1;
         if (UNQ) x.gen += 1u;
         if (begin(0u)) {
@@ -353,7 +363,8 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     // commit a step (if c): new position, one visit of the new voxel (R13);
     // consecutive visits of the same voxel are merged (run length) and flushed with a
     // predicated RED when the voxel changes.  Straight-line except for the UNQ probe.
-    auto commit_if = [&](bool c, float nx_, float ny_, float nz_, uint32_t v) {
+    // v: raster voxel, mk: map key (= v, or the record voxel with RVKEY)
+    auto commit_if = [&](bool c, float nx_, float ny_, float nz_, uint32_t v, uint32_t mk) {
         // without outputs the position of an ended particle is never read again: no select
         x.qx = (c || !KEEPQ) ? nx_ : x.qx;
         x.qy = (c || !KEEPQ) ? ny_ : x.qy;
@@ -366,12 +377,12 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
             x.run_vox = c ? v : x.run_vox;
         } else if (has_map) {
 #if PT_RUNLEN
-            const bool change = v != x.run_vox;
+            const bool change = mk != x.run_vox;
             red_run(c && change && x.run_cnt != 0u, x.run_vox, x.run_cnt);
             x.run_cnt = c ? (change ? 1u : x.run_cnt + 1u) : x.run_cnt;
-            x.run_vox = c ? v : x.run_vox;
+            x.run_vox = c ? mk : x.run_vox;
 #else
-            red_add_if(c, map + v, 1u);  // ablation (iv): one global RED per committed step
+            red_run(c, mk, 1u);  // ablation (iv): one global RED per committed step
 #endif
         }
         if (OUT && a.conn && c) {  // NEXT-2: targets entered by committed steps (R21)
@@ -468,30 +479,67 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         // f_j > fib_thr (R7), strict >, lowest j wins (R8); the first step takes fibre 0
         // (R5; with R24 the round start moved the drawn fibre to slot 0).  "Interpolation()" of
         // Alg. 1 = this sample's record (R2).
-        float vx, vy, vz, f0;
-        x.rv.fibre(0, vx, vy, vz, f0);
-        float bc = __fadd_rn(__fadd_rn(__fmul_rn(vx, x.px), __fmul_rn(vy, x.py)), __fmul_rn(vz, x.pz));
-        float best = f0 > a.fib_thr ? fabsf(bc) : -1.f;
+        float vx, vy, vz, bc, best;
+        bool neg;
+        uint32_t dxy = 0u, dzw = 0u;  // fp16: the chosen direction, packed
+        if constexpr (HALF) {
+            // dot products on the packed halves (exact mixed-precision FMAs, see hdot)
+            // R7 eligibility f_j > fib_thr: on the bench layouts (BL >= 0, launched only for
+            // fib_thr >= 0) an integer compare of f's bits, in the high half of word 2j+1,
+            // with those of the smallest binary16 above fib_thr (finite f, validated on load)
+            auto elig = [&](uint32_t wzw) -> bool {
+                return BL >= 0 ? (int32_t)wzw >= a.fib_h : half_hi(wzw) > a.fib_thr;
+            };
+            uint32_t cxy = x.rv.w[0], czw = x.rv.w[1];
+            bc = hdot(cxy, czw, x.pxy, x.pzw);
+            best = elig(czw) ? fabsf(bc) : -1.f;
 #pragma unroll
-        for (int j = 1; j < F; ++j) {
-            float ux, uy, uz, fu;
-            x.rv.fibre(j, ux, uy, uz, fu);
-            const float cj = __fadd_rn(__fadd_rn(__fmul_rn(ux, x.px), __fmul_rn(uy, x.py)), __fmul_rn(uz, x.pz));
-            const bool pick = !first && fu > a.fib_thr && fabsf(cj) > best;
-            best = pick ? fabsf(cj) : best;
-            bc = pick ? cj : bc;
-            vx = pick ? ux : vx;
-            vy = pick ? uy : vy;
-            vz = pick ? uz : vz;
+            for (int j = 1; j < F; ++j) {
+                const uint32_t uxy = x.rv.w[2 * j], uzw = x.rv.w[2 * j + 1];
+                const float cj = hdot(uxy, uzw, x.pxy, x.pzw);
+                const bool pick = !first && elig(uzw) && fabsf(cj) > best;
+                best = pick ? fabsf(cj) : best;
+                bc = pick ? cj : bc;
+                cxy = pick ? uxy : cxy;
+                czw = pick ? uzw : czw;
+            }
+            neg = first ? (x.W.w >> 31) != 0u : !(bc > 0.f);
+            // sign * v: flip the sign bits (exact negation), then decode (exact)
+            dxy = cxy ^ (neg ? 0x80008000u : 0u);
+            dzw = (czw & 0xFFFFu) ^ (neg ? 0x8000u : 0u);
+            vx = half_lo(dxy);
+            vy = half_hi(dxy);
+            vz = half_lo(dzw);
+        } else {
+            float f0;
+            x.rv.fibre(0, vx, vy, vz, f0);
+            bc = __fadd_rn(__fadd_rn(__fmul_rn(vx, x.px), __fmul_rn(vy, x.py)), __fmul_rn(vz, x.pz));
+            best = f0 > a.fib_thr ? fabsf(bc) : -1.f;
+#pragma unroll
+            for (int j = 1; j < F; ++j) {
+                float ux, uy, uz, fu;
+                x.rv.fibre(j, ux, uy, uz, fu);
+                const float cj = __fadd_rn(__fadd_rn(__fmul_rn(ux, x.px), __fmul_rn(uy, x.py)), __fmul_rn(uz, x.pz));
+                const bool pick = !first && fu > a.fib_thr && fabsf(cj) > best;
+                best = pick ? fabsf(cj) : best;
+                bc = pick ? cj : bc;
+                vx = pick ? ux : vx;
+                vy = pick ? uy : vy;
+                vz = pick ? uz : vz;
+            }
+            neg = first ? (x.W.w >> 31) != 0u : !(bc > 0.f);
         }
         // maximum angle, measured by the dot product (R4); orientation
         // kept (R9); first step: sign = top bit of word 3 of block 0 (R6, R16)
         const bool curv_ok = first || fabsf(bc) > a.curv_thr;
-        const bool neg = first ? (x.W.w >> 31) != 0u : !(bc > 0.f);
-        // StepToNextPoint(): q' = q + h * (sign * v), no FMA
-        const float dx = neg ? -vx : vx, dy = neg ? -vy : vy, dz = neg ? -vz : vz;
+        // StepToNextPoint(): q' = q + h * (sign * v), no FMA (fp16: v already signed)
+        const float dx = (HALF || !neg) ? vx : -vx, dy = (HALF || !neg) ? vy : -vy, dz = (HALF || !neg) ? vz : -vz;
         if (VB) {  // R22: half 0's first direction, defined even if the step is not committed
             const bool rec0 = first && x.alive;
+            if constexpr (HALF) {
+                x.d0xy = rec0 ? dxy : x.d0xy;
+                x.d0zw = rec0 ? dzw : x.d0zw;
+            }
             x.d0x = rec0 ? dx : x.d0x;
             x.d0y = rec0 ? dy : x.d0y;
             x.d0z = rec0 ? dz : x.d0z;
@@ -509,9 +557,15 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         // (without outputs the reason is never read: any value >= 0 marks "ended")
         x.why = (x.alive && !go) ? (!OUT ? kEndMask : maxed ? kEndMaxlen : (!curv_ok ? kEndCurv : kEndMask)) : x.why;
         x.alive = go;
-        x.px = (go || !KEEPQ) ? dx : x.px;  // (an ended particle's direction is never read)
-        x.py = (go || !KEEPQ) ? dy : x.py;
-        x.pz = (go || !KEEPQ) ? dz : x.pz;
+        // (an ended particle's direction is never read)
+        if constexpr (HALF) {
+            x.pxy = (go || !KEEPQ) ? dxy : x.pxy;
+            x.pzw = (go || !KEEPQ) ? dzw : x.pzw;
+        } else {
+            x.px = (go || !KEEPQ) ? dx : x.px;
+            x.py = (go || !KEEPQ) ? dy : x.py;
+            x.pz = (go || !KEEPQ) ? dz : x.pz;
+        }
         if (k < kRoundSteps - 1) {
             if ((k + 1) % 3 == 0) {
                 // the next step opens the round's next Philox block: a live lane has
@@ -520,13 +574,14 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
             }
             const uint32_t w = ((k + 1) % 3 == 0) ? x.W.x : ((k + 1) % 3 == 1) ? x.W.y : x.W.z;
             const uint32_t sk = smode ? x.sfix : sample_of(w, a.S);
-            const bool outside = gather(go, nqx, nqy, nqz, recv(ix, iy, iz, v), v, (uint32_t)x.n + 1u, sk);
+            const uint32_t nrv = recv(ix, iy, iz, v);
+            const bool outside = gather(go, nqx, nqy, nqz, nrv, v, (uint32_t)x.n + 1u, sk);
             x.why = outside ? kEndMask : x.why;
             x.alive = go && !outside;
-            commit_if(x.alive, nqx, nqy, nqz, v);
+            commit_if(x.alive, nqx, nqy, nqz, v, RVKEY ? nrv : v);
         } else {
             x.pend = go;  // next round's start gathers and tests it
-            x.gvox = go ? v : x.gvox;
+            if (!RVKEY) x.gvox = go ? v : x.gvox;
             x.grv = go ? recv(ix, iy, iz, v) : x.grv;
         }
     };
@@ -590,16 +645,18 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
             x.W = philox(t0 / 3u, VB ? x.half : 0u);
             const uint32_t s0 = smode ? x.sfix : sample_of(x.W.x, a.S);
             // the pending candidate, recomputed bit-identically from (q, d) instead of kept
-            const float cqx = x.pend ? __fadd_rn(x.qx, __fmul_rn(a.step, x.px)) : x.qx;
-            const float cqy = x.pend ? __fadd_rn(x.qy, __fmul_rn(a.step, x.py)) : x.qy;
-            const float cqz = x.pend ? __fadd_rn(x.qz, __fmul_rn(a.step, x.pz)) : x.qz;
+            const float ppx = HALF ? half_lo(x.pxy) : x.px, ppy = HALF ? half_hi(x.pxy) : x.py,
+                        ppz = HALF ? half_lo(x.pzw) : x.pz;
+            const float cqx = x.pend ? __fadd_rn(x.qx, __fmul_rn(a.step, ppx)) : x.qx;
+            const float cqy = x.pend ? __fadd_rn(x.qy, __fmul_rn(a.step, ppy)) : x.qy;
+            const float cqz = x.pend ? __fadd_rn(x.qz, __fmul_rn(a.step, ppz)) : x.qz;
             if (VN && init_mode != 0u && !interp && t0 == 0u && (!VB || x.half == 0u) && x.alive)
                 x.winit = philox(0u, 2u).w;  // R24 draw (with PT_INTERP the gather computes it)
             // seed outside the mask (R12) or pending candidate rejected (R11)
             const bool outside = gather(x.alive, cqx, cqy, cqz, x.grv, x.gvox, t0, s0);
             x.why = outside ? kEndMask : x.why;
             x.alive = x.alive && !outside;
-            commit_if(x.pend && !outside, cqx, cqy, cqz, x.gvox);
+            commit_if(x.pend && !outside, cqx, cqy, cqz, x.gvox, RVKEY ? x.grv : x.gvox);
             // R24: the first step of half 0 takes the drawn fibre: move it to slot 0 of the
             // record (the first step uses only the chosen fibre's vector)
             if (VN && F > 1 && init_mode != 0u) {
@@ -694,6 +751,10 @@ cudaError_t launch_track_fh(const TrackArgs& a, const TrackMode& m, int num_sms,
     if (m.out) return launch_track_kernel<F, HALF, true, true, -1, 0, false>(a, num_sms, st);
     if (a.sample_mode) return launch_track_kernel<F, HALF, true, false, -1, 0, false>(a, num_sms, st);
     // the bench path: record layout as a compile-time constant, random sample per step
+    // (the compile-time layouts compare fp16 f bits as integers: fib_thr >= 0 only)
+    // (track_rv_keys: exactly the kBrickLog instantiation keys the map by record voxel)
+    if (track_rv_keys(a, m, HALF)) return launch_track_kernel<F, HALF, true, false, (int)kBrickLog, 0, false>(a, num_sms, st);
+    if (HALF && !(a.fib_thr >= 0.f)) return launch_track_kernel<F, HALF, true, false, -1, 0, false>(a, num_sms, st);
     if (a.rb_log == 0) return launch_track_kernel<F, HALF, true, false, 0, 0, false>(a, num_sms, st);
     if (a.rb_log == kBrickLog) return launch_track_kernel<F, HALF, true, false, (int)kBrickLog, 0, false>(a, num_sms, st);
     return cudaErrorInvalidValue;

@@ -34,8 +34,8 @@ ab)
             --no-parity --no-lengths --no-e2e "$@" 2>/dev/null | tail -1 | python -c "
 import json, sys
 d = json.loads(sys.stdin.read())
-print('$lib', '$cfg', round(d['value'] / 1e9, 2), 'G steps/s', round(d['roofline']['kernel_ms'], 2), 'ms',
-      d['active_lane_fraction'], d['clocks']['sm_mhz'])" | tee -a gpurun_out/${TAG}_ab.log
+print('$lib', '$cfg', round(d['value'] / 1e9, 6), 'G', d['unit'], round(d['roofline'].get('kernel_ms', 0.0), 2), 'ms',
+      d.get('active_lane_fraction'), d['clocks']['sm_mhz'])" | tee -a gpurun_out/${TAG}_ab.log
     done; done; done ;;
 ncu)
     CFG=$1; KRE=${2:-track_kernel}; shift 2 || shift $#
