@@ -48,6 +48,7 @@ struct pt_ctx {
     pt_volume vol{};
     int rec_bytes = 0;
     pt::RecLayout layout{};       // record voxel order (bricked, rec_vox)
+    float max_abs = 0.f;          // largest |vector component| inside the mask (margin test)
     uint8_t* d_rec = nullptr;
     size_t rec_size = 0;
     uint8_t* d_mask = nullptr;    // tracking mask copy (the variant kernel's interpolation)
@@ -412,19 +413,29 @@ pt_status pt_load_samples(pt_ctx* c, const pt_volume* v, const void* dyads, cons
     cudaError_t e = ensure(c->d_mask, c->mask_cap, (size_t)V);
     if (e == cudaSuccess) e = cudaMemcpyAsync(c->d_mask, d_m, (size_t)V, cudaMemcpyDeviceToDevice, c->stream);
     if (e == cudaSuccess) e = cudaMemsetAsync(c->d_stats + pt::kStatBadInput, 0, sizeof(unsigned long long), c->stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(c->d_stats + pt::kStatMaxAbs, 0, sizeof(unsigned long long), c->stream);
     if (e == cudaSuccess)
         e = pt::launch_repack(d_dy, d_f, d_m, c->d_rec, v->nx, v->ny, v->nz, L, v->nsamples, v->nfibres,
-                              v->dtype == PT_F16, rb, c->d_stats + pt::kStatBadInput, c->stream);
+                              v->dtype == PT_F16, rb, c->d_stats + pt::kStatBadInput, c->d_stats + pt::kStatMaxAbs,
+                              c->stream);
     if (e == cudaSuccess) e = cudaEventRecord(c->lev[2], c->stream);
-    unsigned long long bad = 0;
+    unsigned long long bad = 0, maxabs = 0;
     if (e == cudaSuccess)
         e = cudaMemcpyAsync(&bad, c->d_stats + pt::kStatBadInput, sizeof bad, cudaMemcpyDeviceToHost, c->stream);
+    if (e == cudaSuccess)
+        e = cudaMemcpyAsync(&maxabs, c->d_stats + pt::kStatMaxAbs, sizeof maxabs, cudaMemcpyDeviceToHost, c->stream);
     if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
     if (e != cudaSuccess) return cuda_fail(c, e, "pt_load_samples: repack");
     if (bad) return fail(c, PT_ERR_ARG, "pt_load_samples: %llu records inside the mask hold non-finite values", bad);
     c->vol = *v;
     c->rec_bytes = rb;
     c->layout = L;
+    {
+        const uint32_t mb = (uint32_t)maxabs;
+        float m;
+        std::memcpy(&m, &mb, sizeof m);
+        c->max_abs = m;
+    }
     c->loaded = true;
     c->tracked = false;
     c->ntargets = 0;  // targets belong to a volume shape
@@ -553,6 +564,12 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.rb_log = c->layout.b;
     a.rb_nbx = c->layout.nbx;
     a.rb_nby = c->layout.nby;
+    a.rb_off = c->layout.off;
+    {
+        const uint32_t b = c->layout.b, B3 = 1u << (3u * b);
+        a.rb_ky = c->layout.nbx * B3 - (1u << (2u * b));
+        a.rb_kz = c->layout.nbx * c->layout.nby * B3 - B3;
+    }
     a.nx = nxv;
     a.ny = nyv;
     a.nz = nzv;
@@ -562,6 +579,12 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.fcx = (float)a.cx;
     a.fcy = (float)a.cy;
     a.fcz = (float)a.cz;
+    a.pcx = a.cx + (int)c->layout.off;
+    a.pcy = a.cy + (int)c->layout.off;
+    a.pcz = a.cz + (int)c->layout.off;
+    // every candidate stays within the margin: |step * v_a| < off - 1 voxels per axis
+    a.nobounds = (c->layout.off > 0u && std::isfinite(c->max_abs) &&
+                  (double)p->step * (double)c->max_abs < (double)c->layout.off - 1.0) ? 1u : 0u;
     a.S = (uint32_t)c->vol.nsamples;
     a.sample_mode = (fl & PT_SAMPLE_PER_STREAMLINE) ? 1u : 0u;
     a.step = p->step;

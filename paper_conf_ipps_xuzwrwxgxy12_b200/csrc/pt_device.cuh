@@ -198,9 +198,10 @@ __device__ __forceinline__ int axis_index(float q, int c) {
 // being strided by whole planes (fewer DRAM pages and TLB entries per neighbourhood).
 // b = 0 is the plain raster layout (nbx = nx, nby = ny).  Layout only: which record a
 // step reads is unchanged, so results are unaffected.
-__device__ __forceinline__ uint32_t rec_vox(int ix, int iy, int iz, uint32_t b, uint32_t nbx, uint32_t nby) {
+__device__ __forceinline__ uint32_t rec_vox(int ix, int iy, int iz, uint32_t b, uint32_t nbx, uint32_t nby,
+                                            uint32_t off = 0u) {
     const uint32_t m = (1u << b) - 1u;
-    const uint32_t x = (uint32_t)ix, y = (uint32_t)iy, z = (uint32_t)iz;
+    const uint32_t x = (uint32_t)ix + off, y = (uint32_t)iy + off, z = (uint32_t)iz + off;
     const uint32_t br = ((z >> b) * nby + (y >> b)) * nbx + (x >> b);
     return (br << (3u * b)) | ((z & m) << (2u * b)) | ((y & m) << b) | (x & m);
 }
@@ -213,10 +214,10 @@ __host__ __device__ __forceinline__ uint64_t rec_slot(uint32_t rv, uint32_t s, u
 }
 // the same from a raster voxel index (variant / ablation kernels, repack)
 __device__ __forceinline__ uint32_t rec_vox_raster(uint32_t v, uint32_t nx, uint32_t ny, uint32_t b, uint32_t nbx,
-                                                   uint32_t nby) {
+                                                   uint32_t nby, uint32_t off = 0u) {
     if (b == 0u) return v;
     const uint32_t z = v / (nx * ny), r = v - z * (nx * ny), y = r / nx, x = r - y * nx;
-    return rec_vox((int)x, (int)y, (int)z, b, nbx, nby);
+    return rec_vox((int)x, (int)y, (int)z, b, nbx, nby, off);
 }
 
 }  // namespace pt

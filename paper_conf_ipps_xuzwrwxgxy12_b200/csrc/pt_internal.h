@@ -53,7 +53,8 @@ enum StatIdx {
     kStatUnique = 9,     // UNQ: first entries counted (= increments of the unique map)
     kStatLabelMax = 10,  // pt_load_targets: largest label
     kStatBadAccess = 11, // PT_CHECK_BOUNDS builds: a device access outside its buffer
-    kNumStats = 12
+    kStatMaxAbs = 12,    // repack: bits of the largest |vector component| inside the mask
+    kNumStats = 13
 };
 
 // Bounds-checked build (-DPT_CHECK_BOUNDS=1, tests/test_gpu_bounds.py): every record gather,
@@ -77,6 +78,10 @@ enum StatIdx {
 struct TrackArgs {
     const uint8_t* rec;          // [V'][S] records of rec_bytes, voxel order rec_vox() (bricked)
     uint32_t rb_log, rb_nbx, rb_nby;  // record layout: brick edge 2^rb_log (0 or kBrickLog), bricks per row / column
+    uint32_t rb_ky, rb_kz;       // per-axis brick strides minus the shifted part (PT_REC_AFFINE)
+    uint32_t rb_off;             // margin offset of the voxel coordinates (RecLayout::off)
+    int pcx, pcy, pcz;           // cx + rb_off etc.: padded coordinates straight from the lookup
+    uint32_t nobounds;           // 1: the margin covers every candidate (step * max|v| < rb_off)
     int nx, ny, nz;
     int cx, cy, cz;              // floor(N/2) per axis
     float fcx, fcy, fcz;         // the same as floats
@@ -197,14 +202,21 @@ cudaError_t launch_label_max(const uint8_t* labels, int64_t V, unsigned long lon
 // Record layout (see rec_vox in pt_device.cuh): b = brick log2 edge, 0 (raster) or
 // kBrickLog (the default; the main tracking kernel is compiled for these two).
 constexpr uint32_t kBrickLog = 4;
+// PT_REC_MARGIN: bricked layouts get one brick of sentinel records on every side (the
+// voxel coordinates are offset by off = 2^b), so a candidate up to 2^b voxels outside the
+// volume reads a sentinel record: the bench instantiation needs no bounds test per step.
+#ifndef PT_REC_MARGIN
+#define PT_REC_MARGIN 0
+#endif
 struct RecLayout {
     uint32_t b, nbx, nby, nbz;
+    uint32_t off = 0;  // coordinate offset of the volume inside the brick grid (margin)
     uint64_t nvox() const { return (uint64_t)nbx * nby * nbz << (3u * b); }  // allocated voxels (padded)
 };
 RecLayout rec_layout(int nx, int ny, int nz, uint32_t b);
 cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask, uint8_t* rec,
                           int nx, int ny, int nz, const RecLayout& L, int S, int F, bool half, int rec_bytes,
-                          unsigned long long* bad, cudaStream_t st);
+                          unsigned long long* bad, unsigned long long* maxabs, cudaStream_t st);
 // Z-order processing permutation of the seeds: perm[k] = index of the k-th seed in Morton
 // order of its voxel (ties by input index; stable radix sort).  keys, keys_out, idx, perm:
 // device buffers of nseeds; temp: seed_order_temp_bytes(nseeds) bytes.
@@ -229,7 +241,7 @@ int gather_bench_blocks_per_sm(int rec_bytes);
 #define PT_RVKEYS 1  // 0: every instantiation keys the map by raster voxel (A/B switch)
 #endif
 inline bool track_rv_keys(const TrackArgs& a, const TrackMode& m, bool half) {
-    return PT_RVKEYS && !m.simple && !m.unique && !m.var && !m.out && !a.sample_mode &&
+    return PT_RVKEYS && (!PT_REC_MARGIN || a.nobounds) && !m.simple && !m.unique && !m.var && !m.out && !a.sample_mode &&
            !(half && !(a.fib_thr >= 0.f)) && a.rb_log == kBrickLog;
 }
 

@@ -24,7 +24,8 @@ template <bool HALF>
 __global__ void repack_kernel(const void* __restrict__ dyads, const void* __restrict__ fr,
                               const uint8_t* __restrict__ mask, uint8_t* __restrict__ rec,
                               int nx, int ny, int64_t V, RecLayout L, int S, int F, int RB,
-                              unsigned long long* bad) {
+                              unsigned long long* bad, unsigned long long* maxabs) {
+    float vmax = 0.f;  // largest |vector component| of this thread's records inside the mask
     const int64_t total = V * (int64_t)S;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
          i += (int64_t)gridDim.x * blockDim.x) {
@@ -61,8 +62,22 @@ __global__ void repack_kernel(const void* __restrict__ dyads, const void* __rest
             else w[3] = 0xFFFFFFFFu;
         } else if (!ok) {
             atomicAdd(bad, 1ull);
+        } else {
+            for (int j = 0; j < F; ++j) {
+                float c[3];
+                if (HALF) {
+                    c[0] = __half2float(__ushort_as_half((unsigned short)(w[2 * j] & 0xFFFFu)));
+                    c[1] = __half2float(__ushort_as_half((unsigned short)(w[2 * j] >> 16)));
+                    c[2] = __half2float(__ushort_as_half((unsigned short)(w[2 * j + 1] & 0xFFFFu)));
+                } else {
+                    c[0] = __uint_as_float(w[4 * j]);
+                    c[1] = __uint_as_float(w[4 * j + 1]);
+                    c[2] = __uint_as_float(w[4 * j + 2]);
+                }
+                for (int k = 0; k < 3; ++k) vmax = fmaxf(vmax, fabsf(c[k]));
+            }
         }
-        const uint64_t rv = rec_vox_raster((uint32_t)vox, (uint32_t)nx, (uint32_t)ny, L.b, L.nbx, L.nby);
+        const uint64_t rv = rec_vox_raster((uint32_t)vox, (uint32_t)nx, (uint32_t)ny, L.b, L.nbx, L.nby, L.off);
         uint8_t* out = rec + rec_slot((uint32_t)rv, (uint32_t)s, (uint32_t)S, L.b) * RB;
         if (RB == 8) {
             *reinterpret_cast<uint2*>(out) = make_uint2(w[0], w[1]);
@@ -71,6 +86,9 @@ __global__ void repack_kernel(const void* __restrict__ dyads, const void* __rest
                 reinterpret_cast<uint4*>(out)[k] = make_uint4(w[4 * k], w[4 * k + 1], w[4 * k + 2], w[4 * k + 3]);
         }
     }
+    // non-negative floats order like their bit patterns
+    const unsigned m = __reduce_max_sync(kFull, __float_as_uint(vmax));
+    if ((threadIdx.x & 31u) == 0u && m) atomicMax(maxabs, (unsigned long long)m);
 }
 
 // ------------------------------------------------------------------------- seed order
@@ -132,7 +150,7 @@ __global__ void map_sum_kernel(const uint32_t* __restrict__ map, int64_t V, unsi
 __global__ void map_unpermute_kernel(const uint32_t* __restrict__ pm, uint32_t mask, bool rvk, uint32_t nx,
                                      uint32_t ny, RecLayout L, uint32_t* __restrict__ map, int64_t V, bool acc) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < V; i += (int64_t)gridDim.x * blockDim.x) {
-        const uint32_t key = rvk ? rec_vox_raster((uint32_t)i, nx, ny, L.b, L.nbx, L.nby) : (uint32_t)i;
+        const uint32_t key = rvk ? rec_vox_raster((uint32_t)i, nx, ny, L.b, L.nbx, L.nby, L.off) : (uint32_t)i;
         const uint32_t c = pm[mask ? map_perm(key, mask) : key];
         map[i] = acc ? map[i] + c : c;
     }
@@ -231,21 +249,33 @@ RecLayout rec_layout(int nx, int ny, int nz, uint32_t b) {
     L.nbx = ((uint32_t)nx + e - 1u) >> b;
     L.nby = ((uint32_t)ny + e - 1u) >> b;
     L.nbz = ((uint32_t)nz + e - 1u) >> b;
+    if (PT_REC_MARGIN && b) {  // one brick of sentinels on every side
+        L.nbx += 2u;
+        L.nby += 2u;
+        L.nbz += 2u;
+        L.off = e;
+    }
     return L;
 }
 
 cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask, uint8_t* rec,
                           int nx, int ny, int nz, const RecLayout& L, int S, int F, bool half, int rec_bytes,
-                          unsigned long long* bad, cudaStream_t st) {
+                          unsigned long long* bad, unsigned long long* maxabs, cudaStream_t st) {
     const int64_t V = (int64_t)nx * ny * nz;
     const int64_t total = V * (int64_t)S;
+    // bricked layouts: the padding of ragged edge bricks (and the margin bricks) holds
+    // sentinel records (all-ones words: f0 = NaN pattern = outside the mask)
+    if (L.b) {
+        const cudaError_t e = cudaMemsetAsync(rec, 0xFF, (size_t)L.nvox() * (size_t)S * (size_t)rec_bytes, st);
+        if (e != cudaSuccess) return e;
+    }
     int64_t blocks = (total + 255) / 256;
     if (blocks > 148 * 64) blocks = 148 * 64;
     if (blocks < 1) blocks = 1;
     if (half)
-        repack_kernel<true><<<(unsigned)blocks, 256, 0, st>>>(dyads, f, mask, rec, nx, ny, V, L, S, F, rec_bytes, bad);
+        repack_kernel<true><<<(unsigned)blocks, 256, 0, st>>>(dyads, f, mask, rec, nx, ny, V, L, S, F, rec_bytes, bad, maxabs);
     else
-        repack_kernel<false><<<(unsigned)blocks, 256, 0, st>>>(dyads, f, mask, rec, nx, ny, V, L, S, F, rec_bytes, bad);
+        repack_kernel<false><<<(unsigned)blocks, 256, 0, st>>>(dyads, f, mask, rec, nx, ny, V, L, S, F, rec_bytes, bad, maxabs);
     return cudaGetLastError();
 }
 

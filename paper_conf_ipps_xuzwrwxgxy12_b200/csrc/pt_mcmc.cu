@@ -39,7 +39,7 @@ constexpr int kMaxShells = 8;             // distinct b-values handled with one 
 #define PT_MCMC_VPW 2  // voxels per warp for nmeas <= 64 (1: one voxel per warp always)
 #endif
 #ifndef PT_MCMC_MIN_BLOCKS
-#define PT_MCMC_MIN_BLOCKS 4  // CTAs per SM the register budget must allow (16 warps)
+#define PT_MCMC_MIN_BLOCKS 3  // CTAs per SM the register budget must allow (12 warps; 4 spills: -1.3 %, r02u)
 #endif
 
 #ifndef PT_MCMC_FMA

@@ -117,7 +117,7 @@ __global__ void __launch_bounds__(256) seg_kernel(const __grid_constant__ TrackA
             const uint32_t wn = r3 == 0 ? W.x : (r3 == 1 ? W.y : W.z);
             const uint32_t smp = a.sample_mode ? (uint32_t)((s.li[i] % a.P) % a.S) : sample_of(wn, a.S);
             R rv;
-            const uint32_t rvx = rec_vox_raster(vox, (uint32_t)a.nx, (uint32_t)a.ny, a.rb_log, a.rb_nbx, a.rb_nby);
+            const uint32_t rvx = rec_vox_raster(vox, (uint32_t)a.nx, (uint32_t)a.ny, a.rb_log, a.rb_nbx, a.rb_nby, a.rb_off);
             PT_BOUND(a, (uint64_t)rvx * a.S + smp < a.rec_n && smp < a.S);
             ldg_record<RB>(a.rec + rec_slot(rvx, smp, a.S, a.rb_log) * RB, rv.w);
             float vx, vy, vz, f0;

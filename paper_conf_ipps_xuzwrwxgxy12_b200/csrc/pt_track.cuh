@@ -39,6 +39,9 @@
 #include "pt_device.cuh"
 #include "pt_internal.h"
 
+#ifndef PT_REC_AFFINE
+#define PT_REC_AFFINE 0  // experiment: brick position of the bench layout as per-axis terms
+#endif
 #ifndef PT_RUNLEN
 #define PT_RUNLEN 1  // merge consecutive visits of a voxel before the RED (0: ablation iv, one RED per step)
 #endif
@@ -116,6 +119,9 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     // the bench instantiations key the map by the record voxel (track_rv_keys): no raster
     // voxel index on their path
     constexpr bool RVKEY = PT_RVKEYS && BL > 0 && !OUT && !UNQ && VM == 0 && REFILL;
+    // ... and with margin bricks (PT_REC_MARGIN; launched only when a.nobounds) skip the
+    // bounds test of every candidate
+    constexpr bool NOB = PT_REC_MARGIN && RVKEY;
     __shared__ unsigned long long s_li[OUT ? TPB : 1];  // particle index (outputs)
     __shared__ uint32_t s_q[TPB / 32][3];               // per-warp sub-chunk
     __shared__ unsigned long long s_work;               // CTA claim + tickets
@@ -176,14 +182,25 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     bool exhausted = false;  // warp-uniform
 
     // position of voxel (ix, iy, iz) = raster index v in the record volume (rec_vox)
-    auto recv = [&](int ix, int iy, int iz, uint32_t v) -> uint32_t {
-        if (BL == 0) return v;
-        if (BL < 0) return rec_vox(ix, iy, iz, a.rb_log, a.rb_nbx, a.rb_nby);
+    // (recv_p: the same from coordinates already offset by the layout's margin, BL > 0)
+    auto recv_p = [&](uint32_t ux, uint32_t uy, uint32_t uz) -> uint32_t {
         constexpr uint32_t b = BL > 0 ? (uint32_t)BL : 1u;
+#if PT_REC_AFFINE
+        // the same position as a sum of per-axis terms: u_a << (a b) plus (u_a >> b) times
+        // the brick stride minus the part of it the shift already counted (a.rb_k*)
+        return (ux + (ux >> b) * ((1u << (3 * b)) - (1u << b))) + ((uy << b) + (uy >> b) * a.rb_ky) +
+               ((uz << (2 * b)) + (uz >> b) * a.rb_kz);
+#else
         constexpr uint32_t m = (1u << b) - 1u;
-        const uint32_t ux = (uint32_t)ix, uy = (uint32_t)iy, uz = (uint32_t)iz;
         const uint32_t br = ((uz >> b) * a.rb_nby + (uy >> b)) * a.rb_nbx + (ux >> b);
         return (br << (3 * b)) | ((uz & m) << (2 * b)) | ((uy & m) << b) | (ux & m);
+#endif
+    };
+    auto recv = [&](int ix, int iy, int iz, uint32_t v) -> uint32_t {
+        if (BL == 0) return v;
+        if (BL < 0) return rec_vox(ix, iy, iz, a.rb_log, a.rb_nbx, a.rb_nby, a.rb_off);
+        const uint32_t o = PT_REC_MARGIN ? a.rb_off : 0u;
+        return recv_p((uint32_t)ix + o, (uint32_t)iy + o, (uint32_t)iz + o);
     };
     auto rec_at = [&](uint32_t rv, uint32_t s) -> const uint8_t* {
         return a.rec + rec_slot(rv, s, a.S, BL < 0 ? a.rb_log : (uint32_t)BL) * RB;
@@ -548,9 +565,14 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         const float nqx = __fadd_rn(x.qx, __fmul_rn(a.step, dx));
         const float nqy = __fadd_rn(x.qy, __fmul_rn(a.step, dy));
         const float nqz = __fadd_rn(x.qz, __fmul_rn(a.step, dz));
-        const int ix = axis_index(nqx, a.cx), iy = axis_index(nqy, a.cy), iz = axis_index(nqz, a.cz);
-        const bool inb = (unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny && (unsigned)iz < (unsigned)a.nz;
-        const uint32_t v = ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
+        // NOB: coordinates in the margin-padded brick grid straight from the lookup; a
+        // candidate outside the volume lands in a margin (or ragged) brick of sentinel records
+        // and is rejected by its gather like any voxel outside the mask (R11)
+        const int ix = axis_index(nqx, NOB ? a.pcx : a.cx), iy = axis_index(nqy, NOB ? a.pcy : a.cy),
+                  iz = axis_index(nqz, NOB ? a.pcz : a.cz);
+        const bool inb = NOB || ((unsigned)ix < (unsigned)a.nx && (unsigned)iy < (unsigned)a.ny && (unsigned)iz < (unsigned)a.nz);
+        const uint32_t v = NOB ? 0u : ((uint32_t)iz * (uint32_t)a.ny + (uint32_t)iy) * (uint32_t)a.nx + (uint32_t)ix;
+        const uint32_t crv = NOB ? recv_p((uint32_t)ix, (uint32_t)iy, (uint32_t)iz) : recv(ix, iy, iz, v);
         // stop criteria in order: maximum steps (R14), angle, volume (R11)
         const bool maxed = x.n == a.max_steps;
         const bool go = x.alive && !maxed && curv_ok && inb;
@@ -574,7 +596,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
             }
             const uint32_t w = ((k + 1) % 3 == 0) ? x.W.x : ((k + 1) % 3 == 1) ? x.W.y : x.W.z;
             const uint32_t sk = smode ? x.sfix : sample_of(w, a.S);
-            const uint32_t nrv = recv(ix, iy, iz, v);
+            const uint32_t nrv = crv;
             const bool outside = gather(go, nqx, nqy, nqz, nrv, v, (uint32_t)x.n + 1u, sk);
             x.why = outside ? kEndMask : x.why;
             x.alive = go && !outside;
@@ -582,7 +604,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
         } else {
             x.pend = go;  // next round's start gathers and tests it
             if (!RVKEY) x.gvox = go ? v : x.gvox;
-            x.grv = go ? recv(ix, iy, iz, v) : x.grv;
+            x.grv = go ? crv : x.grv;
         }
     };
 
