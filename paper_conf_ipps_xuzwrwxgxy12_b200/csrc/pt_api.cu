@@ -51,6 +51,7 @@ struct pt_ctx {
     float max_abs = 0.f;          // largest |vector component| inside the mask (margin test)
     uint8_t* d_rec = nullptr;
     size_t rec_size = 0;
+    uint64_t rec_payload = 0;     // V x S x record bytes (the size rules below use this, not the padded size)
     uint8_t* d_mask = nullptr;    // tracking mask copy (the variant kernel's interpolation)
     size_t mask_cap = 0;
     // per-call buffers
@@ -354,7 +355,10 @@ pt_status pt_load_samples(pt_ctx* c, const pt_volume* v, const void* dyads, cons
     if (blog != 0u && blog != pt::kBrickLog)
         return fail(c, PT_ERR_ARG, "pt_load_samples: PT_BRICK must be 0 (raster) or %u (16^3 bricks), got %u",
                     pt::kBrickLog, blog);
-    const pt::RecLayout L = pt::rec_layout(v->nx, v->ny, v->nz, blog);
+    // margin bricks (no per-step bounds test) only for volumes that stay "small"; a large
+    // volume (c5) keeps the unpadded bricks, whose extra map and record footprint would cost
+    const uint64_t payload = (uint64_t)V * (uint64_t)S * (uint64_t)rb;
+    const pt::RecLayout L = pt::rec_layout(v->nx, v->ny, v->nz, blog, payload <= PT_BIG_VOLUME);
     if (L.nvox() > 0xFFFFFFFFull) return fail(c, PT_ERR_ARG, "pt_load_samples: padded volume exceeds 2^32-1 voxels");
     const size_t rec_size = L.nvox() * S * (size_t)rb;
 
@@ -430,6 +434,7 @@ pt_status pt_load_samples(pt_ctx* c, const pt_volume* v, const void* dyads, cons
     c->vol = *v;
     c->rec_bytes = rb;
     c->layout = L;
+    c->rec_payload = payload;
     {
         const uint32_t mb = (uint32_t)maxabs;
         float m;
@@ -618,7 +623,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.chunks_per_seed = (uint32_t)((P + a.cta_chunk - 1) / a.cta_chunk);
     a.total_chunks = N * (uint64_t)a.chunks_per_seed;
     a.seeds_per_claim = 1;
-    uint64_t spc = c->rec_size > PT_BIG_VOLUME ? PT_SEEDS_PER_CLAIM_BIG : PT_SEEDS_PER_CLAIM;
+    uint64_t spc = c->rec_payload > PT_BIG_VOLUME ? PT_SEEDS_PER_CLAIM_BIG : PT_SEEDS_PER_CLAIM;
     if (const char* e = getenv("PT_SEEDS_PER_CLAIM")) spc = (uint64_t)atoll(e);  // experiments
     if (a.chunks_per_seed == 1 && spc > 1) {
         // whole seeds per claim: G consecutive seeds (tickets per claim must stay < 2^22)
@@ -707,7 +712,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.map_keys = rvk ? c->layout.nvox() : V;
     int perm = PT_MAP_PERM;
     if (const char* e = getenv("PT_MAP_PERM")) perm = atoi(e);  // experiments
-    const bool permuted = d_map && (perm == 2 || (perm == 1 && c->rec_size <= PT_BIG_VOLUME));
+    const bool permuted = d_map && (perm == 2 || (perm == 1 && c->rec_payload <= PT_BIG_VOLUME));
     const bool scratch = d_map && (permuted || rvk);
     uint32_t pmask = 0u;
     if (scratch) {

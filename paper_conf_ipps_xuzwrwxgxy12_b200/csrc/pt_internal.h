@@ -206,14 +206,14 @@ constexpr uint32_t kBrickLog = 4;
 // voxel coordinates are offset by off = 2^b), so a candidate up to 2^b voxels outside the
 // volume reads a sentinel record: the bench instantiation needs no bounds test per step.
 #ifndef PT_REC_MARGIN
-#define PT_REC_MARGIN 0
+#define PT_REC_MARGIN 1
 #endif
 struct RecLayout {
     uint32_t b, nbx, nby, nbz;
     uint32_t off = 0;  // coordinate offset of the volume inside the brick grid (margin)
     uint64_t nvox() const { return (uint64_t)nbx * nby * nbz << (3u * b); }  // allocated voxels (padded)
 };
-RecLayout rec_layout(int nx, int ny, int nz, uint32_t b);
+RecLayout rec_layout(int nx, int ny, int nz, uint32_t b, bool margin);
 cudaError_t launch_repack(const void* dyads, const void* f, const uint8_t* mask, uint8_t* rec,
                           int nx, int ny, int nz, const RecLayout& L, int S, int F, bool half, int rec_bytes,
                           unsigned long long* bad, unsigned long long* maxabs, cudaStream_t st);
@@ -241,7 +241,7 @@ int gather_bench_blocks_per_sm(int rec_bytes);
 #define PT_RVKEYS 1  // 0: every instantiation keys the map by raster voxel (A/B switch)
 #endif
 inline bool track_rv_keys(const TrackArgs& a, const TrackMode& m, bool half) {
-    return PT_RVKEYS && (!PT_REC_MARGIN || a.nobounds) && !m.simple && !m.unique && !m.var && !m.out && !a.sample_mode &&
+    return PT_RVKEYS && !m.simple && !m.unique && !m.var && !m.out && !a.sample_mode &&
            !(half && !(a.fib_thr >= 0.f)) && a.rb_log == kBrickLog;
 }
 

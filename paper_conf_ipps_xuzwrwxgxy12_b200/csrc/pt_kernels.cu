@@ -242,14 +242,14 @@ cudaError_t launch_track(const TrackArgs& a, const TrackMode& m, int nfibres, bo
     }
 }
 
-RecLayout rec_layout(int nx, int ny, int nz, uint32_t b) {
+RecLayout rec_layout(int nx, int ny, int nz, uint32_t b, bool margin) {
     RecLayout L;
     const uint32_t e = 1u << b;
     L.b = b;
     L.nbx = ((uint32_t)nx + e - 1u) >> b;
     L.nby = ((uint32_t)ny + e - 1u) >> b;
     L.nbz = ((uint32_t)nz + e - 1u) >> b;
-    if (PT_REC_MARGIN && b) {  // one brick of sentinels on every side
+    if (PT_REC_MARGIN && margin && b) {  // one brick of sentinels on every side
         L.nbx += 2u;
         L.nby += 2u;
         L.nbz += 2u;

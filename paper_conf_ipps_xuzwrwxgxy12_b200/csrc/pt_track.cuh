@@ -40,7 +40,7 @@
 #include "pt_internal.h"
 
 #ifndef PT_REC_AFFINE
-#define PT_REC_AFFINE 0  // experiment: brick position of the bench layout as per-axis terms
+#define PT_REC_AFFINE 1  // brick position of the bench layout as per-axis terms (0: the bit-field form)
 #endif
 #ifndef PT_RUNLEN
 #define PT_RUNLEN 1  // merge consecutive visits of a voxel before the RED (0: ablation iv, one RED per step)
@@ -107,7 +107,7 @@ __host__ __device__ constexpr int track_tpb() {
     return REFILL ? (((VM & (kVarInterp | kVarInit)) != 0 || UNQ) ? kThreadsExt : kThreads) : kSimpleThreads;
 }
 
-template <int F, bool HALF, bool REFILL, bool OUT, int BL, int VM, bool UNQ>
+template <int F, bool HALF, bool REFILL, bool OUT, int BL, int VM, bool UNQ, bool NB = false>
 __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(const __grid_constant__ TrackArgs a) {
     using R = Rec<F, HALF>;
     using L = Lane<F, HALF, UNQ>;
@@ -121,7 +121,7 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     constexpr bool RVKEY = PT_RVKEYS && BL > 0 && !OUT && !UNQ && VM == 0 && REFILL;
     // ... and with margin bricks (PT_REC_MARGIN; launched only when a.nobounds) skip the
     // bounds test of every candidate
-    constexpr bool NOB = PT_REC_MARGIN && RVKEY;
+    constexpr bool NOB = PT_REC_MARGIN && RVKEY && NB;
     __shared__ unsigned long long s_li[OUT ? TPB : 1];  // particle index (outputs)
     __shared__ uint32_t s_q[TPB / 32][3];               // per-warp sub-chunk
     __shared__ unsigned long long s_work;               // CTA claim + tickets
@@ -716,9 +716,9 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
 
 // grid of one launch: persistent (at most #SMs x resident CTAs, or fewer when the job or the
 // UNQ hash sets are smaller) or one thread per particle
-template <int F, bool HALF, bool REFILL, bool OUT, int BL, int VM, bool UNQ>
+template <int F, bool HALF, bool REFILL, bool OUT, int BL, int VM, bool UNQ, bool NB = false>
 cudaError_t launch_track_kernel(const TrackArgs& a, int num_sms, cudaStream_t st) {
-    auto k = track_kernel<F, HALF, REFILL, OUT, BL, VM, UNQ>;
+    auto k = track_kernel<F, HALF, REFILL, OUT, BL, VM, UNQ, NB>;
     constexpr int TPB = track_tpb<REFILL, VM, UNQ>();
     if (a.nparticles == 0) return cudaSuccess;
     unsigned grid;
@@ -775,7 +775,11 @@ cudaError_t launch_track_fh(const TrackArgs& a, const TrackMode& m, int num_sms,
     // the bench path: record layout as a compile-time constant, random sample per step
     // (the compile-time layouts compare fp16 f bits as integers: fib_thr >= 0 only)
     // (track_rv_keys: exactly the kBrickLog instantiation keys the map by record voxel)
-    if (track_rv_keys(a, m, HALF)) return launch_track_kernel<F, HALF, true, false, (int)kBrickLog, 0, false>(a, num_sms, st);
+    if (track_rv_keys(a, m, HALF)) {  // with margin bricks covering every candidate: no bounds test
+        if (PT_REC_MARGIN && a.nobounds)
+            return launch_track_kernel<F, HALF, true, false, (int)kBrickLog, 0, false, true>(a, num_sms, st);
+        return launch_track_kernel<F, HALF, true, false, (int)kBrickLog, 0, false>(a, num_sms, st);
+    }
     if (HALF && !(a.fib_thr >= 0.f)) return launch_track_kernel<F, HALF, true, false, -1, 0, false>(a, num_sms, st);
     if (a.rb_log == 0) return launch_track_kernel<F, HALF, true, false, 0, 0, false>(a, num_sms, st);
     if (a.rb_log == kBrickLog) return launch_track_kernel<F, HALF, true, false, (int)kBrickLog, 0, false>(a, num_sms, st);

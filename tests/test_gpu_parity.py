@@ -193,6 +193,35 @@ def test_timed_instantiation_map_vs_oracle(pt, tracker, cfg):
     assert st["particles"] == w.nparticles
 
 
+@pytest.mark.parametrize("step", [0.5, 7.9, 14.5, 15.5, 40.0])
+@pytest.mark.parametrize("half", [False, True])
+def test_margin_bricks_and_bounds(pt, tracker, step, half):
+    """The bench launch on the margin-padded brick layout: while step * max|v| <
+    15 voxels the kernel takes no bounds test and leaving the volume is caught by the
+    sentinel records of the margin / ragged bricks; above that the bounds-checked
+    instantiation runs.  Large steps make particles leave the volume on every side, from
+    ragged (non-multiple-of-16) edges: the map and the step counter must equal the oracle's."""
+    import torch
+    w = phantom.crossing(nx=45, ny=37, nz=21, lo=10, hi=30, zlo=3, zhi=18, sigma=0.4, f_jitter=0.05,
+                         nseeds=96, particles_per_seed=64, nsamples=12)
+    w = w.replace(step=step, max_steps=400)
+    if half:
+        w = phantom.to_half(w)
+    tracker.load_volume(w.volume)
+    m = tracker.track_workload(w, flags=0)
+    torch.cuda.synchronize()
+    st = tracker.stats()
+    gm = m.cpu().numpy().view(np.uint32)
+    r = oracle.track(w, want_particles=False)
+    assert np.array_equal(gm.astype(np.uint64), r["map"]), \
+        f"{np.count_nonzero(gm.astype(np.uint64) != r['map'])} map cells differ"
+    assert st["total_steps"] == int(r["map"].sum())
+    # and per particle through the outputs instantiation (bounds-checked, runtime layout)
+    g = gpu_run(tracker, w)
+    ro = oracle.track(w)
+    assert_parity(g, ro)
+
+
 @pytest.mark.parametrize("cfg", ["c2", "c2_dispersed"])
 def test_timed_instantiation_full_config(pt, tracker, cfg):
     """configs[1] in the bench launch (flags = 0): the full map bit-exact vs the oracle."""
