@@ -120,7 +120,10 @@ typedef struct {
  * raster order; any other value is PT_ERR_ARG), so the records of a 3-D neighbourhood
  * are contiguous.
  * The layout is internal: it changes no result, only the padded device footprint
- * (ceil(n/2^b)*2^b per axis x S x record bytes).
+ * (ceil(n/2^b)*2^b per axis x S x record bytes; for volumes of <= 4 GB of records, one
+ * more brick of sentinel records on every side of every axis, so that the tracking
+ * kernel needs no bounds test per step; the largest |vector component| is recorded for
+ * that bound).
  *   dyads: [F][S][nz][ny][nx][3] (x fastest, xyz innermost), float32 or binary16 bits
  *   f    : [F][S][nz][ny][nx], same dtype
  *   mask : [nz][ny][nx] uint8, != 0 inside
@@ -156,6 +159,10 @@ typedef struct {
  *              the order of the seeds.
  *   map      : [nz][ny][nx] uint32 visitation counts (one per committed step at the new
  *              voxel, R13), zeroed first unless PT_MAP_ACCUMULATE; may be NULL.
+ * The kernels count into a context-owned scratch map (a permuted and/or record-ordered
+ * copy: one uint32 per padded record voxel, rounded up to a power of two when permuted)
+ * that pt_track adds into `map` after the kernel;
+ * `map` itself always receives raster-ordered counts.
  * With device pointers the call is asynchronous on ctx's stream; a host `map` makes it
  * synchronous (device map, then a device-to-host copy).  Per-particle outputs selected
  * by flags stay on the device until pt_get_paths.  Errors: PT_ERR_STATE before
