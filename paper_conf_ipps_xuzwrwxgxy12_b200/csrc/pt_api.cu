@@ -18,15 +18,21 @@
 
 #ifndef PT_SEEDS_PER_CLAIM
 // Whole seeds per CTA claim when every seed fits one claim: a CTA walks G consecutive
-// (Morton-adjacent) seeds, so its L1 keeps serving the shared tract voxels (sweep 1..64:
-// c3 74.6/75.3/76.0/76.4/77.0/77.2/76.9 G steps/s; G = 32 for c3 / c4).  With a record volume
-// far beyond L2 (c5: 7.2 GB) the chip-wide span of in-flight seeds (#SMs x G) decides the
-// L2 working set instead: G = 1 / 4 / 8 / 32 give c5 94.3 / 96.8 / 94.8 / 88.5 G
-// (profiles/r02h_c5_claims_ab.log), so above PT_BIG_VOLUME bytes of records G is 4.
-#define PT_SEEDS_PER_CLAIM 32
+// (Morton-adjacent) seeds, so its L1 keeps serving the shared tract voxels, while the
+// chip-wide span of in-flight seeds (#SMs x G) sets the L2 working set.  Round 1 (raster
+// map) preferred G = 32 on c3 / c4 (sweep 1..64: 74.6 ... 77.2 G); once the map REDs were
+// spread over the L2 slices (permuted scratch map, r02n) the L2 side dominates: G = 1 / 2 /
+// 4 / 8 / 16 / 32 give c3 161.9 / 163.7 / 163.5 / 161.1 / 155.4 / 146.8 G, c4 (half the
+// record bytes) peaks at G = 8-12 (185.5-186.2 G), c5 at 4 (97.9 G)
+// (profiles/r02y_claims_ab.log, r02z_claims_sweep.log, r02aa_claims_small.log): G = 8 for
+// record payloads up to PT_SMALL_VOLUME bytes, else 4.
+#define PT_SEEDS_PER_CLAIM 8
 #endif
 #ifndef PT_SEEDS_PER_CLAIM_BIG
 #define PT_SEEDS_PER_CLAIM_BIG 4
+#endif
+#ifndef PT_SMALL_VOLUME
+#define PT_SMALL_VOLUME (1ull << 30)
 #endif
 #ifndef PT_BIG_VOLUME
 #define PT_BIG_VOLUME (4ull << 30)
@@ -623,7 +629,7 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
     a.chunks_per_seed = (uint32_t)((P + a.cta_chunk - 1) / a.cta_chunk);
     a.total_chunks = N * (uint64_t)a.chunks_per_seed;
     a.seeds_per_claim = 1;
-    uint64_t spc = c->rec_payload > PT_BIG_VOLUME ? PT_SEEDS_PER_CLAIM_BIG : PT_SEEDS_PER_CLAIM;
+    uint64_t spc = c->rec_payload > PT_SMALL_VOLUME ? PT_SEEDS_PER_CLAIM_BIG : PT_SEEDS_PER_CLAIM;
     if (const char* e = getenv("PT_SEEDS_PER_CLAIM")) spc = (uint64_t)atoll(e);  // experiments
     if (a.chunks_per_seed == 1 && spc > 1) {
         // whole seeds per claim: G consecutive seeds (tickets per claim must stay < 2^22)
