@@ -733,6 +733,8 @@ pt_status pt_track(pt_ctx* c, const float* seeds_xyz, const uint64_t* seed_ids, 
         a.map = c->d_pmap;
     }
     a.map_mask = pmask;
+    // the no-bounds instantiation also takes the permuted map as given (pt_track.cuh, NOB)
+    if (!permuted) a.nobounds = 0u;
     // experiment (env PT_MAP_PERSIST=1): the map as a persisting L2 access-policy window
     const bool persist = d_map && getenv("PT_MAP_PERSIST") && atoi(getenv("PT_MAP_PERSIST")) > 0;
     if (persist) {

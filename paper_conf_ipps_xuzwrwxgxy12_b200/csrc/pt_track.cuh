@@ -247,7 +247,8 @@ __global__ void __launch_bounds__(track_tpb<REFILL, VM, UNQ>(), 1) track_kernel(
     // a run of visits of one voxel: one predicated RED
     auto red_run = [&](bool p, uint32_t vox, uint32_t cnt) {
         if (p) PT_BOUND(a, vox < a.map_keys);
-        red_add_if(p, map + map_cell(a, vox), cnt);
+        // (the NOB instantiation is launched only with a permuted scratch map: no select)
+        red_add_if(p, map + (NOB ? map_perm(vox, a.map_mask) : map_cell(a, vox)), cnt);
     };
     auto flush_run = [&]() {
         if (!UNQ && has_map) red_run(x.run_cnt != 0u, x.run_vox, x.run_cnt);
